@@ -1,0 +1,327 @@
+// Context, device graph residency, page partitioning (Strategy-P / -S), NCCL.
+//
+// Paper: Alg 1 lines 2-3 create streams and device buffers per GPU;
+// Strategy-P copies a different set of pages to each GPU with h(j) = j mod N
+// (P:346-354), Strategy-S gives each GPU a different WA chunk.
+// B200: one process per GPU (torchrun), one context per process; NCCL comm
+// from a unique id broadcast by the caller's process group.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+#include <new>
+
+#include "runtime.h"
+
+namespace gts {
+
+std::pair<cudaEvent_t, cudaEvent_t> Timer::next() {
+    if (used == pairs.size()) {
+        cudaEvent_t a, b;
+        cudaEventCreate(&a);
+        cudaEventCreate(&b);
+        pairs.emplace_back(a, b);
+    }
+    return pairs[used++];
+}
+
+double Timer::sum_s() {
+    double s = 0;
+    for (size_t i = 0; i < used; ++i) {
+        float ms = 0;
+        if (cudaEventElapsedTime(&ms, pairs[i].first, pairs[i].second) == cudaSuccess) s += ms * 1e-3;
+    }
+    used = 0;
+    return s;
+}
+
+int Context::buf(int slot, size_t bytes, void** out) {
+    if ((size_t)slot >= scratch.size()) scratch.resize(slot + 1, {nullptr, 0});
+    auto& b = scratch[slot];
+    if (b.second < bytes) {
+        if (b.first) cudaFree(b.first);
+        b.first = nullptr;
+        b.second = 0;
+        size_t sz = bytes < 256 ? 256 : bytes;
+        cudaError_t e = cudaMalloc(&b.first, sz);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(GTS_ENOMEM, "cudaMalloc(%zu) for scratch slot %d: %s", sz, slot, cudaGetErrorString(e));
+        }
+        b.second = sz;
+    }
+    *out = b.first;
+    return GTS_OK;
+}
+
+void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t>& owner,
+               std::vector<uint64_t>& vrange) {
+    const uint64_t P = g->num_pages;
+    owner.assign(P, 0);
+    vrange.assign(world + 1, g->n);
+    vrange[0] = 0;
+    if (world <= 1) return;
+    if (strategy == GTS_STRATEGY_P) {
+        for (uint64_t j = 0; j < P; ++j) owner[j] = (int32_t)(j % (uint64_t)world);   // h(j) = j mod N
+        return;
+    }
+    // Strategy-S: contiguous VID ranges cut at page boundaries (never inside an
+    // LP run) with ~equal page counts; rank r owns WA[vrange[r], vrange[r+1]).
+    uint64_t p = 0;
+    for (int r = 0; r < world; ++r) {
+        uint64_t target = (P * (uint64_t)(r + 1)) / (uint64_t)world;
+        if (r == world - 1) target = P;
+        uint64_t first = p;
+        while (p < target || (p < P && p > 0 && g->kind[p] == GTS_PAGE_LP && g->lp_first[p] != (int64_t)p)) {
+            owner[p] = r;
+            ++p;
+        }
+        vrange[r] = first < P ? g->start_vid[first] : g->n;
+        if (r == 0) vrange[0] = 0;
+    }
+    // ranks left without pages own an empty range at the end
+    for (int r = 1; r <= world; ++r) vrange[r] = std::max(vrange[r], vrange[r - 1]);
+    vrange[world] = g->n;
+}
+
+int pinned_register(Graph* g) {
+    if (g->host_registered || g->pages_alloc == 0) return GTS_OK;
+    cudaError_t e = cudaHostRegister(g->pages, (g->pages_alloc + 4095) & ~(size_t)4095, cudaHostRegisterPortable);
+    if (e != cudaSuccess) {
+        cudaGetLastError();   // pageable fallback for the copy source is still correct, only slower
+        return GTS_OK;
+    }
+    g->host_registered = true;
+    return GTS_OK;
+}
+
+static void free_devgraph(DevGraph& d) {
+    cudaFree(d.pages);
+    cudaFree(d.rvt_start);
+    cudaFree(d.nslots);
+    cudaFree(d.loc);
+    cudaFree(d.local_list);
+    cudaFree(d.hot_keys);
+    d = DevGraph();
+}
+
+int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resident, double* upload_s) {
+    Graph* g = const_cast<Graph*>(gc);
+    double t0 = now_s();
+    uint32_t strat_key = c->world > 1 ? strategy : 0;
+    if (c->dg.uid != g->uid || c->dg.strategy != strat_key || c->dg.world != c->world) {
+        free_devgraph(c->dg);
+        DevGraph& d = c->dg;
+        d.uid = g->uid;
+        d.strategy = strat_key;
+        d.world = c->world;
+        std::vector<uint64_t> vrange;
+        partition(g, strategy, c->world, d.h_owner, vrange);
+        d.vlo = vrange[c->rank];
+        d.vhi = vrange[c->rank + 1];
+        const uint64_t P = g->num_pages;
+        std::vector<uint32_t> loc(P, UINT32_MAX);
+        d.h_local_list.clear();
+        for (uint64_t j = 0; j < P; ++j)
+            if (d.h_owner[j] == c->rank) {
+                loc[j] = (uint32_t)d.h_local_list.size();
+                d.h_local_list.push_back((uint32_t)j);
+            }
+        d.n_local = (uint32_t)d.h_local_list.size();
+        d.all_local = d.n_local == P;
+        GTS_CUDA(cudaMalloc(&d.rvt_start, std::max<size_t>(P, 1) * 4));
+        GTS_CUDA(cudaMalloc(&d.nslots, std::max<size_t>(P, 1) * 4));
+        GTS_CUDA(cudaMalloc(&d.loc, std::max<size_t>(P, 1) * 4));
+        GTS_CUDA(cudaMalloc(&d.local_list, std::max<size_t>(d.n_local, 1) * 4));
+        GTS_CUDA(cudaMalloc(&d.hot_keys, kHotSlots * 4));
+        GTS_CUDA(cudaMemcpyAsync(d.rvt_start, g->start_vid.data(), P * 4, cudaMemcpyHostToDevice, c->stream));
+        GTS_CUDA(cudaMemcpyAsync(d.nslots, g->nslots.data(), P * 4, cudaMemcpyHostToDevice, c->stream));
+        GTS_CUDA(cudaMemcpyAsync(d.loc, loc.data(), P * 4, cudaMemcpyHostToDevice, c->stream));
+        if (d.n_local)
+            GTS_CUDA(cudaMemcpyAsync(d.local_list, d.h_local_list.data(), d.n_local * 4ull, cudaMemcpyHostToDevice,
+                                     c->stream));
+        GTS_CUDA(cudaMemcpyAsync(d.hot_keys, g->hot_keys.data(), kHotSlots * 4, cudaMemcpyHostToDevice, c->stream));
+        GTS_CUDA(cudaStreamSynchronize(c->stream));   // host vectors above are temporaries
+    }
+    DevGraph& d = c->dg;
+    if (need_resident && !d.resident) {
+        GTS_TRY(pinned_register(g));
+        const size_t pb = g->page_bytes;
+        d.pages_bytes = (size_t)d.n_local * pb;
+        cudaError_t e = cudaMalloc(&d.pages, std::max<size_t>(d.pages_bytes, 256));
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(GTS_ENOMEM, "resident pages: cudaMalloc(%zu) failed: %s", d.pages_bytes,
+                        cudaGetErrorString(e));
+        }
+        // copy runs of consecutive local pages in one cudaMemcpyAsync each
+        uint32_t i = 0;
+        while (i < d.n_local) {
+            uint32_t j = i + 1;
+            while (j < d.n_local && d.h_local_list[j] == d.h_local_list[j - 1] + 1) ++j;
+            GTS_CUDA(cudaMemcpyAsync(d.pages + (size_t)i * pb, g->pages + (size_t)d.h_local_list[i] * pb,
+                                     (size_t)(j - i) * pb, cudaMemcpyHostToDevice, c->stream));
+            i = j;
+        }
+        GTS_CUDA(cudaStreamSynchronize(c->stream));
+        d.resident = true;
+        if (upload_s) *upload_s = now_s() - t0;
+    }
+    return GTS_OK;
+}
+
+int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* cfg, gts_run_config* out) {
+    if (!ctx || !g) return fail(GTS_EINVAL, "NULL context or graph");
+    gts_run_config d;
+    std::memset(&d, 0, sizeof(d));
+    d.struct_size = sizeof(d);
+    d.strategy = GTS_STRATEGY_P;
+    d.residency = GTS_RESIDENCY_AUTO;
+    if (cfg) {
+        if (cfg->struct_size && cfg->struct_size < sizeof(gts_run_config))
+            return fail(GTS_EINVAL, "gts_run_config.struct_size too small");
+        d = *cfg;
+    }
+    if (d.strategy > GTS_STRATEGY_S) return fail(GTS_EINVAL, "unknown strategy %u", d.strategy);
+    if (d.residency > GTS_STREAMED) return fail(GTS_EINVAL, "unknown residency %u", d.residency);
+    if (d.out_location > GTS_OUT_DEVICE) return fail(GTS_EINVAL, "unknown out_location %u", d.out_location);
+    if (d.ring_slots == 0) d.ring_slots = 4;
+    if (d.batch_pages == 0) d.batch_pages = 8;
+    if (d.ring_slots > 32) return fail(GTS_EINVAL, "ring_slots must be <= 32");
+    *out = d;
+    cudaError_t e = cudaSetDevice(ctx->device);
+    if (e != cudaSuccess) return fail(GTS_ECUDA, "cudaSetDevice(%d): %s", ctx->device, cudaGetErrorString(e));
+    return GTS_OK;
+}
+
+int copy_out(Context* c, const void* dsrc, void* dst, size_t bytes, uint32_t out_location) {
+    if (bytes == 0) return GTS_OK;
+    GTS_CUDA(cudaMemcpyAsync(dst, dsrc, bytes,
+                             out_location == GTS_OUT_DEVICE ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                             c->stream));
+    GTS_CUDA(cudaStreamSynchronize(c->stream));
+    return GTS_OK;
+}
+
+int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid) {
+    int per_sm = 0;
+    GTS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem));
+    if (per_sm < 1) per_sm = 1;
+    *grid = per_sm * c->num_sms;
+    return GTS_OK;
+}
+
+}  // namespace gts
+
+using namespace gts;
+
+extern "C" int gts_get_unique_id(uint8_t out[128]) {
+    clear_error();
+    if (!out) return fail(GTS_EINVAL, "NULL out");
+    ncclUniqueId id;
+    GTS_NCCL(ncclGetUniqueId(&id));
+    static_assert(sizeof(id) == 128, "ncclUniqueId is 128 bytes");
+    std::memcpy(out, &id, 128);
+    return GTS_OK;
+}
+
+extern "C" int gts_context_create(int device, int rank, int world_size, const uint8_t* unique_id,
+                                  gts_context** out) {
+    clear_error();
+    if (!out) return fail(GTS_EINVAL, "NULL out");
+    *out = nullptr;
+    if (world_size < 1 || rank < 0 || rank >= world_size) return fail(GTS_EINVAL, "bad rank/world_size");
+    if (world_size > 1 && !unique_id) return fail(GTS_EINVAL, "world_size > 1 needs an NCCL unique id");
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return fail(GTS_ECUDA, "no CUDA device available (%s); libgts has no CPU fallback",
+                    cudaGetErrorString(e));
+    }
+    if (device < 0 || device >= ndev) return fail(GTS_EINVAL, "device %d out of range (%d devices)", device, ndev);
+    GTS_CUDA(cudaSetDevice(device));
+    gts_context* c = new (std::nothrow) gts_context();
+    if (!c) return fail(GTS_ENOMEM, "context alloc");
+    c->device = device;
+    c->rank = rank;
+    c->world = world_size;
+    cudaDeviceProp prop;
+    GTS_CUDA(cudaGetDeviceProperties(&prop, device));
+    c->num_sms = prop.multiProcessorCount;
+    GTS_CUDA(cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking));
+    GTS_CUDA(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+    c->stream = c->own_stream;
+    GTS_CUDA(cudaMallocHost(&c->h_small, 4096));
+    if (world_size > 1) {
+        ncclUniqueId id;
+        std::memcpy(&id, unique_id, sizeof(id));
+        ncclResult_t r = ncclCommInitRank(&c->comm, world_size, id, rank);
+        if (r != ncclSuccess) {
+            delete c;
+            return fail(GTS_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+        }
+    }
+    *out = c;
+    return GTS_OK;
+}
+
+extern "C" void gts_context_free(gts_context* c) {
+    if (!c) return;
+    cudaSetDevice(c->device);
+    cudaDeviceSynchronize();
+    free_devgraph(c->dg);
+    for (auto& b : c->scratch) cudaFree(b.first);
+    for (Timer* t : {&c->t_main, &c->t_finish, &c->t_merge, &c->t_h2d})
+        for (auto& p : t->pairs) {
+            cudaEventDestroy(p.first);
+            cudaEventDestroy(p.second);
+        }
+    if (c->ring_events)
+        for (int i = 0; i < 64; ++i) {
+            cudaEventDestroy(c->ring_ready[i]);
+            cudaEventDestroy(c->ring_free[i]);
+        }
+    if (c->comm) ncclCommDestroy(c->comm);
+    cudaFreeHost(c->h_small);
+    cudaStreamDestroy(c->own_stream);
+    cudaStreamDestroy(c->copy_stream);
+    delete c;
+}
+
+extern "C" int gts_context_evict(gts_context* c, const gts_graph* g) {
+    clear_error();
+    if (!c) return fail(GTS_EINVAL, "NULL context");
+    cudaSetDevice(c->device);
+    cudaStreamSynchronize(c->stream);
+    if (!g || c->dg.uid == g->uid) free_devgraph(c->dg);
+    return GTS_OK;
+}
+
+extern "C" int gts_context_set_stream(gts_context* c, void* s) {
+    clear_error();
+    if (!c) return fail(GTS_EINVAL, "NULL context");
+    c->stream = s ? (cudaStream_t)s : c->own_stream;
+    return GTS_OK;
+}
+
+extern "C" void gts_graph_free(gts_graph* g) {
+    if (!g) return;
+    if (g->host_registered) cudaHostUnregister(g->pages);
+    std::free(g->pages);
+    delete g;
+}
+
+extern "C" int gts_partition_pages(const gts_graph* g, uint32_t strategy, int world_size, int32_t* owner,
+                                   uint64_t* vrange) {
+    clear_error();
+    if (!g || !owner || world_size < 1) return fail(GTS_EINVAL, "bad argument");
+    if (strategy > GTS_STRATEGY_S) return fail(GTS_EINVAL, "unknown strategy");
+    std::vector<int32_t> o;
+    std::vector<uint64_t> vr;
+    partition(g, strategy, world_size, o, vr);
+    std::memcpy(owner, o.data(), o.size() * 4);
+    if (vrange) std::memcpy(vrange, vr.data(), vr.size() * 8);
+    return GTS_OK;
+}

@@ -1,0 +1,176 @@
+// Generic page expansion for sm_100a: one CTA per slotted page at a time
+// (persistent grid, dynamic page queue), shared by BFS, SSSP, PageRank, WCC.
+//
+// Paper: K_SP / K_LP (Alg 2-5) assign one warp per vertex of an
+// SP (VWC) and one thread per ADJLIST entry of an LP.  B200 design
+// (DESIGN.md "Kernels"): a CTA takes a whole page; an SP is processed in tiles
+// of kTile consecutive slots: the tile's selected vertices (frontier test, or
+// all for PageRank-like sweeps) are compacted with __ballot_sync/__popc, their
+// degrees prefix-summed, and the tile's edges are then expanded edge-parallel
+// (4 consecutive edges per thread, one binary search per 4 edges), so a
+// degree-13 K vertex and a run of degree-1 vertices are balanced alike.  An LP
+// is swept by the whole CTA; a huge vertex spans several LPs and so several
+// CTAs (high-degree split).
+#pragma once
+
+#include <cstdint>
+
+#include "runtime.h"
+
+namespace gts {
+
+constexpr int kThreads = 512;
+constexpr int kTile = 512;
+constexpr int kEdgesPerThread = 4;
+constexpr int kWarps = kThreads / 32;
+
+__device__ __forceinline__ uint32_t ld32(const uint8_t* p) { return __ldg(reinterpret_cast<const uint32_t*>(p)); }
+
+__device__ __forceinline__ void page_at(const PageSet& ps, uint32_t i, uint32_t& pid, const uint8_t*& data) {
+    pid = ps.list ? __ldg(ps.list + i) : i;
+    uint64_t di = ps.mode == kAddrByPid ? pid : (ps.mode == kAddrByLoc ? __ldg(ps.loc + pid) : i);
+    data = ps.base + di * (uint64_t)ps.page_bytes;
+}
+
+// ADJLIST entry -> VID (App A: VID = RVT[ADJ_PID].START_VID + ADJ_OFF)
+__device__ __forceinline__ uint32_t decode_entry(const PageSet& ps, uint32_t e) {
+    return ps.entry_encoding == GTS_ENTRY_VID32 ? e : __ldg(ps.rvt_start + (e >> 16)) + (e & 0xFFFFu);
+}
+
+__device__ __forceinline__ bool test_bit(const uint32_t* bm, uint32_t v) {
+    return (__ldg(bm + (v >> 5)) >> (v & 31)) & 1u;
+}
+
+struct TileSmem {
+    uint32_t off[kTile];       // word index of the first ADJLIST entry of item j
+    uint32_t deg[kTile];
+    uint32_t src[kTile];       // VID of item j
+    uint32_t payload[kTile];
+    uint32_t pre[kTile + 1];   // exclusive prefix of deg over items
+    uint32_t wsum[kWarps];
+    uint32_t wcnt[kWarps];
+    uint32_t item;
+};
+
+// Tile scan: frontier compaction by __ballot_sync/__popc (position of each
+// selected vertex among the tile's selected vertices) fused with the exclusive
+// prefix sum of the selected vertices' degrees.  Two __syncthreads.
+__device__ __forceinline__ void tile_scan(bool sel, uint32_t deg, uint32_t& pos, uint32_t& nf,
+                                          uint32_t& deg_excl, uint32_t& deg_total, TileSmem& sm) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t mask = __ballot_sync(0xFFFFFFFFu, sel);
+    const uint32_t rank_in_warp = __popc(mask & ((1u << lane) - 1u));
+    uint32_t x = deg;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) {
+        sm.wsum[warp] = x;
+        sm.wcnt[warp] = __popc(mask);
+    }
+    __syncthreads();
+    if (warp == 0) {
+        uint32_t s = lane < kWarps ? sm.wsum[lane] : 0u;
+        uint32_t c = lane < kWarps ? sm.wcnt[lane] : 0u;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint32_t y = __shfl_up_sync(0xFFFFFFFFu, s, o);
+            uint32_t z = __shfl_up_sync(0xFFFFFFFFu, c, o);
+            if (lane >= o) { s += y; c += z; }
+        }
+        if (lane < kWarps) { sm.wsum[lane] = s; sm.wcnt[lane] = c; }   // inclusive warp prefixes
+    }
+    __syncthreads();
+    deg_excl = (warp > 0 ? sm.wsum[warp - 1] : 0u) + x - deg;
+    deg_total = sm.wsum[kWarps - 1];
+    pos = (warp > 0 ? sm.wcnt[warp - 1] : 0u) + rank_in_warp;
+    nf = sm.wcnt[kWarps - 1];
+}
+
+// Op interface:
+//   static constexpr bool kReadWeights;
+//   bool select(uint32_t vid)                            -- SP vertex expanded?
+//   uint32_t payload(uint32_t vid, uint32_t deg)         -- per selected vertex
+//   bool select_lp(uint32_t vid, uint32_t total_deg, uint32_t chunk_len, uint32_t& payload)
+//   void edge(uint32_t dst, uint32_t w, uint32_t payload, uint32_t src)
+//   void end_page()
+template <class Op>
+__device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
+    const uint32_t count = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
+    const int tid = threadIdx.x;
+    for (;;) {
+        if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
+        __syncthreads();
+        const uint32_t i = sm.item;
+        __syncthreads();
+        if (i >= count) break;
+        uint32_t pid;
+        const uint8_t* data;
+        page_at(ps, i, pid, data);
+        const uint8_t* end = data + ps.page_bytes;
+        const uint32_t kind = ld32(end - 4);
+        const uint32_t nslots = ld32(end - 8);
+        const uint32_t* words = reinterpret_cast<const uint32_t*>(data);
+        if (kind == GTS_PAGE_LP) {
+            const uint32_t vid = ld32(end - kLpFooter - kSlotBytes);
+            const uint32_t total = ld32(end - 16);
+            const uint32_t len = ld32(data);
+            uint32_t payload = 0;
+            if (op.select_lp(vid, total, len, payload)) {
+                const uint32_t* adj = words + 1;
+                for (uint32_t k = tid; k < len; k += kThreads) {
+                    uint32_t dst = decode_entry(ps, __ldg(adj + k));
+                    uint32_t w = Op::kReadWeights ? __ldg(adj + len + k) : 0u;
+                    op.edge(dst, w, payload, vid);
+                }
+            }
+        } else {
+            const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
+            for (uint32_t t0 = 0; t0 < nslots; t0 += kTile) {
+                const uint32_t nv = min((uint32_t)kTile, nslots - t0);
+                const uint32_t v = start + t0 + tid;
+                const bool sel = (uint32_t)tid < nv && op.select(v);
+                uint32_t deg = 0, off = 0;
+                if (sel) {
+                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
+                    off = ld32(slot + 4);
+                    deg = ld32(data + off);
+                }
+                uint32_t pos, nf, excl, total;
+                tile_scan(sel, deg, pos, nf, excl, total, sm);
+                if (sel) {
+                    sm.off[pos] = off / 4 + 1;
+                    sm.deg[pos] = deg;
+                    sm.src[pos] = v;
+                    sm.payload[pos] = op.payload(v, deg);
+                    sm.pre[pos] = excl;
+                }
+                if (tid == 0) sm.pre[nf] = total;
+                __syncthreads();
+                for (uint32_t e0 = (uint32_t)tid * kEdgesPerThread; e0 < total; e0 += kThreads * kEdgesPerThread) {
+                    uint32_t lo = 0, hi = nf;              // pre[lo] <= e0 < pre[hi]
+                    while (hi - lo > 1) {
+                        uint32_t mid = (lo + hi) >> 1;
+                        if (sm.pre[mid] <= e0) lo = mid; else hi = mid;
+                    }
+                    uint32_t j = lo;
+                    const uint32_t e_end = min(e0 + kEdgesPerThread, total);
+                    for (uint32_t e = e0; e < e_end; ++e) {
+                        while (e >= sm.pre[j + 1]) ++j;
+                        const uint32_t local = e - sm.pre[j];
+                        const uint32_t* adj = words + sm.off[j];
+                        uint32_t dst = decode_entry(ps, __ldg(adj + local));
+                        uint32_t w = Op::kReadWeights ? __ldg(adj + sm.deg[j] + local) : 0u;
+                        op.edge(dst, w, sm.payload[j], sm.src[j]);
+                    }
+                }
+                __syncthreads();
+            }
+        }
+        op.end_page();
+    }
+}
+
+}  // namespace gts

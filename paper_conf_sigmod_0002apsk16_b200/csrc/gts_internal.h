@@ -1,0 +1,76 @@
+// Internal declarations shared by the libgts translation units (host + device).
+// Nothing here is visible through the C ABI (include/gts.h).
+#pragma once
+
+#include <cstdint>
+#include <cstddef>
+#include <string>
+#include <vector>
+
+#include "gts.h"
+
+#ifdef __CUDACC__
+#define GTS_HD __host__ __device__ __forceinline__
+#else
+#define GTS_HD inline
+#endif
+
+namespace gts {
+
+// ---- error plumbing (capi.cpp) ------------------------------------------
+int fail(int code, const char* fmt, ...);          // sets the thread-local message, returns code
+void clear_error();
+
+// ---- page layout constants (include/gts.h "Page layout") ----------------
+constexpr uint32_t kSpFooter = 8;    // u32 nslots, u32 kind
+constexpr uint32_t kLpFooter = 16;   // u32 total_deg, u32 chunk_idx, u32 nslots, u32 kind
+constexpr uint32_t kSlotBytes = 8;   // u32 vid, u32 off
+constexpr uint32_t kDefaultPageBytes = 1u << 20;
+
+// ---- hot-destination table (PageRank CTA pre-aggregation, DESIGN.md K-PR) ----
+// Bucketed two-choice hash table of VIDs; a key lives in bucket h1 if h1 had a
+// free way when it was inserted, else in h2.  No deletion, so a lookup may stop
+// at h1 when h1 has an empty way.
+constexpr uint32_t kHotBuckets = 2048;
+constexpr uint32_t kHotWays = 4;
+constexpr uint32_t kHotSlots = kHotBuckets * kHotWays;
+constexpr uint32_t kHotMax = 4096;          // load factor 0.5
+constexpr uint32_t kHotMinIndeg = 64;
+constexpr uint32_t kHotEmpty = 0xFFFFFFFFu;
+
+GTS_HD uint32_t hot_h1(uint32_t v) { return (v * 0x9E3779B1u) >> 21; }
+GTS_HD uint32_t hot_h2(uint32_t v) { return ((v ^ (v >> 15)) * 0x85EBCA77u) >> 21; }
+
+// ---- graph ---------------------------------------------------------------
+struct Graph {
+    uint64_t n = 0, m = 0;
+    uint32_t page_bytes = 0;
+    uint32_t entry_encoding = 0;
+    bool weighted = false;
+    uint64_t num_pages = 0, n_sp = 0, n_lp = 0, n_lp_vertices = 0, used_bytes = 0, max_outdeg = 0;
+    uint8_t* pages = nullptr;          // host, 4 KiB aligned, num_pages * page_bytes
+    size_t pages_alloc = 0;
+    std::vector<uint32_t> start_vid;   // RVT START_VID
+    std::vector<uint32_t> nslots;      // vertices in the page (1 for LP)
+    std::vector<uint32_t> kind;        // GTS_PAGE_SP / GTS_PAGE_LP
+    std::vector<int64_t> lp_first, lp_last;
+    std::vector<uint32_t> hot_keys;    // kHotSlots entries, kHotEmpty when free
+    uint32_t n_hot = 0;
+    uint64_t uid = 0;                  // process-unique id (device cache key)
+    bool host_registered = false;      // cudaHostRegister'ed by a context
+};
+
+struct PagePlanEntry {
+    uint32_t start_vid;
+    uint32_t nslots;
+    uint32_t kind;
+    int64_t lp_first, lp_last;
+};
+
+// builder.cpp
+int plan_pages(uint64_t n, const uint64_t* row_ptr, bool weighted, uint32_t page_bytes,
+               uint32_t entry_encoding, std::vector<PagePlanEntry>& plan, gts_graph_stats* st);
+
+}  // namespace gts
+
+struct gts_graph : gts::Graph {};

@@ -1,0 +1,116 @@
+// Context / device-graph state shared by the CUDA translation units.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <chrono>
+#include <utility>
+#include <vector>
+
+#include "gts_internal.h"
+
+namespace gts {
+
+#define GTS_CUDA(call)                                                                        \
+    do {                                                                                      \
+        cudaError_t e_ = (call);                                                              \
+        if (e_ != cudaSuccess)                                                                \
+            return ::gts::fail(GTS_ECUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call,          \
+                               cudaGetErrorString(e_));                                       \
+    } while (0)
+
+#define GTS_NCCL(call)                                                                        \
+    do {                                                                                      \
+        ncclResult_t r_ = (call);                                                             \
+        if (r_ != ncclSuccess)                                                                \
+            return ::gts::fail(GTS_ENCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call,          \
+                               ncclGetErrorString(r_));                                       \
+    } while (0)
+
+#define GTS_TRY(call)                   \
+    do {                                \
+        int rc_ = (call);               \
+        if (rc_ != GTS_OK) return rc_;  \
+    } while (0)
+
+// How a kernel finds the bytes of its i-th work page.
+enum PageAddrMode : uint32_t {
+    kAddrByPid = 0,   // data = base + pid * page_bytes          (all pages resident in ID order)
+    kAddrByLoc = 1,   // data = base + loc[pid] * page_bytes     (this rank's pages resident, compacted)
+    kAddrByPos = 2,   // data = base + i * page_bytes            (streamed batch in a ring slot)
+};
+
+struct PageSet {
+    const uint8_t* base;
+    const uint32_t* list;      // global page ids of the work items; nullptr = identity (pid = i)
+    const uint32_t* loc;       // kAddrByLoc: page id -> index within base
+    const uint32_t* d_count;   // device-side item count (nullptr: use count)
+    uint32_t count;
+    uint32_t page_bytes;
+    uint32_t mode;
+    uint32_t entry_encoding;
+    const uint32_t* rvt_start; // START_VID per page (PID16 decode)
+};
+
+// Device copy of a graph for one rank.
+struct DevGraph {
+    uint64_t uid = 0;
+    uint32_t strategy = 0;
+    int world = 1;
+    uint8_t* pages = nullptr;          // this rank's resident pages (compacted in local order)
+    size_t pages_bytes = 0;
+    uint32_t* rvt_start = nullptr;     // [num_pages] START_VID
+    uint32_t* nslots = nullptr;        // [num_pages]
+    uint32_t* loc = nullptr;           // [num_pages] local index or UINT32_MAX
+    uint32_t* local_list = nullptr;    // [n_local] global page ids owned by this rank
+    uint32_t* hot_keys = nullptr;      // [kHotSlots]
+    uint32_t n_local = 0;
+    bool all_local = true;             // every page is local and loc == identity
+    bool resident = false;             // pages uploaded
+    std::vector<uint32_t> h_local_list;
+    std::vector<int32_t> h_owner;
+    uint64_t vlo = 0, vhi = 0;         // Strategy-S WA range of this rank
+};
+
+struct Timer {               // event pairs around launches; summed after the call synchronises
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> pairs;
+    size_t used = 0;
+    std::pair<cudaEvent_t, cudaEvent_t> next();
+    double sum_s();          // sums pairs[0..used) and resets used
+};
+
+struct Context {
+    int device = 0, rank = 0, world = 1;
+    int num_sms = 148;
+    cudaStream_t own_stream = nullptr, stream = nullptr, copy_stream = nullptr;
+    ncclComm_t comm = nullptr;
+    DevGraph dg;
+    std::vector<std::pair<void*, size_t>> scratch;
+    void* h_small = nullptr;   // pinned host scratch (4 KiB)
+    Timer t_main, t_finish, t_merge, t_h2d;
+    cudaEvent_t ring_ready[64], ring_free[64];
+    bool ring_events = false;
+    uint64_t launches = 0, main_launches = 0;
+
+    int buf(int slot, size_t bytes, void** out);   // grow-only scratch device buffer
+};
+
+// context.cu
+int ensure_graph(Context* c, const Graph* g, uint32_t strategy, bool need_resident, double* upload_s);
+int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* cfg, gts_run_config* out);
+int copy_out(Context* c, const void* dsrc, void* dst, size_t bytes, uint32_t out_location);
+int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid);
+int pinned_register(Graph* g);
+
+// P-strategy page ownership (h(j) = j mod N) and S ranges.
+void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t>& owner,
+               std::vector<uint64_t>& vrange);
+
+inline double now_s() {
+    return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+}  // namespace gts
+
+struct gts_context : gts::Context {};

@@ -1,0 +1,387 @@
+// BFS-like algorithms over slotted pages: BFS and SSSP (SURVEY 8(a) a2, a4-a6,
+// a10, a12, a13).
+//
+// Paper: Alg 1 BFS-like path: nextPIDSet holds the pages to visit
+// next; per level the kernels run over those pages only, set LV of unvisited
+// neighbours to curLevel+1 and mark nextPIDSetGPU; the CPU unions the local
+// sets.  Kernels: K_BFS_SP / K_BFS_LP (Alg 2/3).
+//
+// B200 design: frontier = bitmap (n/8 bytes, L2-resident);
+// inside an active page only frontier vertices are expanded (ballot/popc
+// compaction, expand.cuh); discovery is exactly-once through atomicOr on the
+// visited bitmap (a plain test first, then test-and-set); the level array is
+// written once per vertex, coalesced, by the finish kernel from the
+// next-frontier bitmap (equivalent to Alg 2 line 18's store of curLevel+1 by
+// every discoverer); the next page set is the set of pages whose VID range
+// holds a next-frontier bit (segmented OR), computed on the device, so no
+// per-edge RVT lookup is needed.  Multi-GPU Strategy-P: next-frontier bitmaps
+// are all-gathered over NCCL and OR-ed in the finish kernel (NCCL has no
+// bitwise-OR reduction).
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+
+#include "expand.cuh"
+
+namespace gts {
+
+// ------------------------------------------------------------------ ops ---
+
+struct BfsOp {
+    static constexpr bool kReadWeights = false;
+    const uint32_t* cur;
+    uint32_t* visited;
+    uint32_t* next;
+    unsigned long long edges;
+    __device__ bool select(uint32_t v) { return test_bit(cur, v); }
+    __device__ uint32_t payload(uint32_t, uint32_t deg) {
+        edges += deg;
+        return 0u;
+    }
+    __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t len, uint32_t&) {
+        if (!test_bit(cur, vid)) return false;
+        if (threadIdx.x == 0) edges += len;
+        return true;
+    }
+    // Alg 2 lines 17-20: if LV[ADJ_VID] = NULL then discover it.  Exactly one
+    // thread wins the visited bit and records the vertex in the next frontier.
+    __device__ void edge(uint32_t dst, uint32_t, uint32_t, uint32_t) {
+        const uint32_t wi = dst >> 5, b = 1u << (dst & 31);
+        if (!(__ldca(visited + wi) & b)) {
+            if (!(atomicOr(visited + wi, b) & b)) atomicOr(next + wi, b);
+        }
+    }
+    __device__ void end_page() {}
+};
+
+struct SsspOp {
+    static constexpr bool kReadWeights = true;
+    const uint32_t* cur;
+    uint32_t* dist;
+    uint32_t* next;
+    unsigned long long edges;
+    bool ovf;
+    __device__ bool select(uint32_t v) { return test_bit(cur, v); }
+    __device__ uint32_t payload(uint32_t v, uint32_t deg) {
+        edges += deg;
+        return *((volatile uint32_t*)dist + v);
+    }
+    __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t len, uint32_t& pl) {
+        if (!test_bit(cur, vid)) return false;
+        if (threadIdx.x == 0) edges += len;
+        pl = *((volatile uint32_t*)dist + vid);
+        return true;
+    }
+    // relax (u,v,w): candidates >= 2^32-1 are dropped and flagged (checked
+    // exactly after convergence, see sssp_overflow_kernel)
+    __device__ void edge(uint32_t dst, uint32_t w, uint32_t du, uint32_t) {
+        const uint64_t nd = (uint64_t)du + w;
+        if (nd >= (uint64_t)GTS_UNREACHED) {
+            ovf = true;
+            return;
+        }
+        const uint32_t nd32 = (uint32_t)nd;
+        if (nd32 < __ldcg(dist + dst)) {
+            if (nd32 < atomicMin(dist + dst, nd32)) atomicOr(next + (dst >> 5), 1u << (dst & 31));
+        }
+    }
+    __device__ void end_page() {}
+};
+
+struct SsspCheckOp {   // exact overflow test: an edge from a finite vertex into an unreached one
+    static constexpr bool kReadWeights = false;
+    const uint32_t* dist;
+    bool bad;
+    __device__ bool select(uint32_t v) { return __ldg(dist + v) != GTS_UNREACHED; }
+    __device__ uint32_t payload(uint32_t, uint32_t) { return 0u; }
+    __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t&) { return __ldg(dist + vid) != GTS_UNREACHED; }
+    __device__ void edge(uint32_t dst, uint32_t, uint32_t, uint32_t) {
+        if (__ldg(dist + dst) == GTS_UNREACHED) bad = true;
+    }
+    __device__ void end_page() {}
+};
+
+__device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned long long* out) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
+    if ((threadIdx.x & 31) == 0 && v) atomicAdd(out, v);
+}
+
+// -------------------------------------------------------------- kernels ---
+
+__global__ void __launch_bounds__(kThreads, 2)
+bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
+                  uint32_t* work_ctr, unsigned long long* edges_out) {
+    __shared__ TileSmem sm;
+    BfsOp op{cur, visited, next, 0ull};
+    expand_pages(ps, op, sm, work_ctr);
+    block_add_u64(op.edges, edges_out);
+}
+
+__global__ void __launch_bounds__(kThreads, 2)
+sssp_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* dist, uint32_t* next,
+                   uint32_t* work_ctr, unsigned long long* edges_out, uint32_t* ovf_flag) {
+    __shared__ TileSmem sm;
+    SsspOp op{cur, dist, next, 0ull, false};
+    expand_pages(ps, op, sm, work_ctr);
+    block_add_u64(op.edges, edges_out);
+    if (__syncthreads_or(op.ovf) && threadIdx.x == 0) *ovf_flag = 1u;
+}
+
+__global__ void __launch_bounds__(kThreads, 2)
+sssp_check_kernel(PageSet ps, const uint32_t* __restrict__ dist, uint32_t* work_ctr, uint32_t* bad_flag) {
+    __shared__ TileSmem sm;
+    SsspCheckOp op{dist, false};
+    expand_pages(ps, op, sm, work_ctr);
+    if (__syncthreads_or(op.bad) && threadIdx.x == 0) *bad_flag = 1u;
+}
+
+// Merge the per-rank next frontiers (world > 1: OR of the all-gathered
+// bitmaps), add them to visited, write LV = new_level once per newly reached
+// vertex (when level != nullptr) and count them.
+__global__ void frontier_finish_kernel(const uint32_t* __restrict__ gathered, int world, uint64_t words,
+                                       uint32_t* next, uint32_t* visited, uint32_t* level, uint32_t new_level,
+                                       unsigned long long* count) {
+    unsigned long long c = 0;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
+        uint32_t bits = gathered[w];
+        for (int r = 1; r < world; ++r) bits |= gathered[(uint64_t)r * words + w];
+        if (world > 1) {
+            next[w] = bits;
+            if (visited) visited[w] |= bits;
+        }
+        c += __popc(bits);
+        if (level) {
+            while (bits) {
+                const int b = __ffs(bits) - 1;
+                level[w * 32 + b] = new_level;
+                bits &= bits - 1;
+            }
+        }
+    }
+    block_add_u64(c, count);
+}
+
+// Next page set (nextPIDSet, Alg 1 lines 29-30): the pages among
+// `pages` (this rank's) whose VID range [START_VID, START_VID + nslots) has a
+// bit set in `bits`.  One warp per page.
+__global__ void frontier_pages_kernel(const uint32_t* __restrict__ bits, const uint32_t* __restrict__ rvt_start,
+                                      const uint32_t* __restrict__ nslots, const uint32_t* __restrict__ pages,
+                                      uint32_t npages, uint32_t* out_list, uint32_t* out_count) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t warps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < npages; i += warps) {
+        const uint32_t p = pages ? pages[i] : i;
+        const uint64_t lo = rvt_start[p], hi = lo + nslots[p];   // [lo, hi)
+        const uint64_t w0 = lo >> 5, w1 = (hi - 1) >> 5;
+        bool any = false;
+        for (uint64_t w = w0 + lane; w <= w1; w += 32) {
+            uint32_t m = bits[w];
+            if (w == w0) m &= 0xFFFFFFFFu << (lo & 31);
+            if (w == w1 && ((hi & 31) != 0)) m &= 0xFFFFFFFFu >> (32 - (hi & 31));
+            any |= m != 0;
+        }
+        if (__any_sync(0xFFFFFFFFu, any) && lane == 0) out_list[atomicAdd(out_count, 1u)] = p;
+    }
+}
+
+__global__ void set_source_kernel(uint32_t* value, uint32_t* visited, uint32_t* cur, uint64_t src) {
+    value[src] = 0;
+    if (visited) visited[src >> 5] |= 1u << (src & 31);
+    cur[src >> 5] |= 1u << (src & 31);
+}
+
+// ---------------------------------------------------------------- driver ---
+
+struct Counters {               // device scratch, slot kCtr
+    uint32_t work;
+    uint32_t list_count;
+    unsigned long long count;
+    unsigned long long edges;
+    uint32_t flag;
+    uint32_t flag2;
+};
+
+enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather };
+
+// pages holding vertex v among this rank's pages (Alg 1 line 5: "page ID containing start vertex")
+static std::vector<uint32_t> pages_of_vertex(const Graph* g, const DevGraph& d, int rank, uint64_t v) {
+    std::vector<uint32_t> out;
+    auto it = std::upper_bound(g->start_vid.begin(), g->start_vid.end(), (uint32_t)v);
+    int64_t p = (int64_t)(it - g->start_vid.begin()) - 1;
+    if (p < 0) return out;
+    int64_t a = p, b = p;
+    if (g->kind[p] == GTS_PAGE_LP) {
+        a = g->lp_first[p];
+        b = g->lp_last[p];
+    }
+    for (int64_t q = a; q <= b; ++q)
+        if (d.h_owner[q] == rank) out.push_back((uint32_t)q);
+    return out;
+}
+
+static PageSet resident_set(Context* c, const Graph* g, const uint32_t* list, const uint32_t* d_count) {
+    PageSet ps;
+    ps.base = c->dg.pages;
+    ps.list = list;
+    ps.loc = c->dg.loc;
+    ps.d_count = d_count;
+    ps.count = 0;
+    ps.page_bytes = g->page_bytes;
+    ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
+    ps.entry_encoding = g->entry_encoding;
+    ps.rvt_start = c->dg.rvt_start;
+    return ps;
+}
+
+enum Algo { kBFS, kSSSP };
+
+static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_run_config* cfg, uint32_t* out,
+                    gts_run_stats* st, Algo algo) {
+    clear_error();
+    const double t_start = now_s();
+    gts_run_config rc;
+    GTS_TRY(validate_common(c, g, cfg, &rc));
+    if (!out) return fail(GTS_EINVAL, "NULL output");
+    if (src >= g->n) return fail(GTS_EINVAL, "src %llu >= n %llu", (unsigned long long)src, (unsigned long long)g->n);
+    if (algo == kSSSP && !g->weighted) return fail(GTS_EUNSUPPORTED, "gts_sssp needs a graph built with weights");
+    if (rc.residency == GTS_STREAMED) return fail(GTS_EUNSUPPORTED, "streamed residency not available for this call yet");
+    if (rc.strategy == GTS_STRATEGY_S && c->world > 1)
+        return fail(GTS_EUNSUPPORTED, "Strategy-S traversal not available yet");
+    double upload_s = 0;
+    GTS_TRY(ensure_graph(c, g, rc.strategy, true, &upload_s));
+    const bool timing = rc.flags & GTS_RUN_TIMING;
+    const uint64_t n = g->n, words = (n + 31) / 32;
+    uint32_t *value, *visited = nullptr, *cur, *next, *list, *gathered = nullptr;
+    Counters* ctr;
+    GTS_TRY(c->buf(kBufValue, n * 4, (void**)&value));
+    if (algo == kBFS) GTS_TRY(c->buf(kBufVisited, words * 4, (void**)&visited));
+    GTS_TRY(c->buf(kBufCur, words * 4, (void**)&cur));
+    GTS_TRY(c->buf(kBufNext, words * 4, (void**)&next));
+    GTS_TRY(c->buf(kBufList, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&list));
+    GTS_TRY(c->buf(kBufCtr, sizeof(Counters), (void**)&ctr));
+    if (c->world > 1) GTS_TRY(c->buf(kBufGather, words * 4 * c->world, (void**)&gathered));
+    cudaStream_t s = c->stream;
+    GTS_CUDA(cudaMemsetAsync(value, 0xFF, n * 4, s));
+    if (visited) GTS_CUDA(cudaMemsetAsync(visited, 0, words * 4, s));
+    GTS_CUDA(cudaMemsetAsync(cur, 0, words * 4, s));
+    GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
+    GTS_CUDA(cudaMemsetAsync(ctr, 0, sizeof(Counters), s));
+    set_source_kernel<<<1, 1, 0, s>>>(value, visited, cur, src);
+    uint64_t launches = 1, main_launches = 0;
+    std::vector<uint32_t> l0 = pages_of_vertex(g, c->dg, c->rank, src);
+    uint32_t* hs = (uint32_t*)c->h_small;
+    hs[0] = (uint32_t)l0.size();
+    if (!l0.empty()) GTS_CUDA(cudaMemcpyAsync(list, l0.data(), l0.size() * 4, cudaMemcpyHostToDevice, s));
+    GTS_CUDA(cudaMemcpyAsync(&ctr->list_count, hs, 4, cudaMemcpyHostToDevice, s));
+
+    const void* kexp = algo == kBFS ? (const void*)bfs_expand_kernel : (const void*)sssp_expand_kernel;
+    int grid = 0;
+    GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
+    const int fin_grid = c->num_sms * 4;
+    PageSet ps = resident_set(c, g, list, &ctr->list_count);
+    uint64_t pages_processed = l0.size(), nccl_bytes = 0;
+    uint32_t levels = 0;
+    Counters h;
+    for (uint32_t L = 0;; ++L) {
+        GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+        std::pair<cudaEvent_t, cudaEvent_t> ev;
+        if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+        if (algo == kBFS)
+            bfs_expand_kernel<<<grid, kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges);
+        else
+            sssp_expand_kernel<<<grid, kThreads, 0, s>>>(ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag);
+        if (timing) cudaEventRecord(ev.second, s);
+        GTS_CUDA(cudaGetLastError());
+        ++launches;
+        ++main_launches;
+        if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
+        if (c->world > 1) {
+            GTS_NCCL(ncclGroupStart());
+            if (algo == kSSSP) GTS_NCCL(ncclAllReduce(value, value, n, ncclUint32, ncclMin, c->comm, s));
+            GTS_NCCL(ncclAllGather(next, gathered, words, ncclUint32, c->comm, s));
+            GTS_NCCL(ncclGroupEnd());
+            nccl_bytes += words * 4 + (algo == kSSSP ? n * 4 : 0);
+        }
+        if (timing) { cudaEventRecord(ev.second, s); ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
+        GTS_CUDA(cudaMemsetAsync(&ctr->count, 0, 8, s));
+        GTS_CUDA(cudaMemsetAsync(&ctr->list_count, 0, 4, s));
+        frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, next,
+                                                        visited, algo == kBFS ? value : nullptr, L + 1,
+                                                        &ctr->count);
+        frontier_pages_kernel<<<fin_grid, 256, 0, s>>>(next, c->dg.rvt_start, c->dg.nslots,
+                                                       c->dg.all_local ? nullptr : c->dg.local_list,
+                                                       c->dg.all_local ? (uint32_t)g->num_pages : c->dg.n_local,
+                                                       list, &ctr->list_count);
+        if (timing) cudaEventRecord(ev.second, s);
+        launches += 2;
+        GTS_CUDA(cudaGetLastError());
+        GTS_CUDA(cudaMemcpyAsync(&h, ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+        ++levels;
+        if (h.count == 0) break;
+        pages_processed += h.list_count;
+        std::swap(cur, next);
+        GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
+    }
+    if (algo == kSSSP && c->world > 1) {   // every rank must agree before the collective check
+        GTS_NCCL(ncclAllReduce(&ctr->flag, &ctr->flag, 1, ncclUint32, ncclMax, c->comm, s));
+        GTS_CUDA(cudaMemcpyAsync(&h.flag, &ctr->flag, 4, cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+    }
+    if (algo == kSSSP && h.flag) {
+        // exact overflow test (see SsspOp::edge): sweep all local pages once
+        GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+        GTS_CUDA(cudaMemsetAsync(&ctr->flag2, 0, 4, s));
+        PageSet all = resident_set(c, g, c->dg.all_local ? nullptr : c->dg.local_list, nullptr);
+        all.count = c->dg.n_local;
+        int g2 = 0;
+        GTS_TRY(sms_grid(c, (const void*)sssp_check_kernel, kThreads, 0, &g2));
+        sssp_check_kernel<<<g2, kThreads, 0, s>>>(all, value, &ctr->work, &ctr->flag2);
+        ++launches;
+        uint32_t bad = 0;
+        if (c->world > 1) GTS_NCCL(ncclAllReduce(&ctr->flag2, &ctr->flag2, 1, ncclUint32, ncclMax, c->comm, s));
+        GTS_CUDA(cudaMemcpyAsync(&bad, &ctr->flag2, 4, cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+        if (bad) return fail(GTS_EOVERFLOW, "an SSSP distance reaches 2^32-1");
+    }
+    GTS_TRY(copy_out(c, value, out, n * 4, rc.out_location));
+    if (st) {
+        std::memset(st, 0, sizeof(*st));
+        st->wall_s = now_s() - t_start;
+        st->upload_s = upload_s;
+        if (timing) {
+            st->main_kernel_s = c->t_main.sum_s();
+            st->merge_s = c->t_merge.sum_s();
+            st->finish_s = c->t_finish.sum_s();
+        }
+        st->pages_processed = pages_processed;
+        st->edges_traversed = h.edges;
+        st->nccl_bytes = nccl_bytes;
+        st->launches = launches;
+        st->main_kernel_launches = main_launches;
+        st->levels_or_iters = levels;
+    } else if (timing) {
+        c->t_main.sum_s();
+        c->t_merge.sum_s();
+        c->t_finish.sum_s();
+    }
+    return GTS_OK;
+}
+
+}  // namespace gts
+
+using namespace gts;
+
+extern "C" int gts_bfs(gts_context* ctx, const gts_graph* g, uint64_t src, const gts_run_config* cfg,
+                       uint32_t* level_out, gts_run_stats* stats) {
+    return traverse(ctx, g, src, cfg, level_out, stats, kBFS);
+}
+
+extern "C" int gts_sssp(gts_context* ctx, const gts_graph* g, uint64_t src, const gts_run_config* cfg,
+                        uint32_t* dist_out, gts_run_stats* stats) {
+    return traverse(ctx, g, src, cfg, dist_out, stats, kSSSP);
+}

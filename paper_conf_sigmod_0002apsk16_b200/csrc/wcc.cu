@@ -1,0 +1,153 @@
+// Weakly connected components over slotted pages (R12).
+//
+// Paper: "connected components" is a PageRank-like algorithm run by GTS
+// (P:308), i.e. whole-topology sweeps (ALL_PAGES, Alg 1 line 7); no
+// kernel is given.  B200 design: min-label propagation, label[v] = v
+// initially; every sweep visits every edge (u,v) of every page and lowers
+// the larger of label[u], label[v] to the smaller with atomicMin (labels only
+// decrease, so the fixpoint labels each weakly connected component with its
+// minimum VID); a pointer-jumping pass label[v] = label[label[v]] follows each
+// sweep.  Stops after a sweep that changes nothing.  Strategy-P: labels are
+// merged with an NCCL all-reduce(min) after each sweep.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <cstring>
+
+#include "expand.cuh"
+
+namespace gts {
+
+struct WccOp {
+    static constexpr bool kReadWeights = false;
+    uint32_t* label;
+    bool changed;
+    __device__ bool select(uint32_t) { return true; }
+    __device__ uint32_t payload(uint32_t v, uint32_t deg) { return deg ? __ldcg(label + v) : 0u; }
+    __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t& pl) {
+        pl = __ldcg(label + vid);
+        return true;
+    }
+    __device__ void edge(uint32_t dst, uint32_t, uint32_t lu, uint32_t src) {
+        const uint32_t lv = __ldcg(label + dst);
+        if (lu < lv) {
+            if (atomicMin(label + dst, lu) > lu) changed = true;
+        } else if (lv < lu) {
+            if (atomicMin(label + src, lv) > lv) changed = true;
+        }
+    }
+    __device__ void end_page() {}
+};
+
+__global__ void __launch_bounds__(kThreads, 2)
+wcc_sweep_kernel(PageSet ps, uint32_t* label, uint32_t* work_ctr, uint32_t* changed) {
+    __shared__ TileSmem sm;
+    WccOp op{label, false};
+    expand_pages(ps, op, sm, work_ctr);
+    if (__syncthreads_or(op.changed) && threadIdx.x == 0) *changed = 1u;
+}
+
+__global__ void wcc_init_kernel(uint32_t* label, uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) label[i] = (uint32_t)i;
+}
+
+__global__ void wcc_jump_kernel(uint32_t* label, uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const uint32_t l = label[i];
+        const uint32_t ll = __ldcg(label + l);
+        if (ll < l) label[i] = ll;
+    }
+}
+
+enum { kBufLabel = 30, kBufWccCtr };
+
+}  // namespace gts
+
+using namespace gts;
+
+extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config* cfg, uint32_t* label_out,
+                       gts_run_stats* st) {
+    clear_error();
+    const double t_start = now_s();
+    gts_run_config rc;
+    GTS_TRY(validate_common(c, g, cfg, &rc));
+    if (!label_out) return fail(GTS_EINVAL, "NULL output");
+    if (rc.residency == GTS_STREAMED) return fail(GTS_EUNSUPPORTED, "streamed residency not available for this call yet");
+    if (rc.strategy == GTS_STRATEGY_S && c->world > 1) return fail(GTS_EUNSUPPORTED, "Strategy-S WCC not available yet");
+    double upload_s = 0;
+    GTS_TRY(ensure_graph(c, g, rc.strategy, true, &upload_s));
+    const bool timing = rc.flags & GTS_RUN_TIMING;
+    const uint64_t n = g->n;
+    uint32_t *label, *ctr;
+    GTS_TRY(c->buf(kBufLabel, n * 4, (void**)&label));
+    GTS_TRY(c->buf(kBufWccCtr, 8, (void**)&ctr));
+    cudaStream_t s = c->stream;
+    const int eg = c->num_sms * 4;
+    wcc_init_kernel<<<eg, 256, 0, s>>>(label, n);
+    int grid = 0;
+    GTS_TRY(sms_grid(c, (const void*)wcc_sweep_kernel, kThreads, 0, &grid));
+    PageSet ps;
+    ps.base = c->dg.pages;
+    ps.list = c->dg.all_local ? nullptr : c->dg.local_list;
+    ps.loc = c->dg.loc;
+    ps.d_count = nullptr;
+    ps.count = c->dg.n_local;
+    ps.page_bytes = g->page_bytes;
+    ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
+    ps.entry_encoding = g->entry_encoding;
+    ps.rvt_start = c->dg.rvt_start;
+    uint64_t launches = 1, main_launches = 0, nccl_bytes = 0;
+    uint32_t sweeps = 0;
+    uint32_t* hs = (uint32_t*)c->h_small;
+    for (;;) {
+        GTS_CUDA(cudaMemsetAsync(ctr, 0, 8, s));
+        std::pair<cudaEvent_t, cudaEvent_t> ev;
+        if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+        wcc_sweep_kernel<<<grid, kThreads, 0, s>>>(ps, label, ctr, ctr + 1);
+        if (timing) cudaEventRecord(ev.second, s);
+        GTS_CUDA(cudaGetLastError());
+        ++launches;
+        ++main_launches;
+        ++sweeps;
+        if (c->world > 1) {
+            if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
+            GTS_NCCL(ncclGroupStart());
+            GTS_NCCL(ncclAllReduce(label, label, n, ncclUint32, ncclMin, c->comm, s));
+            GTS_NCCL(ncclAllReduce(ctr + 1, ctr + 1, 1, ncclUint32, ncclMax, c->comm, s));
+            GTS_NCCL(ncclGroupEnd());
+            if (timing) cudaEventRecord(ev.second, s);
+            nccl_bytes += n * 4 + 4;
+        }
+        if (timing) { ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
+        wcc_jump_kernel<<<eg, 256, 0, s>>>(label, n);
+        if (timing) cudaEventRecord(ev.second, s);
+        ++launches;
+        GTS_CUDA(cudaMemcpyAsync(hs, ctr + 1, 4, cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+        if (hs[0] == 0) break;
+    }
+    GTS_TRY(copy_out(c, label, label_out, n * 4, rc.out_location));
+    if (st) {
+        std::memset(st, 0, sizeof(*st));
+        st->wall_s = now_s() - t_start;
+        st->upload_s = upload_s;
+        if (timing) {
+            st->main_kernel_s = c->t_main.sum_s();
+            st->merge_s = c->t_merge.sum_s();
+            st->finish_s = c->t_finish.sum_s();
+        }
+        st->pages_processed = (uint64_t)c->dg.n_local * sweeps;
+        st->edges_traversed = g->m * (uint64_t)sweeps / (uint64_t)c->world;
+        st->nccl_bytes = nccl_bytes;
+        st->launches = launches;
+        st->main_kernel_launches = main_launches;
+        st->levels_or_iters = sweeps;
+    } else if (timing) {
+        c->t_main.sum_s();
+        c->t_merge.sum_s();
+        c->t_finish.sum_s();
+    }
+    return GTS_OK;
+}
