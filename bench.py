@@ -1,0 +1,383 @@
+#!/usr/bin/env python
+"""Benchmark of the GTS hot path on B200 (driver contract).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gts|reference] [--scale S]
+
+One step = one pass of the whole hot path over the resident RMAT-S graph
+(default S = 27, BASELINE.json configs[2]): BFS from vertex 0, 10 PageRank
+iterations, SSSP from vertex 0 (hashed weights), WCC.  `value` is BFS GTEPS
+(edges traversed / BFS device time, all ranks' work / max-over-ranks time);
+PageRank s/iter, SSSP and WCC seconds are reported beside it.  Inputs (the
+9.8 GB topology) are larger than L2, so no flush is needed between steps.
+
+N > 1: launched by torchrun, one process per GPU, Strategy-P (pages
+partitioned h(j) = j mod N, WA merged by NCCL inside libgts).
+
+--impl reference runs the oracle (the paper-defined CPU program of oracle/) on
+the host cores as the reference arm (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+FALLBACK_HBM_GBS = 6650.0
+METRIC = "BFS GTEPS and PageRank s/iter on RMAT-27..30 at 1/2/4/8 B200; % HBM/link BW"
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.lines = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                          "-lms", "200", "-i", str(self.device)], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception as e:  # pragma: no cover
+            log("clock sampler unavailable:", e)
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# --------------------------------------------------------------------- reference arm ---
+
+def run_reference(args, rank):
+    if rank != 0:
+        return
+    import inputs
+    import oracle
+    scale = args.ref_scale
+    log(f"[reference] generating RMAT-{scale} sample")
+    g = inputs.rmat(scale)
+    times, edges = [], 0
+    deg = np.diff(g.row_ptr).astype(np.int64)
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        lv = oracle.bfs(g.row_ptr, g.col, 0)
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+        edges = int(deg[lv != oracle.UNREACHED].sum())
+    t = float(np.sum(times))
+    gteps = edges * len(times) / t / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": gteps, "unit": "GTEPS", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / len(times),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": f"rmat{args.scale}_bfs (reference arm: oracle BFS on the RMAT-{scale} sample)",
+                       "sample_scale": scale, "src": 0},
+            "cpu_baseline": {"value": gteps, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                             "sample": f"oracle BFS from vertex 0 on RMAT-{scale} (same generator as RMAT-{args.scale},"
+                                       f" 1/{2 ** (args.scale - scale)} of its edges), single thread, per step"},
+            "e2e": {"value": gteps, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- GPU arm ---
+
+def cpu_baseline(args):
+    import inputs
+    import oracle
+    scale = args.ref_scale
+    g = inputs.rmat(scale)
+    deg = np.diff(g.row_ptr).astype(np.int64)
+    t0 = time.perf_counter()
+    lv = oracle.bfs(g.row_ptr, g.col, 0)
+    t_bfs = time.perf_counter() - t0
+    edges = int(deg[lv != oracle.UNREACHED].sum())
+    t0 = time.perf_counter()
+    oracle.pagerank(g.row_ptr, g.col, 1, 0.85)
+    t_pr = time.perf_counter() - t0
+    return {"value": edges / t_bfs / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+            "sample": f"oracle BFS from vertex 0 on RMAT-{scale} (same generator, 1/{2 ** (args.scale - scale)} of the "
+                      f"RMAT-{args.scale} edges), single thread; plus 1 oracle PageRank iteration (incl. its transpose)",
+            "bfs_s": t_bfs, "pagerank_s_per_iter": t_pr, "sample_m": g.m}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gts", choices=["gts", "reference"])
+    ap.add_argument("--scale", type=int, default=27)
+    ap.add_argument("--ref-scale", type=int, default=None)
+    ap.add_argument("--page-bytes", type=int, default=1 << 20)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--algos", default="bfs,pr,sssp,wcc")
+    args = ap.parse_args()
+    if args.ref_scale is None:
+        args.ref_scale = min(args.scale, 24)
+    args.warmup = max(args.warmup, 3) if args.impl == "gts" else args.warmup
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus > 1 and world != args.gpus:
+        sys.exit(f"--gpus {args.gpus} must be launched with torchrun --nproc-per-node {args.gpus}")
+
+    if args.impl == "reference":
+        run_reference(args, rank)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import inputs
+    import paper_conf_sigmod_0002apsk16_b200 as G
+
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        os.environ.setdefault("OMP_NUM_THREADS", str(max(1, os.cpu_count() // world)))
+    algos = args.algos.split(",")
+
+    t0 = time.time()
+    g = inputs.rmat(args.scale)
+    n, m = g.n, g.m
+    log(f"[rank {rank}] RMAT-{args.scale} generated n={n} m={m} in {time.time() - t0:.1f}s")
+    t0 = time.time()
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=args.page_bytes)
+    grw = None
+    if "sssp" in algos:
+        w = inputs.edge_weights(g)
+        grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=args.page_bytes)
+        del w
+    gst = gr.stats()
+    log(f"[rank {rank}] pages built in {time.time() - t0:.1f}s: {gst}")
+    del g
+
+    uid = None
+    if world > 1:
+        obj = [G.gts_get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    ctx = G.gts_context_create(local_rank, rank, world, uid)
+    stream = torch.cuda.current_stream()
+    ctx.set_stream(stream.cuda_stream)
+
+    lv = torch.empty(n, dtype=torch.int32, device="cuda")
+    pr = torch.empty(n, dtype=torch.float32, device="cuda")
+    ds = torch.empty(n, dtype=torch.int32, device="cuda")
+    lab = torch.empty(n, dtype=torch.int32, device="cuda")
+
+    def step(record):
+        evs = {}
+        res = {}
+        for a in algos:
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            if a == "bfs":
+                _, st = G.gts_bfs(ctx, gr, 0, out=lv, timing=True)
+            elif a == "pr":
+                _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=pr, timing=True)
+            elif a == "sssp":
+                _, st = G.gts_sssp(ctx, grw, 0, out=ds, timing=True)
+            else:
+                _, st = G.gts_wcc(ctx, gr, out=lab, timing=True)
+            e1.record(stream)
+            evs[a] = (e0, e1)
+            res[a] = st
+        torch.cuda.synchronize()
+        if record is not None:
+            for a in algos:
+                record.setdefault(a, []).append((evs[a][0].elapsed_time(evs[a][1]) * 1e-3, res[a]))
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for i in range(args.warmup):
+        step(None)
+        log(f"[rank {rank}] warmup {i} done")
+    sampler = ClockSampler(local_rank)
+    sampler.start()
+    rec = {}
+    barrier()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    for _ in range(args.steps):
+        step(rec)
+    t_end.record(stream)
+    barrier()
+    clocks = sampler.stop()
+    total_s = t_start.elapsed_time(t_end) * 1e-3
+
+    def maxred(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sumred(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    total_s = maxred(total_s)
+    out = {}
+    for a in algos:
+        out[a] = {"s": maxred(sum(t for t, _ in rec[a])),
+                  "main_s": maxred(sum(st["main_kernel_s"] for _, st in rec[a])),
+                  "main_launches": sum(st["main_kernel_launches"] for _, st in rec[a]),
+                  "launches": sum(st["launches"] for _, st in rec[a]),
+                  "edges": sumred(float(sum(st["edges_traversed"] for _, st in rec[a]))),
+                  "iters": rec[a][-1][1]["levels_or_iters"],
+                  "merge_s": maxred(sum(st["merge_s"] for _, st in rec[a]))}
+    K = args.steps
+    bfs_gteps = out["bfs"]["edges"] / out["bfs"]["s"] / 1e9 if "bfs" in algos else None
+    pr_s_iter = out["pr"]["s"] / (10 * K) if "pr" in algos else None
+
+    # roofline for the dominant kernel (largest share of the step among the main kernels)
+    peak, peak_src = measured_peaks()
+    B_pr_scatter = 12 * m + 16 * n          # topology 4m+12n, x 4n, acc RMW 8m
+    cand = {}
+    if "pr" in algos:
+        cand["pr_scatter_kernel"] = (out["pr"]["main_s"], out["pr"]["main_launches"], B_pr_scatter / world)
+    if "wcc" in algos:
+        cand["wcc_sweep_kernel"] = (out["wcc"]["main_s"], out["wcc"]["main_launches"], (4 * m + 12 * n + 8 * m) / world)
+    if "bfs" in algos:
+        eb = out["bfs"]["edges"] / K
+        cand["bfs_expand_kernel"] = (out["bfs"]["main_s"], out["bfs"]["main_launches"],
+                                     (4 * eb + 12 * n + 4 * eb) / max(1, out["bfs"]["main_launches"] / K) / world)
+    dom = max(cand, key=lambda k: cand[k][0]) if cand else None
+    roof = None
+    if dom:
+        ks, kl, bytes_per_launch = cand[dom]
+        avg = ks / max(1, kl)
+        ach = bytes_per_launch / avg / 1e9 if avg > 0 else 0.0
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tp):
+            traffic = json.load(open(tp)).get(dom)
+        roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                "traffic": traffic, "algorithmic_bytes_per_launch": bytes_per_launch, "avg_launch_s": avg,
+                "share_of_step": ks / total_s if total_s else None, "peak_source": peak_src}
+
+    # end-to-end through the public API with host buffers (pages re-uploaded from pinned host memory)
+    e2e = None
+    if not args.no_e2e and "bfs" in algos:
+        hl = np.empty(n, np.uint32)
+        hp = np.empty(n, np.float32)
+        tb, tp_ = [], []
+        for _ in range(max(1, min(K, 3))):
+            ctx.evict(gr)
+            barrier()
+            t0 = time.perf_counter()
+            _, st = G.gts_bfs(ctx, gr, 0, out=hl)
+            tb.append(maxred(time.perf_counter() - t0))
+            ctx.evict(gr)
+            barrier()
+            t0 = time.perf_counter()
+            G.gts_pagerank(ctx, gr, 10, 0.85, out=hp)
+            tp_.append(maxred(time.perf_counter() - t0))
+        e2e = {"value": out["bfs"]["edges"] / K / float(np.median(tb)) / 1e9, "unit": "GTEPS",
+               "h2d_bytes_per_step": int(gst["topo_bytes"] / world), "d2h_bytes_per_step": 4 * n,
+               "what": "gts_bfs on an evicted context with a host output: H2D of this rank's pinned pages + BFS + "
+                       "D2H of the level array, wall clock, median",
+               "pagerank_s_per_iter": float(np.median(tp_)) / 10}
+
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
+        try:
+            cpu = cpu_baseline(args)
+        except Exception as e:  # pragma: no cover
+            cpu = {"error": str(e)}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": bfs_gteps, "unit": "GTEPS", "n_gpus": world, "steps": K,
+                "warmup": args.warmup, "ms_per_step": 1e3 * total_s / K, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "config": {"workload": f"rmat{args.scale}_bfs_pr_sssp_wcc", "scale": args.scale, "n": n, "m": m,
+                           "edge_factor": 16, "abc": [0.57, 0.19, 0.19], "seed": args.scale, "src": 0,
+                           "page_bytes": args.page_bytes, "num_pages": gst["num_pages"], "n_lp": gst["n_lp"],
+                           "topo_bytes": gst["topo_bytes"], "residency": "resident",
+                           "strategy": "P" if world > 1 else "single",
+                           "parallelism": f"strategy-P x{world}",
+                           "l2": "inputs larger than L2 (topology %.1f GB vs 126 MB L2), no flush" %
+                                 (gst["topo_bytes"] / 1e9),
+                           "step": "+".join(algos)},
+                "pagerank_s_per_iter": pr_s_iter, "pagerank_dtype": "f32",
+                "bfs_levels": out.get("bfs", {}).get("iters"),
+                "sssp_s": out["sssp"]["s"] / K if "sssp" in algos else None,
+                "sssp_rounds": out.get("sssp", {}).get("iters"),
+                "wcc_s": out["wcc"]["s"] / K if "wcc" in algos else None,
+                "wcc_sweeps": out.get("wcc", {}).get("iters"),
+                "kernel_s_per_step": {a: out[a]["main_s"] / K for a in algos},
+                "merge_s_per_step": {a: out[a]["merge_s"] / K for a in algos},
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "gpu_launches": int(sum(out[a]["launches"] for a in algos))}
+        print(json.dumps(line), flush=True)
+    ctx.free()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
