@@ -48,13 +48,10 @@ static inline void rmat_edge(const rmat_p* p, uint64_t e, uint32_t* su, uint32_t
         uint64_t r;
         if ((l & 1) == 0) { h = splitmix64(p->seed_mix + ((e << 5) | (uint64_t)(l >> 1))); r = h >> 32; }
         else r = h & 0xFFFFFFFFULL;
-        uint64_t sb, db;
-        if (r < p->ta) { sb = 0; db = 0; }
-        else if (r < p->tab) { sb = 0; db = 1; }
-        else if (r < p->tabc) { sb = 1; db = 0; }
-        else { sb = 1; db = 1; }
-        u = (u << 1) | sb;
-        v = (v << 1) | db;
+        /* quadrant: [0,a) -> (0,0), [a,a+b) -> (0,1), [a+b,a+b+c) -> (1,0), else (1,1); branch-free */
+        uint64_t ga = r >= p->ta, gab = r >= p->tab, gabc = r >= p->tabc;
+        u = (u << 1) | gab;
+        v = (v << 1) | (ga ^ gab ^ gabc);
     }
     *su = (uint32_t)u; *sv = (uint32_t)v;
 }
@@ -116,20 +113,22 @@ int gen_rmat(int scale, uint64_t edge_factor, double a, double b, double c, uint
     p.seed_mix = splitmix64(seed ^ 0x524D4154ULL /* "RMAT" */);
     p.scale = scale;
     uint64_t* cnt = (uint64_t*)calloc(n, sizeof(uint64_t));
-    if (!cnt) return -2;
+    uint32_t* tmp = (uint32_t*)malloc(2 * m * sizeof(uint32_t));   /* one generation pass: (u, v) pairs */
+    if (!cnt || !tmp) { free(cnt); free(tmp); return -2; }
     #pragma omp parallel for schedule(static, 65536)
     for (int64_t e = 0; e < (int64_t)m; ++e) {
         uint32_t u, v; rmat_edge(&p, (uint64_t)e, &u, &v);
+        tmp[2 * e] = u; tmp[2 * e + 1] = v;
         __atomic_fetch_add(&cnt[u], 1, __ATOMIC_RELAXED);
     }
     scan_counts(n, cnt, row_ptr);
     memcpy(cnt, row_ptr, n * sizeof(uint64_t)); /* cursors */
     #pragma omp parallel for schedule(static, 65536)
     for (int64_t e = 0; e < (int64_t)m; ++e) {
-        uint32_t u, v; rmat_edge(&p, (uint64_t)e, &u, &v);
-        uint64_t pos = __atomic_fetch_add(&cnt[u], 1, __ATOMIC_RELAXED);
-        col[pos] = v;
+        uint64_t pos = __atomic_fetch_add(&cnt[tmp[2 * e]], 1, __ATOMIC_RELAXED);
+        col[pos] = tmp[2 * e + 1];
     }
+    free(tmp);
     free(cnt);
     sort_rows(n, row_ptr, col);
     return 0;
