@@ -111,7 +111,18 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
     double t0 = now_s();
     uint32_t strat_key = c->world > 1 ? strategy : 0;
     if (c->dg.uid != g->uid || c->dg.strategy != strat_key || c->dg.world != c->world) {
-        free_devgraph(c->dg);
+        if (c->dg.uid) {                              // park the current graph, bring back g if parked
+            c->parked.push_back(std::move(c->dg));
+            c->dg = DevGraph();
+        }
+        for (size_t i = 0; i < c->parked.size(); ++i)
+            if (c->parked[i].uid == g->uid && c->parked[i].strategy == strat_key && c->parked[i].world == c->world) {
+                c->dg = std::move(c->parked[i]);
+                c->parked.erase(c->parked.begin() + i);
+                break;
+            }
+    }
+    if (c->dg.uid != g->uid) {
         DevGraph& d = c->dg;
         d.uid = g->uid;
         d.strategy = strat_key;
@@ -150,6 +161,12 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
         const size_t pb = g->page_bytes;
         d.pages_bytes = (size_t)d.n_local * pb;
         cudaError_t e = cudaMalloc(&d.pages, std::max<size_t>(d.pages_bytes, 256));
+        while (e != cudaSuccess && !c->parked.empty()) {   // make room: drop the oldest parked graph
+            cudaGetLastError();
+            free_devgraph(c->parked.front());
+            c->parked.erase(c->parked.begin());
+            e = cudaMalloc(&d.pages, std::max<size_t>(d.pages_bytes, 256));
+        }
         if (e != cudaSuccess) {
             cudaGetLastError();
             return fail(GTS_ENOMEM, "resident pages: cudaMalloc(%zu) failed: %s", d.pages_bytes,
@@ -272,6 +289,7 @@ extern "C" void gts_context_free(gts_context* c) {
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
     free_devgraph(c->dg);
+    for (auto& d : c->parked) free_devgraph(d);
     for (auto& b : c->scratch) cudaFree(b.first);
     for (Timer* t : {&c->t_main, &c->t_finish, &c->t_merge, &c->t_h2d})
         for (auto& p : t->pairs) {
@@ -296,6 +314,11 @@ extern "C" int gts_context_evict(gts_context* c, const gts_graph* g) {
     cudaSetDevice(c->device);
     cudaStreamSynchronize(c->stream);
     if (!g || c->dg.uid == g->uid) free_devgraph(c->dg);
+    for (size_t i = c->parked.size(); i-- > 0;)
+        if (!g || c->parked[i].uid == g->uid) {
+            free_devgraph(c->parked[i]);
+            c->parked.erase(c->parked.begin() + i);
+        }
     return GTS_OK;
 }
 

@@ -85,7 +85,8 @@ struct Context {
     int num_sms = 148;
     cudaStream_t own_stream = nullptr, stream = nullptr, copy_stream = nullptr;
     ncclComm_t comm = nullptr;
-    DevGraph dg;
+    DevGraph dg;                   // the graph of the current call
+    std::vector<DevGraph> parked;  // other graphs kept resident (evicted LRU-first under memory pressure)
     std::vector<std::pair<void*, size_t>> scratch;
     void* h_small = nullptr;   // pinned host scratch (4 KiB)
     Timer t_main, t_finish, t_merge, t_h2d;
