@@ -1,0 +1,49 @@
+// Cache-policy-tagged global memory operations for sm_100a.
+//
+// Topology pages and the read-only attribute vector are streamed once per
+// sweep: they are loaded with an L2 evict_first policy (and no L1 allocation)
+// so they do not push the randomly-updated write attribute vector (acc /
+// labels / bitmaps) out of the 126 MB L2.
+#pragma once
+
+#include <cstdint>
+
+namespace gts {
+
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+
+__device__ __forceinline__ uint4 ld_stream_v4(const void* p, uint64_t pol) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                 : "l"(p), "l"(pol));
+    return r;
+}
+
+__device__ __forceinline__ uint32_t ld_stream_u32(const void* p, uint64_t pol) {
+    uint32_t r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    return r;
+}
+
+__device__ __forceinline__ uint2 ld_stream_v2(const void* p, uint64_t pol) {
+    uint2 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
+                 : "=r"(r.x), "=r"(r.y)
+                 : "l"(p), "l"(pol));
+    return r;
+}
+
+__device__ __forceinline__ float ld_stream_f32(const float* p, uint64_t pol) {
+    return __uint_as_float(ld_stream_u32(p, pol));
+}
+
+__device__ __forceinline__ uint32_t word_of(const uint4& v, int k) {
+    return k == 0 ? v.x : k == 1 ? v.y : k == 2 ? v.z : v.w;
+}
+
+}  // namespace gts
