@@ -15,6 +15,7 @@
 
 #include <cstdint>
 
+#include "memops.cuh"
 #include "runtime.h"
 
 namespace gts {
@@ -94,12 +95,18 @@ __device__ __forceinline__ void tile_scan(bool sel, uint32_t deg, uint32_t& pos,
 //   bool select(uint32_t vid)                            -- SP vertex expanded?
 //   uint32_t payload(uint32_t vid, uint32_t deg)         -- per selected vertex
 //   bool select_lp(uint32_t vid, uint32_t total_deg, uint32_t chunk_len, uint32_t& payload)
-//   void edge(uint32_t dst, uint32_t w, uint32_t payload, uint32_t src)
+//   void edges(const uint32_t dst[E], const uint32_t w[E], const uint32_t pl[E], const uint32_t src[E],
+//              const bool valid[E])                      -- E = kEdgesPerThread edges, loads already issued
 //   void end_page()
+// Edges reach the op in groups of kEdgesPerThread whose adjacency words were
+// loaded back to back, so each thread has that many independent loads in
+// flight, and the op can issue its own per-edge loads (visited bits, dist,
+// labels) as a batch before acting on them.
 template <class Op>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
     const uint32_t count = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
     const int tid = threadIdx.x;
+    const uint64_t pol = policy_evict_first();
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
         __syncthreads();
@@ -120,10 +127,21 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             uint32_t payload = 0;
             if (op.select_lp(vid, total, len, payload)) {
                 const uint32_t* adj = words + 1;
-                for (uint32_t k = tid; k < len; k += kThreads) {
-                    uint32_t dst = decode_entry(ps, __ldg(adj + k));
-                    uint32_t w = Op::kReadWeights ? __ldg(adj + len + k) : 0u;
-                    op.edge(dst, w, payload, vid);
+                for (uint32_t k0 = tid; k0 < len; k0 += kThreads * kEdgesPerThread) {
+                    uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
+                    bool valid[kEdgesPerThread];
+#pragma unroll
+                    for (int q = 0; q < kEdgesPerThread; ++q) {
+                        const uint32_t k = k0 + q * kThreads;
+                        valid[q] = k < len;
+                        dst[q] = valid[q] ? ld_stream_u32(adj + k, pol) : 0u;
+                        w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_u32(adj + len + k, pol) : 0u;
+                        pl[q] = payload;
+                        src[q] = vid;
+                    }
+#pragma unroll
+                    for (int q = 0; q < kEdgesPerThread; ++q) dst[q] = decode_entry(ps, dst[q]);
+                    op.edges(dst, w, pl, src, valid);
                 }
             }
         } else {
@@ -135,9 +153,10 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 uint32_t deg = 0, off = 0;
                 if (sel) {
                     const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
-                    off = ld32(slot + 4);
-                    deg = ld32(data + off);
+                    off = ld_stream_u32(slot + 4, pol);
+                    deg = ld_stream_u32(data + off, pol);
                 }
+                if (!__syncthreads_or(sel)) continue;   // no frontier vertex in this tile
                 uint32_t pos, nf, excl, total;
                 tile_scan(sel, deg, pos, nf, excl, total, sm);
                 if (sel) {
@@ -155,16 +174,26 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                         uint32_t mid = (lo + hi) >> 1;
                         if (sm.pre[mid] <= e0) lo = mid; else hi = mid;
                     }
-                    uint32_t j = lo;
-                    const uint32_t e_end = min(e0 + kEdgesPerThread, total);
-                    for (uint32_t e = e0; e < e_end; ++e) {
-                        while (e >= sm.pre[j + 1]) ++j;
+                    uint32_t j = lo, nxt = sm.pre[lo + 1];
+                    uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
+                    bool valid[kEdgesPerThread];
+#pragma unroll
+                    for (int q = 0; q < kEdgesPerThread; ++q) {
+                        const uint32_t e = e0 + q;
+                        valid[q] = e < total;
+                        if (valid[q]) {
+                            while (e >= nxt) nxt = sm.pre[++j + 1];
+                        }
                         const uint32_t local = e - sm.pre[j];
                         const uint32_t* adj = words + sm.off[j];
-                        uint32_t dst = decode_entry(ps, __ldg(adj + local));
-                        uint32_t w = Op::kReadWeights ? __ldg(adj + sm.deg[j] + local) : 0u;
-                        op.edge(dst, w, sm.payload[j], sm.src[j]);
+                        dst[q] = valid[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
+                        w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_l1_u32(adj + sm.deg[j] + local, pol) : 0u;
+                        pl[q] = sm.payload[j];
+                        src[q] = sm.src[j];
                     }
+#pragma unroll
+                    for (int q = 0; q < kEdgesPerThread; ++q) dst[q] = decode_entry(ps, dst[q]);
+                    op.edges(dst, w, pl, src, valid);
                 }
                 __syncthreads();
             }

@@ -30,6 +30,13 @@ __device__ __forceinline__ uint32_t ld_stream_u32(const void* p, uint64_t pol) {
     return r;
 }
 
+// L1-allocating variant: for small strided loads that re-touch the same sectors
+__device__ __forceinline__ uint32_t ld_stream_l1_u32(const void* p, uint64_t pol) {
+    uint32_t r;
+    asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    return r;
+}
+
 __device__ __forceinline__ uint2 ld_stream_v2(const void* p, uint64_t pol) {
     uint2 r;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"

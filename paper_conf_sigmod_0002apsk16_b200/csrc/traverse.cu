@@ -34,23 +34,32 @@ struct BfsOp {
     const uint32_t* cur;
     uint32_t* visited;
     uint32_t* next;
-    unsigned long long edges;
+    unsigned long long nedges;
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
-        edges += deg;
+        nedges += deg;
         return 0u;
     }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t len, uint32_t&) {
         if (!test_bit(cur, vid)) return false;
-        if (threadIdx.x == 0) edges += len;
+        if (threadIdx.x == 0) nedges += len;
         return true;
     }
     // Alg 2 lines 17-20: if LV[ADJ_VID] = NULL then discover it.  Exactly one
     // thread wins the visited bit and records the vertex in the next frontier.
-    __device__ void edge(uint32_t dst, uint32_t, uint32_t, uint32_t) {
-        const uint32_t wi = dst >> 5, b = 1u << (dst & 31);
-        if (!(__ldca(visited + wi) & b)) {
-            if (!(atomicOr(visited + wi, b) & b)) atomicOr(next + wi, b);
+    // The visited words of the whole edge group are loaded first (independent
+    // loads in flight), then tested; the atomic is issued only for clear bits.
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*, const uint32_t*,
+                                          const bool* valid) {
+        uint32_t vis[kEdgesPerThread];
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) vis[q] = valid[q] ? __ldca(visited + (dst[q] >> 5)) : ~0u;
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            const uint32_t wi = dst[q] >> 5, b = 1u << (dst[q] & 31);
+            if (!(vis[q] & b)) {
+                if (!(atomicOr(visited + wi, b) & b)) atomicOr(next + wi, b);
+            }
         }
     }
     __device__ void end_page() {}
@@ -61,30 +70,37 @@ struct SsspOp {
     const uint32_t* cur;
     uint32_t* dist;
     uint32_t* next;
-    unsigned long long edges;
+    unsigned long long nedges;
     bool ovf;
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t v, uint32_t deg) {
-        edges += deg;
+        nedges += deg;
         return *((volatile uint32_t*)dist + v);
     }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t len, uint32_t& pl) {
         if (!test_bit(cur, vid)) return false;
-        if (threadIdx.x == 0) edges += len;
+        if (threadIdx.x == 0) nedges += len;
         pl = *((volatile uint32_t*)dist + vid);
         return true;
     }
     // relax (u,v,w): candidates >= 2^32-1 are dropped and flagged (checked
-    // exactly after convergence, see sssp_overflow_kernel)
-    __device__ void edge(uint32_t dst, uint32_t w, uint32_t du, uint32_t) {
-        const uint64_t nd = (uint64_t)du + w;
-        if (nd >= (uint64_t)GTS_UNREACHED) {
-            ovf = true;
-            return;
-        }
-        const uint32_t nd32 = (uint32_t)nd;
-        if (nd32 < __ldcg(dist + dst)) {
-            if (nd32 < atomicMin(dist + dst, nd32)) atomicOr(next + (dst >> 5), 1u << (dst & 31));
+    // exactly after convergence, see sssp_check_kernel)
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t* w, const uint32_t* du,
+                                          const uint32_t*, const bool* valid) {
+        uint32_t cd[kEdgesPerThread];
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) cd[q] = valid[q] ? __ldcg(dist + dst[q]) : 0u;
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            if (!valid[q]) continue;
+            const uint64_t nd = (uint64_t)du[q] + w[q];
+            if (nd >= (uint64_t)GTS_UNREACHED) {
+                ovf = true;
+                continue;
+            }
+            const uint32_t nd32 = (uint32_t)nd;
+            if (nd32 < cd[q] && nd32 < atomicMin(dist + dst[q], nd32))
+                atomicOr(next + (dst[q] >> 5), 1u << (dst[q] & 31));
         }
     }
     __device__ void end_page() {}
@@ -97,8 +113,11 @@ struct SsspCheckOp {   // exact overflow test: an edge from a finite vertex into
     __device__ bool select(uint32_t v) { return __ldg(dist + v) != GTS_UNREACHED; }
     __device__ uint32_t payload(uint32_t, uint32_t) { return 0u; }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t&) { return __ldg(dist + vid) != GTS_UNREACHED; }
-    __device__ void edge(uint32_t dst, uint32_t, uint32_t, uint32_t) {
-        if (__ldg(dist + dst) == GTS_UNREACHED) bad = true;
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*, const uint32_t*,
+                                          const bool* valid) {
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q)
+            if (valid[q] && __ldg(dist + dst[q]) == GTS_UNREACHED) bad = true;
     }
     __device__ void end_page() {}
 };
@@ -117,7 +136,7 @@ bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visite
     __shared__ TileSmem sm;
     BfsOp op{cur, visited, next, 0ull};
     expand_pages(ps, op, sm, work_ctr);
-    block_add_u64(op.edges, edges_out);
+    block_add_u64(op.nedges, edges_out);
 }
 
 __global__ void __launch_bounds__(kThreads, 2)
@@ -126,7 +145,7 @@ sssp_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* dist,
     __shared__ TileSmem sm;
     SsspOp op{cur, dist, next, 0ull, false};
     expand_pages(ps, op, sm, work_ctr);
-    block_add_u64(op.edges, edges_out);
+    block_add_u64(op.nedges, edges_out);
     if (__syncthreads_or(op.ovf) && threadIdx.x == 0) *ovf_flag = 1u;
 }
 

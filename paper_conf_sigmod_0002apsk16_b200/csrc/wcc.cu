@@ -28,12 +28,19 @@ struct WccOp {
         pl = __ldcg(label + vid);
         return true;
     }
-    __device__ void edge(uint32_t dst, uint32_t, uint32_t lu, uint32_t src) {
-        const uint32_t lv = __ldcg(label + dst);
-        if (lu < lv) {
-            if (atomicMin(label + dst, lu) > lu) changed = true;
-        } else if (lv < lu) {
-            if (atomicMin(label + src, lv) > lv) changed = true;
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t* lu,
+                                          const uint32_t* src, const bool* valid) {
+        uint32_t lv[kEdgesPerThread];
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) lv[q] = valid[q] ? __ldcg(label + dst[q]) : 0u;
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            if (!valid[q]) continue;
+            if (lu[q] < lv[q]) {
+                if (atomicMin(label + dst[q], lu[q]) > lu[q]) changed = true;
+            } else if (lv[q] < lu[q]) {
+                if (atomicMin(label + src[q], lv[q]) > lv[q]) changed = true;
+            }
         }
     }
     __device__ void end_page() {}
