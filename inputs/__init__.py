@@ -51,6 +51,10 @@ def lib():
         L.gen_edge_weights.argtypes = [ctypes.c_uint64, u64p, u32p, ctypes.c_uint64, u32p]
         L.gen_edge_weights.restype = None
         L.gen_num_threads.restype = ctypes.c_int
+        L.gen_permute_csr.argtypes = [ctypes.c_uint64, u64p, u32p, u32p, u64p, u32p]
+        L.gen_permute_csr.restype = ctypes.c_int
+        L.gen_indegree_order.argtypes = [ctypes.c_uint64, u64p, u32p, u32p]
+        L.gen_indegree_order.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -114,6 +118,24 @@ def twitter_like(n: int = TWITTER_N, m: int = TWITTER_M, beta: float = TWITTER_B
     if rc != 0:
         raise RuntimeError(f"gen_twitter_like failed rc={rc}")
     return CSR(row_ptr, col, name=f"twitter_like_n{n}")
+
+
+def indegree_order(g: CSR) -> np.ndarray:
+    """new_of_old: rank of each vertex by in-degree (descending, ties by VID)."""
+    p = np.empty(g.n, dtype=np.uint32)
+    lib().gen_indegree_order(g.n, _p64(g.row_ptr), _p32(g.col), _p32(p))
+    return p
+
+
+def permute(g: CSR, new_of_old: np.ndarray) -> CSR:
+    """The same graph with vertex v renamed new_of_old[v] (rows re-sorted)."""
+    new_of_old = np.ascontiguousarray(new_of_old, dtype=np.uint32)
+    rp = np.empty_like(g.row_ptr)
+    col = np.empty_like(g.col)
+    rc = lib().gen_permute_csr(g.n, _p64(g.row_ptr), _p32(g.col), _p32(new_of_old), _p64(rp), _p32(col))
+    if rc:
+        raise RuntimeError(f"gen_permute_csr rc={rc}")
+    return CSR(rp, col, None, g.name + "_perm")
 
 
 def edge_weights(g: CSR, seed: int = 0x53535350) -> np.ndarray:

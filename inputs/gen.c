@@ -230,3 +230,47 @@ void gen_edge_weights(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, 
         }
     }
 }
+
+/* ------------------------------------------------------------ relabel --- */
+
+/* Apply a vertex permutation to a CSR graph: vertex v becomes new_of_old[v];
+ * out rows sorted.  (Input preparation for ordering experiments.) */
+int gen_permute_csr(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, const uint32_t* new_of_old,
+                    uint64_t* out_row_ptr, uint32_t* out_col) {
+    uint64_t* deg = (uint64_t*)malloc(n * sizeof(uint64_t));
+    uint32_t* old_of_new = (uint32_t*)malloc(n * sizeof(uint32_t));
+    if (!deg || !old_of_new) return -2;
+    #pragma omp parallel for
+    for (int64_t v = 0; v < (int64_t)n; ++v) {
+        old_of_new[new_of_old[v]] = (uint32_t)v;
+    }
+    #pragma omp parallel for
+    for (int64_t u = 0; u < (int64_t)n; ++u) deg[u] = row_ptr[old_of_new[u] + 1] - row_ptr[old_of_new[u]];
+    scan_counts(n, deg, out_row_ptr);
+    #pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t u = 0; u < (int64_t)n; ++u) {
+        uint64_t o = row_ptr[old_of_new[u]], b = out_row_ptr[u], e = out_row_ptr[u + 1];
+        for (uint64_t k = 0; k < e - b; ++k) out_col[b + k] = new_of_old[col[o + k]];
+    }
+    free(deg); free(old_of_new);
+    sort_rows(n, out_row_ptr, out_col);
+    return 0;
+}
+
+/* new_of_old = rank of v by in-degree (descending, ties by VID) */
+int gen_indegree_order(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, uint32_t* new_of_old) {
+    uint64_t m = row_ptr[n];
+    uint32_t* indeg = (uint32_t*)calloc(n, sizeof(uint32_t));
+    if (!indeg) return -2;
+    #pragma omp parallel for schedule(static, 65536)
+    for (int64_t k = 0; k < (int64_t)m; ++k) __atomic_fetch_add(&indeg[col[k]], 1u, __ATOMIC_RELAXED);
+    /* counting sort by in-degree descending (stable in VID) */
+    uint32_t maxd = 0;
+    for (uint64_t v = 0; v < n; ++v) if (indeg[v] > maxd) maxd = indeg[v];
+    uint64_t* bucket = (uint64_t*)calloc((size_t)maxd + 2, sizeof(uint64_t));
+    for (uint64_t v = 0; v < n; ++v) bucket[maxd - indeg[v] + 1]++;
+    for (uint64_t d = 1; d <= (uint64_t)maxd + 1; ++d) bucket[d] += bucket[d - 1];
+    for (uint64_t v = 0; v < n; ++v) new_of_old[v] = (uint32_t)(bucket[maxd - indeg[v]]++);
+    free(bucket); free(indeg);
+    return 0;
+}

@@ -188,6 +188,32 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
     return GTS_OK;
 }
 
+int ensure_ring(Context* c, const Graph* g, uint32_t slots, uint32_t batch_pages, uint8_t** ring) {
+    GTS_TRY(pinned_register(const_cast<Graph*>(g)));
+    if (!c->ring_events) {
+        for (int i = 0; i < 64; ++i) {
+            GTS_CUDA(cudaEventCreateWithFlags(&c->ring_ready[i], cudaEventDisableTiming));
+            GTS_CUDA(cudaEventCreateWithFlags(&c->ring_free[i], cudaEventDisableTiming));
+        }
+        c->ring_events = true;
+    }
+    return c->buf(60 /* kBufRing */, (size_t)slots * batch_pages * g->page_bytes, (void**)ring);
+}
+
+bool choose_streamed(Context* c, const Graph* g, const gts_run_config& rc, uint64_t attr_bytes) {
+    if (rc.residency == GTS_STREAMED) return true;
+    if (rc.residency == GTS_RESIDENT) return false;
+    if (c->dg.uid == g->uid && c->dg.resident) return false;
+    size_t free_b = 0, total_b = 0;
+    if (cudaMemGetInfo(&free_b, &total_b) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    uint64_t P = g->num_pages, local = c->world > 1 ? (P + c->world - 1) / c->world : P;
+    uint64_t need = local * g->page_bytes + attr_bytes + (1ull << 30);
+    return need > free_b;
+}
+
 int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* cfg, gts_run_config* out) {
     if (!ctx || !g) return fail(GTS_EINVAL, "NULL context or graph");
     gts_run_config d;

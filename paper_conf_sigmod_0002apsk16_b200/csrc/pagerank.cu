@@ -26,6 +26,7 @@
 
 #include "expand.cuh"
 #include "memops.cuh"
+#include "sweep.cuh"
 
 namespace gts {
 
@@ -264,12 +265,12 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     if (!rank_out) return fail(GTS_EINVAL, "NULL output");
     if (!(damping >= 0.0 && damping <= 1.0)) return fail(GTS_EINVAL, "damping must be in [0,1]");
     if (dangling > GTS_DANGLING_DROP) return fail(GTS_EINVAL, "unknown dangling mode %u", dangling);
-    if (rc.residency == GTS_STREAMED) return fail(GTS_EUNSUPPORTED, "streamed residency not available for this call yet");
     if (rc.strategy == GTS_STRATEGY_S && c->world > 1) return fail(GTS_EUNSUPPORTED, "Strategy-S PageRank not available yet");
-    double upload_s = 0;
-    GTS_TRY(ensure_graph(c, g, rc.strategy, true, &upload_s));
-    const bool timing = rc.flags & GTS_RUN_TIMING;
     const uint64_t n = g->n;
+    const bool streamed = choose_streamed(c, g, rc, 8 * n);
+    double upload_s = 0;
+    GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
+    const bool timing = rc.flags & GTS_RUN_TIMING;
     float *x, *acc;
     double* dang;
     uint32_t* ctr;
@@ -286,26 +287,23 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     pr_init_kernel<<<eg, 256, 0, s>>>(x, acc, n, (float)(1.0 / (double)n));
     GTS_CUDA(cudaMemsetAsync(dang, 0, 2 * sizeof(double), s));
     uint64_t launches = 1, main_launches = 0, nccl_bytes = 0;
-    PageSet ps;
-    ps.base = c->dg.pages;
-    ps.list = c->dg.all_local ? nullptr : c->dg.local_list;
-    ps.loc = c->dg.loc;
-    ps.d_count = nullptr;
-    ps.count = c->dg.n_local;
-    ps.page_bytes = g->page_bytes;
-    ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
-    ps.entry_encoding = g->entry_encoding;
-    ps.rvt_start = c->dg.rvt_start;
+    SweepStats ss;
+    const uint32_t* d_list = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
     for (uint32_t it = 0; it < iters; ++it) {
         double* D = dang + (it & 1);
-        GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
         std::pair<cudaEvent_t, cudaEvent_t> ev;
-        if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-        kern<<<grid, kThreads, kPrDynSmem, s>>>(ps, x, acc, c->dg.hot_keys, (float)damping, D, ctr);
-        if (timing) cudaEventRecord(ev.second, s);
-        GTS_CUDA(cudaGetLastError());
-        ++launches;
-        ++main_launches;
+        GTS_TRY(sweep_pages(c, g, rc, streamed, &c->dg.h_local_list, d_list, c->dg.n_local, nullptr,
+                            [&](const PageSet& ps, int cap) -> int {
+                                GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
+                                std::pair<cudaEvent_t, cudaEvent_t> e2;
+                                if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
+                                kern<<<std::min(grid, cap), kThreads, kPrDynSmem, s>>>(ps, x, acc, c->dg.hot_keys,
+                                                                                     (float)damping, D, ctr);
+                                if (timing) cudaEventRecord(e2.second, s);
+                                GTS_CUDA(cudaGetLastError());
+                                ++main_launches;
+                                return GTS_OK;
+                            }, &ss));
         if (c->world > 1) {
             if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
             GTS_NCCL(ncclGroupStart());
@@ -321,6 +319,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         if (timing) cudaEventRecord(ev.second, s);
         ++launches;
     }
+    launches += main_launches;
     GTS_CUDA(cudaGetLastError());
     GTS_TRY(copy_out(c, x, rank_out, n * 4, rc.out_location));
     if (st) {
@@ -333,6 +332,8 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
             st->finish_s = c->t_finish.sum_s();
         }
         st->pages_processed = (uint64_t)c->dg.n_local * iters;
+        st->h2d_bytes = ss.h2d_bytes;
+        if (timing) st->h2d_s = c->t_h2d.sum_s();
         st->edges_traversed = g->m * (uint64_t)iters / (uint64_t)c->world;
         st->nccl_bytes = nccl_bytes;
         st->launches = launches;
@@ -342,6 +343,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         c->t_main.sum_s();
         c->t_merge.sum_s();
         c->t_finish.sum_s();
+        c->t_h2d.sum_s();
     }
     return GTS_OK;
 }

@@ -103,6 +103,8 @@ int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* 
 int copy_out(Context* c, const void* dsrc, void* dst, size_t bytes, uint32_t out_location);
 int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid);
 int pinned_register(Graph* g);
+// residency decision (GTS_RESIDENCY_AUTO: resident iff this rank's pages + attributes fit in free HBM)
+bool choose_streamed(Context* c, const Graph* g, const gts_run_config& rc, uint64_t attr_bytes);
 
 // P-strategy page ownership (h(j) = j mod N) and S ranges.
 void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t>& owner,

@@ -24,6 +24,7 @@
 #include <cstring>
 
 #include "expand.cuh"
+#include "sweep.cuh"
 
 namespace gts {
 
@@ -267,13 +268,13 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     if (!out) return fail(GTS_EINVAL, "NULL output");
     if (src >= g->n) return fail(GTS_EINVAL, "src %llu >= n %llu", (unsigned long long)src, (unsigned long long)g->n);
     if (algo == kSSSP && !g->weighted) return fail(GTS_EUNSUPPORTED, "gts_sssp needs a graph built with weights");
-    if (rc.residency == GTS_STREAMED) return fail(GTS_EUNSUPPORTED, "streamed residency not available for this call yet");
     if (rc.strategy == GTS_STRATEGY_S && c->world > 1)
         return fail(GTS_EUNSUPPORTED, "Strategy-S traversal not available yet");
-    double upload_s = 0;
-    GTS_TRY(ensure_graph(c, g, rc.strategy, true, &upload_s));
-    const bool timing = rc.flags & GTS_RUN_TIMING;
     const uint64_t n = g->n, words = (n + 31) / 32;
+    const bool streamed = choose_streamed(c, g, rc, 4 * n + 16 * words);
+    double upload_s = 0;
+    GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
+    const bool timing = rc.flags & GTS_RUN_TIMING;
     uint32_t *value, *visited = nullptr, *cur, *next, *list, *gathered = nullptr;
     Counters* ctr;
     GTS_TRY(c->buf(kBufValue, n * 4, (void**)&value));
@@ -301,22 +302,29 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     int grid = 0;
     GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
     const int fin_grid = c->num_sms * 4;
-    PageSet ps = resident_set(c, g, list, &ctr->list_count);
     uint64_t pages_processed = l0.size(), nccl_bytes = 0;
     uint32_t levels = 0;
     Counters h;
+    SweepStats ss;
+    std::vector<uint32_t> h_list = l0;             // streamed mode: this level's pages on the host (ascending)
     for (uint32_t L = 0;; ++L) {
-        GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+        GTS_TRY(sweep_pages(c, g, rc, streamed, &h_list, list, (uint32_t)h_list.size(), &ctr->list_count,
+                            [&](const PageSet& ps, int cap) -> int {
+                                GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+                                std::pair<cudaEvent_t, cudaEvent_t> ev;
+                                if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+                                if (algo == kBFS)
+                                    bfs_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next,
+                                                                                         &ctr->work, &ctr->edges);
+                                else
+                                    sssp_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(
+                                        ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag);
+                                if (timing) cudaEventRecord(ev.second, s);
+                                GTS_CUDA(cudaGetLastError());
+                                ++main_launches;
+                                return GTS_OK;
+                            }, &ss));
         std::pair<cudaEvent_t, cudaEvent_t> ev;
-        if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-        if (algo == kBFS)
-            bfs_expand_kernel<<<grid, kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges);
-        else
-            sssp_expand_kernel<<<grid, kThreads, 0, s>>>(ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag);
-        if (timing) cudaEventRecord(ev.second, s);
-        GTS_CUDA(cudaGetLastError());
-        ++launches;
-        ++main_launches;
         if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
         if (c->world > 1) {
             GTS_NCCL(ncclGroupStart());
@@ -343,6 +351,16 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         ++levels;
         if (h.count == 0) break;
         pages_processed += h.list_count;
+        if (streamed) {                          // the host drives the copies: fetch and sort the page set
+            h_list.resize(h.list_count);
+            if (h.list_count) {
+                GTS_CUDA(cudaMemcpyAsync(h_list.data(), list, h.list_count * 4ull, cudaMemcpyDeviceToHost, s));
+                GTS_CUDA(cudaStreamSynchronize(s));
+                std::sort(h_list.begin(), h_list.end());
+                GTS_CUDA(cudaMemcpyAsync(list, h_list.data(), h.list_count * 4ull, cudaMemcpyHostToDevice, s));
+                GTS_CUDA(cudaStreamSynchronize(s));
+            }
+        }
         std::swap(cur, next);
         GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
     }
@@ -352,15 +370,20 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         GTS_CUDA(cudaStreamSynchronize(s));
     }
     if (algo == kSSSP && h.flag) {
-        // exact overflow test (see SsspOp::edge): sweep all local pages once
-        GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+        // exact overflow test (see SsspOp::edges): sweep all local pages once
         GTS_CUDA(cudaMemsetAsync(&ctr->flag2, 0, 4, s));
-        PageSet all = resident_set(c, g, c->dg.all_local ? nullptr : c->dg.local_list, nullptr);
-        all.count = c->dg.n_local;
         int g2 = 0;
         GTS_TRY(sms_grid(c, (const void*)sssp_check_kernel, kThreads, 0, &g2));
-        sssp_check_kernel<<<g2, kThreads, 0, s>>>(all, value, &ctr->work, &ctr->flag2);
-        ++launches;
+        GTS_TRY(sweep_pages(c, g, rc, streamed, &c->dg.h_local_list,
+                            (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list, c->dg.n_local, nullptr,
+                            [&](const PageSet& ps, int cap) -> int {
+                                GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+                                sssp_check_kernel<<<std::min(g2, cap), kThreads, 0, s>>>(ps, value, &ctr->work,
+                                                                                        &ctr->flag2);
+                                GTS_CUDA(cudaGetLastError());
+                                ++launches;
+                                return GTS_OK;
+                            }, &ss));
         uint32_t bad = 0;
         if (c->world > 1) GTS_NCCL(ncclAllReduce(&ctr->flag2, &ctr->flag2, 1, ncclUint32, ncclMax, c->comm, s));
         GTS_CUDA(cudaMemcpyAsync(&bad, &ctr->flag2, 4, cudaMemcpyDeviceToHost, s));
@@ -378,15 +401,18 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
             st->finish_s = c->t_finish.sum_s();
         }
         st->pages_processed = pages_processed;
+        st->h2d_bytes = ss.h2d_bytes;
+        if (timing) st->h2d_s = c->t_h2d.sum_s();
         st->edges_traversed = h.edges;
         st->nccl_bytes = nccl_bytes;
-        st->launches = launches;
+        st->launches = launches + main_launches;
         st->main_kernel_launches = main_launches;
         st->levels_or_iters = levels;
     } else if (timing) {
         c->t_main.sum_s();
         c->t_merge.sum_s();
         c->t_finish.sum_s();
+        c->t_h2d.sum_s();
     }
     return GTS_OK;
 }

@@ -15,6 +15,7 @@
 #include <cstring>
 
 #include "expand.cuh"
+#include "sweep.cuh"
 
 namespace gts {
 
@@ -81,12 +82,12 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     gts_run_config rc;
     GTS_TRY(validate_common(c, g, cfg, &rc));
     if (!label_out) return fail(GTS_EINVAL, "NULL output");
-    if (rc.residency == GTS_STREAMED) return fail(GTS_EUNSUPPORTED, "streamed residency not available for this call yet");
     if (rc.strategy == GTS_STRATEGY_S && c->world > 1) return fail(GTS_EUNSUPPORTED, "Strategy-S WCC not available yet");
-    double upload_s = 0;
-    GTS_TRY(ensure_graph(c, g, rc.strategy, true, &upload_s));
-    const bool timing = rc.flags & GTS_RUN_TIMING;
     const uint64_t n = g->n;
+    const bool streamed = choose_streamed(c, g, rc, 4 * n);
+    double upload_s = 0;
+    GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
+    const bool timing = rc.flags & GTS_RUN_TIMING;
     uint32_t *label, *ctr;
     GTS_TRY(c->buf(kBufLabel, n * 4, (void**)&label));
     GTS_TRY(c->buf(kBufWccCtr, 8, (void**)&ctr));
@@ -95,28 +96,25 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     wcc_init_kernel<<<eg, 256, 0, s>>>(label, n);
     int grid = 0;
     GTS_TRY(sms_grid(c, (const void*)wcc_sweep_kernel, kThreads, 0, &grid));
-    PageSet ps;
-    ps.base = c->dg.pages;
-    ps.list = c->dg.all_local ? nullptr : c->dg.local_list;
-    ps.loc = c->dg.loc;
-    ps.d_count = nullptr;
-    ps.count = c->dg.n_local;
-    ps.page_bytes = g->page_bytes;
-    ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
-    ps.entry_encoding = g->entry_encoding;
-    ps.rvt_start = c->dg.rvt_start;
     uint64_t launches = 1, main_launches = 0, nccl_bytes = 0;
     uint32_t sweeps = 0;
     uint32_t* hs = (uint32_t*)c->h_small;
+    SweepStats ss;
+    const uint32_t* d_list = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
     for (;;) {
-        GTS_CUDA(cudaMemsetAsync(ctr, 0, 8, s));
+        GTS_CUDA(cudaMemsetAsync(ctr + 1, 0, 4, s));
         std::pair<cudaEvent_t, cudaEvent_t> ev;
-        if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-        wcc_sweep_kernel<<<grid, kThreads, 0, s>>>(ps, label, ctr, ctr + 1);
-        if (timing) cudaEventRecord(ev.second, s);
-        GTS_CUDA(cudaGetLastError());
-        ++launches;
-        ++main_launches;
+        GTS_TRY(sweep_pages(c, g, rc, streamed, &c->dg.h_local_list, d_list, c->dg.n_local, nullptr,
+                            [&](const PageSet& ps, int cap) -> int {
+                                GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
+                                std::pair<cudaEvent_t, cudaEvent_t> e2;
+                                if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
+                                wcc_sweep_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(ps, label, ctr, ctr + 1);
+                                if (timing) cudaEventRecord(e2.second, s);
+                                GTS_CUDA(cudaGetLastError());
+                                ++main_launches;
+                                return GTS_OK;
+                            }, &ss));
         ++sweeps;
         if (c->world > 1) {
             if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
@@ -146,15 +144,18 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
             st->finish_s = c->t_finish.sum_s();
         }
         st->pages_processed = (uint64_t)c->dg.n_local * sweeps;
+        st->h2d_bytes = ss.h2d_bytes;
+        if (timing) st->h2d_s = c->t_h2d.sum_s();
         st->edges_traversed = g->m * (uint64_t)sweeps / (uint64_t)c->world;
         st->nccl_bytes = nccl_bytes;
-        st->launches = launches;
+        st->launches = launches + main_launches;
         st->main_kernel_launches = main_launches;
         st->levels_or_iters = sweeps;
     } else if (timing) {
         c->t_main.sum_s();
         c->t_merge.sum_s();
         c->t_finish.sum_s();
+        c->t_h2d.sum_s();
     }
     return GTS_OK;
 }

@@ -214,3 +214,32 @@ def test_graph_switch_and_evict(G, ctx):
     ctx.evict(ga)
     got, st = G.gts_bfs(ctx, ga, 0)
     assert st["upload_s"] > 0 and np.array_equal(got, oracle.bfs(a.row_ptr, a.col, 0))
+
+
+# ----------------------------------------------------------- streamed mode ---
+
+@pytest.mark.parametrize("name", ["fig1", "rmat16_4k", "rmat16_64k", "rmat20", "twitter20", "instar", "bintree"])
+@pytest.mark.parametrize("ring,batch", [(2, 1), (4, 8), (3, 5)])
+def test_streamed_equals_resident_and_oracle(G, ctx, name, ring, batch):
+    """Pages streamed from pinned host memory through a ring of `ring` slots of
+    `batch` pages: integer outputs identical to the resident run and the oracle."""
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
+    kw = dict(residency=G.GTS_STREAMED, ring_slots=ring, batch_pages=batch)
+    src = int(np.argmax(np.diff(g.row_ptr)))
+    want = oracle.bfs(g.row_ptr, g.col, src)
+    got, st = G.gts_bfs(ctx, gr, src, **kw)
+    assert np.array_equal(got, want)
+    res, _ = G.gts_bfs(ctx, gr, src, residency=G.GTS_RESIDENT)
+    assert np.array_equal(got, res)
+    assert st["h2d_bytes"] > 0 and st["h2d_bytes"] % pb == 0
+    got, st = G.gts_wcc(ctx, gr, **kw)
+    assert np.array_equal(got, oracle.wcc(g.row_ptr, g.col))
+    assert st["h2d_bytes"] == st["levels_or_iters"] * gr.stats()["topo_bytes"]
+    got, st = G.gts_pagerank(ctx, gr, 10, 0.85, **kw)
+    _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, "streamed"))
+    assert st["h2d_bytes"] == 10 * gr.stats()["topo_bytes"]
+    w = inputs.edge_weights(g)
+    grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb)
+    got, _ = G.gts_sssp(ctx, grw, src, **kw)
+    assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, src))
