@@ -77,6 +77,13 @@ enum { GTS_RESIDENCY_AUTO = 0, GTS_RESIDENT = 1, GTS_STREAMED = 2 };
 enum { GTS_DANGLING_UNIFORM = 0, GTS_DANGLING_DROP = 1 };
 enum { GTS_OUT_HOST = 0, GTS_OUT_DEVICE = 1 };
 enum { GTS_RUN_TIMING = 1u };   /* gts_run_config.flags: time the main kernels with CUDA events */
+/* gts_page_config.flags: store vertices in descending in-degree order (ties by
+ * VID) inside the pages.  A builder policy, not a different graph: every call
+ * maps its source vertex in and its result out, so callers always see their
+ * own VIDs.  The directory and page bytes of such a graph hold the internal
+ * IDs (gts_graph_order gives the mapping).  Used by the B200 PageRank kernel
+ * to keep the most-updated WA entries contiguous. */
+enum { GTS_BUILD_DEGREE_ORDER = 1u };
 
 #define GTS_UNREACHED 0xFFFFFFFFu
 
@@ -89,7 +96,7 @@ typedef struct {
     uint32_t struct_size;     /* sizeof(gts_page_config) */
     uint32_t page_bytes;      /* power of two, 256 B .. 1 GiB; default (0) = 1 MiB (R14) */
     uint32_t entry_encoding;  /* GTS_ENTRY_VID32 (default) | GTS_ENTRY_PID16_SLOT16 */
-    uint32_t flags;           /* reserved, 0 */
+    uint32_t flags;           /* 0 or GTS_BUILD_DEGREE_ORDER */
 } gts_page_config;
 
 typedef struct {
@@ -101,7 +108,7 @@ typedef struct {
     uint64_t max_outdeg;
     uint32_t weighted, entry_encoding;
     uint32_t n_hot;           /* entries in the hot-destination table (PageRank, DESIGN.md K-PR) */
-    uint32_t reserved;
+    uint32_t ordered;         /* 1 if built with GTS_BUILD_DEGREE_ORDER */
 } gts_graph_stats;
 
 typedef struct gts_graph gts_graph;   /* opaque; owns the host pages + directory (RVT) */
@@ -131,6 +138,9 @@ const uint8_t* gts_graph_pages(const gts_graph* g);
  * Any pointer may be NULL. */
 int gts_graph_directory(const gts_graph* g, uint32_t* start_vid, uint32_t* nslots, uint32_t* kind,
                         int64_t* lp_first, int64_t* lp_last);
+/* For a GTS_BUILD_DEGREE_ORDER graph: internal_of[v] = internal ID of caller VID v
+ * (n entries).  For other graphs the identity.  EINVAL on NULL. */
+int gts_graph_order(const gts_graph* g, uint32_t* internal_of);
 void gts_graph_free(gts_graph* g);
 
 /* ------------------------------------------------------------ contexts --- */

@@ -170,6 +170,55 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
     if (bad_col) return fail(GTS_EINVAL, "col_idx has an entry >= n");
 
     const bool weighted = weights != nullptr;
+    const bool ordered = cfg && (cfg->flags & GTS_BUILD_DEGREE_ORDER);
+    if (cfg && (cfg->flags & ~(uint32_t)GTS_BUILD_DEGREE_ORDER)) return fail(GTS_EINVAL, "unknown page_config flags");
+    // Degree ordering (GTS_BUILD_DEGREE_ORDER): rename vertices by descending
+    // in-degree (ties by VID) and build the pages of the renamed graph.
+    std::vector<uint32_t> new_of_old, old_of_new;
+    std::vector<uint64_t> o_row;
+    std::vector<uint32_t> o_col, o_w;
+    if (ordered) {
+        std::vector<uint32_t> indeg(n, 0);
+        #pragma omp parallel for schedule(static, 1 << 16)
+        for (int64_t k = 0; k < (int64_t)m; ++k) __atomic_fetch_add(&indeg[col_idx[k]], 1u, __ATOMIC_RELAXED);
+        uint32_t maxd = 0;
+        for (uint64_t v = 0; v < n; ++v) maxd = std::max(maxd, indeg[v]);
+        std::vector<uint64_t> bucket((size_t)maxd + 2, 0);
+        for (uint64_t v = 0; v < n; ++v) bucket[maxd - indeg[v] + 1]++;
+        for (size_t b = 1; b < bucket.size(); ++b) bucket[b] += bucket[b - 1];
+        new_of_old.resize(n);
+        old_of_new.resize(n);
+        for (uint64_t v = 0; v < n; ++v) {
+            uint32_t id = (uint32_t)(bucket[maxd - indeg[v]]++);
+            new_of_old[v] = id;
+            old_of_new[id] = (uint32_t)v;
+        }
+        std::vector<uint32_t>().swap(indeg);
+        o_row.resize(n + 1);
+        o_row[0] = 0;
+        for (uint64_t i = 0; i < n; ++i) o_row[i + 1] = o_row[i] + (row_ptr[old_of_new[i] + 1] - row_ptr[old_of_new[i]]);
+        o_col.resize(m);
+        if (weighted) o_w.resize(m);
+        #pragma omp parallel for schedule(dynamic, 1024)
+        for (int64_t i = 0; i < (int64_t)n; ++i) {
+            const uint64_t src = row_ptr[old_of_new[i]], b = o_row[i], len = o_row[i + 1] - b;
+            if (!weighted) {
+                for (uint64_t k = 0; k < len; ++k) o_col[b + k] = new_of_old[col_idx[src + k]];
+                std::sort(o_col.begin() + b, o_col.begin() + b + len);
+            } else {
+                std::vector<std::pair<uint32_t, uint32_t>> e(len);
+                for (uint64_t k = 0; k < len; ++k) e[k] = {new_of_old[col_idx[src + k]], weights[src + k]};
+                std::sort(e.begin(), e.end());
+                for (uint64_t k = 0; k < len; ++k) {
+                    o_col[b + k] = e[k].first;
+                    o_w[b + k] = e[k].second;
+                }
+            }
+        }
+        row_ptr = o_row.data();
+        col_idx = o_col.data();
+        if (weighted) weights = o_w.data();
+    }
     std::vector<PagePlanEntry> plan;
     gts_graph_stats st;
     int rc = plan_pages(n, row_ptr, weighted, pb, enc, plan, &st);
@@ -266,6 +315,11 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
         }
     }
     build_hot_table(*g, col_idx);
+    if (ordered) {
+        g->ordered = true;
+        g->new_of_old = std::move(new_of_old);
+        g->old_of_new = std::move(old_of_new);
+    }
     *out = g;
     return GTS_OK;
 }
@@ -286,7 +340,8 @@ extern "C" int gts_graph_get_stats(const gts_graph* g, gts_graph_stats* out) {
     out->max_outdeg = g->max_outdeg;
     out->weighted = g->weighted ? 1 : 0;
     out->entry_encoding = g->entry_encoding;
-    out->n_hot = g->n_hot;
+    out->n_hot = g->ordered ? (uint32_t)std::min<uint64_t>(g->n, kHotDense) : g->n_hot;
+    out->ordered = g->ordered ? 1 : 0;
     return GTS_OK;
 }
 
@@ -302,5 +357,14 @@ extern "C" int gts_graph_directory(const gts_graph* g, uint32_t* start_vid, uint
     if (kind) std::memcpy(kind, g->kind.data(), P * 4);
     if (lp_first) std::memcpy(lp_first, g->lp_first.data(), P * 8);
     if (lp_last) std::memcpy(lp_last, g->lp_last.data(), P * 8);
+    return GTS_OK;
+}
+
+extern "C" int gts_graph_order(const gts_graph* g, uint32_t* internal_of) {
+    clear_error();
+    if (!g || !internal_of) return fail(GTS_EINVAL, "NULL argument");
+    if (g->ordered) std::memcpy(internal_of, g->new_of_old.data(), g->n * 4);
+    else
+        for (uint64_t v = 0; v < g->n; ++v) internal_of[v] = (uint32_t)v;
     return GTS_OK;
 }

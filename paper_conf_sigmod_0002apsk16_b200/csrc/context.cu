@@ -103,6 +103,8 @@ static void free_devgraph(DevGraph& d) {
     cudaFree(d.loc);
     cudaFree(d.local_list);
     cudaFree(d.hot_keys);
+    cudaFree(d.new_of_old);
+    cudaFree(d.old_of_new);
     d = DevGraph();
 }
 
@@ -131,6 +133,7 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
         partition(g, strategy, c->world, d.h_owner, vrange);
         d.vlo = vrange[c->rank];
         d.vhi = vrange[c->rank + 1];
+        d.h_vrange = vrange;
         const uint64_t P = g->num_pages;
         std::vector<uint32_t> loc(P, UINT32_MAX);
         d.h_local_list.clear();
@@ -153,6 +156,12 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
             GTS_CUDA(cudaMemcpyAsync(d.local_list, d.h_local_list.data(), d.n_local * 4ull, cudaMemcpyHostToDevice,
                                      c->stream));
         GTS_CUDA(cudaMemcpyAsync(d.hot_keys, g->hot_keys.data(), kHotSlots * 4, cudaMemcpyHostToDevice, c->stream));
+        if (g->ordered) {
+            GTS_CUDA(cudaMalloc(&d.new_of_old, g->n * 4));
+            GTS_CUDA(cudaMalloc(&d.old_of_new, g->n * 4));
+            GTS_CUDA(cudaMemcpyAsync(d.new_of_old, g->new_of_old.data(), g->n * 4, cudaMemcpyHostToDevice, c->stream));
+            GTS_CUDA(cudaMemcpyAsync(d.old_of_new, g->old_of_new.data(), g->n * 4, cudaMemcpyHostToDevice, c->stream));
+        }
         GTS_CUDA(cudaStreamSynchronize(c->stream));   // host vectors above are temporaries
     }
     DevGraph& d = c->dg;
@@ -230,7 +239,11 @@ int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* 
     if (d.residency > GTS_STREAMED) return fail(GTS_EINVAL, "unknown residency %u", d.residency);
     if (d.out_location > GTS_OUT_DEVICE) return fail(GTS_EINVAL, "unknown out_location %u", d.out_location);
     if (d.ring_slots == 0) d.ring_slots = 4;
-    if (d.batch_pages == 0) d.batch_pages = 8;
+    if (d.batch_pages == 0) {   // >= 64 MiB per batch: enough pages in flight to keep the link busy
+        const uint32_t pb = g->page_bytes;
+        d.batch_pages = pb >= (64u << 20) ? 1u : std::max(8u, (64u << 20) / pb);
+        d.batch_pages = std::min<uint32_t>(d.batch_pages, 256);
+    }
     if (d.ring_slots > 32) return fail(GTS_EINVAL, "ring_slots must be <= 32");
     *out = d;
     cudaError_t e = cudaSetDevice(ctx->device);
@@ -238,13 +251,99 @@ int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* 
     return GTS_OK;
 }
 
+// Result D2H (Alg 1 line 28, "copy WA back").  Device outputs: one D2D copy.
+// Pinned host outputs: one DMA.  Pageable host outputs: DMA into two pinned
+// staging chunks, each drained by a parallel host memcpy while the next chunk
+// is in flight (a plain cudaMemcpy to pageable memory runs at a few GB/s).
 int copy_out(Context* c, const void* dsrc, void* dst, size_t bytes, uint32_t out_location) {
     if (bytes == 0) return GTS_OK;
-    GTS_CUDA(cudaMemcpyAsync(dst, dsrc, bytes,
-                             out_location == GTS_OUT_DEVICE ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
-                             c->stream));
-    GTS_CUDA(cudaStreamSynchronize(c->stream));
+    if (out_location == GTS_OUT_DEVICE) {
+        GTS_CUDA(cudaMemcpyAsync(dst, dsrc, bytes, cudaMemcpyDeviceToDevice, c->stream));
+        GTS_CUDA(cudaStreamSynchronize(c->stream));
+        return GTS_OK;
+    }
+    cudaPointerAttributes pa;
+    bool pinned = cudaPointerGetAttributes(&pa, dst) == cudaSuccess && pa.type == cudaMemoryTypeHost;
+    cudaGetLastError();
+    if (pinned || bytes <= (1u << 20)) {
+        GTS_CUDA(cudaMemcpyAsync(dst, dsrc, bytes, cudaMemcpyDeviceToHost, c->stream));
+        GTS_CUDA(cudaStreamSynchronize(c->stream));
+        return GTS_OK;
+    }
+    const size_t chunk = 32u << 20;
+    if (!c->h_stage) GTS_CUDA(cudaMallocHost(&c->h_stage, 2 * chunk));
+    if (!c->stage_ev[0]) {
+        GTS_CUDA(cudaEventCreateWithFlags(&c->stage_ev[0], cudaEventDisableTiming));
+        GTS_CUDA(cudaEventCreateWithFlags(&c->stage_ev[1], cudaEventDisableTiming));
+    }
+    const uint8_t* src = static_cast<const uint8_t*>(dsrc);
+    uint8_t* out = static_cast<uint8_t*>(dst);
+    const size_t nchunks = (bytes + chunk - 1) / chunk;
+    auto issue = [&](size_t k) -> int {
+        const size_t off = k * chunk, len = std::min(chunk, bytes - off);
+        GTS_CUDA(cudaMemcpyAsync(c->h_stage + (k & 1) * chunk, src + off, len, cudaMemcpyDeviceToHost, c->stream));
+        GTS_CUDA(cudaEventRecord(c->stage_ev[k & 1], c->stream));
+        return GTS_OK;
+    };
+    GTS_TRY(issue(0));
+    for (size_t k = 0; k < nchunks; ++k) {
+        if (k + 1 < nchunks) GTS_TRY(issue(k + 1));
+        GTS_CUDA(cudaEventSynchronize(c->stage_ev[k & 1]));
+        const size_t off = k * chunk, len = std::min(chunk, bytes - off);
+        const uint8_t* st = c->h_stage + (k & 1) * chunk;
+        const int T = 8;
+        #pragma omp parallel for num_threads(T) schedule(static)
+        for (int t = 0; t < T; ++t) {
+            const size_t a = len * t / T, b = len * (t + 1) / T;
+            std::memcpy(out + off + a, st + a, b - a);
+        }
+    }
     return GTS_OK;
+}
+
+__global__ void gather_kernel(uint32_t* out, const uint32_t* __restrict__ vals, const uint32_t* __restrict__ idx,
+                              uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) out[v] = vals[idx[v]];
+}
+
+__global__ void label_min_kernel(uint32_t* minorig, const uint32_t* __restrict__ label,
+                                 const uint32_t* __restrict__ old_of_new, uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
+        atomicMin(minorig + label[i], old_of_new[i]);
+}
+
+__global__ void label_map_kernel(uint32_t* tmp, const uint32_t* __restrict__ label, const uint32_t* __restrict__ minorig,
+                                 uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) tmp[i] = minorig[label[i]];
+}
+
+int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_t out_location, bool labels) {
+    const uint64_t n = g->n;
+    if (!g->ordered) return copy_out(c, vals, out, n * 4, out_location);
+    const int eg = c->num_sms * 4;
+    const uint32_t* src = vals;
+    if (labels) {             // internal min-ID label -> min caller VID of the component
+        uint32_t *minorig, *tmp;
+        GTS_TRY(c->buf(70, n * 4, (void**)&minorig));
+        GTS_TRY(c->buf(71, n * 4, (void**)&tmp));
+        GTS_CUDA(cudaMemsetAsync(minorig, 0xFF, n * 4, c->stream));
+        label_min_kernel<<<eg, 256, 0, c->stream>>>(minorig, vals, c->dg.old_of_new, n);
+        label_map_kernel<<<eg, 256, 0, c->stream>>>(tmp, vals, minorig, n);
+        src = tmp;
+    }
+    uint32_t* dst;
+    if (out_location == GTS_OUT_DEVICE) dst = static_cast<uint32_t*>(out);
+    else GTS_TRY(c->buf(72, n * 4, (void**)&dst));
+    gather_kernel<<<eg, 256, 0, c->stream>>>(dst, src, c->dg.new_of_old, n);
+    GTS_CUDA(cudaGetLastError());
+    if (out_location == GTS_OUT_DEVICE) {
+        GTS_CUDA(cudaStreamSynchronize(c->stream));
+        return GTS_OK;
+    }
+    return copy_out(c, dst, out, n * 4, out_location);
 }
 
 int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid) {
@@ -329,6 +428,9 @@ extern "C" void gts_context_free(gts_context* c) {
         }
     if (c->comm) ncclCommDestroy(c->comm);
     cudaFreeHost(c->h_small);
+    if (c->h_stage) cudaFreeHost(c->h_stage);
+    for (cudaEvent_t e : c->stage_ev)
+        if (e) cudaEventDestroy(e);
     cudaStreamDestroy(c->own_stream);
     cudaStreamDestroy(c->copy_stream);
     delete c;

@@ -37,6 +37,8 @@ constexpr uint32_t kHotSlots = kHotBuckets * kHotWays;
 constexpr uint32_t kHotMax = 4096;          // load factor 0.5
 constexpr uint32_t kHotMinIndeg = 64;
 constexpr uint32_t kHotEmpty = 0xFFFFFFFFu;
+// Degree-ordered graphs: the hot set is simply internal IDs [0, kHotDense).
+constexpr uint32_t kHotDense = 24576;
 
 GTS_HD uint32_t hot_h1(uint32_t v) { return (v * 0x9E3779B1u) >> 21; }
 GTS_HD uint32_t hot_h2(uint32_t v) { return ((v ^ (v >> 15)) * 0x85EBCA77u) >> 21; }
@@ -57,6 +59,9 @@ struct Graph {
     std::vector<uint32_t> hot_keys;    // kHotSlots entries, kHotEmpty when free
     uint32_t n_hot = 0;
     uint64_t uid = 0;                  // process-unique id (device cache key)
+    bool ordered = false;              // GTS_BUILD_DEGREE_ORDER: pages hold internal IDs
+    std::vector<uint32_t> new_of_old;  // caller VID -> internal ID (ordered graphs)
+    std::vector<uint32_t> old_of_new;  // internal ID -> caller VID
     bool host_registered = false;      // cudaHostRegister'ed by a context
 };
 

@@ -22,6 +22,7 @@
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <cstdlib>
 #include <cstring>
 
 #include "expand.cuh"
@@ -33,15 +34,21 @@ namespace gts {
 // Per-thread destination emitter: combines runs of equal destinations (rows
 // are sorted), routes hot destinations to the CTA's shared-memory partial sums
 // and everything else to a fire-and-forget fp32 red.add into acc.
+template <bool kDense>
 struct PrEmitter {
     float* acc;
-    const uint32_t* hkeys;   // shared memory, kHotSlots
-    float* hacc;             // shared memory, kHotSlots
+    const uint32_t* hkeys;   // shared memory, kHotSlots (hash-table mode)
+    float* hacc;             // shared memory, kHotSlots (hash) or kHotDense (dense) partial sums
     uint32_t last;
     float sum;
     bool has;
 
     __device__ __forceinline__ void emit(uint32_t dst, float c) {
+        if (kDense) {                                   // degree-ordered graph: hot = [0, kHotDense)
+            if (dst < kHotDense) atomicAdd(hacc + dst, c);
+            else atomicAdd(acc + dst, c);
+            return;
+        }
         uint32_t b = hot_h1(dst);
         uint4 k = reinterpret_cast<const uint4*>(hkeys)[b];
         int way = k.x == dst ? 0 : k.y == dst ? 1 : k.z == dst ? 2 : k.w == dst ? 3 : -1;
@@ -70,6 +77,7 @@ struct PrEmitter {
 };
 
 constexpr size_t kPrDynSmem = kHotSlots * (sizeof(uint32_t) + sizeof(float));
+constexpr size_t kPrDynSmemDense = kHotDense * sizeof(float);
 constexpr int kPrUnroll = 4;            // 16-byte loads in flight per thread
 
 struct PrSmem {
@@ -87,24 +95,28 @@ __device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const ui
 // packed in VID order from offset 0), streamed with 16-byte evict_first loads,
 // kPrUnroll in flight per thread; the owner of each 4-word group is found by a
 // binary search over the tile's record offsets in shared memory.
-template <bool kWeighted>
+template <bool kWeighted, bool kDense>
 __global__ void __launch_bounds__(kThreads, 2)
 pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__ hot_keys,
-                  float d, double* dang_out, uint32_t* work_ctr) {
+                  float d, double* dang_out, uint32_t* work_ctr, uint32_t n_dense) {
     __shared__ PrSmem sm;
     extern __shared__ uint4 dyn_smem[];
     uint32_t* hkeys = reinterpret_cast<uint32_t*>(dyn_smem);
-    float* hacc = reinterpret_cast<float*>(hkeys + kHotSlots);
+    float* hacc = kDense ? reinterpret_cast<float*>(dyn_smem) : reinterpret_cast<float*>(hkeys + kHotSlots);
     const int tid = threadIdx.x;
-    for (uint32_t i = tid; i < kHotSlots; i += kThreads) {
-        hkeys[i] = __ldg(hot_keys + i);
-        hacc[i] = 0.f;
+    if (kDense) {
+        for (uint32_t i = tid; i < kHotDense; i += kThreads) hacc[i] = 0.f;
+    } else {
+        for (uint32_t i = tid; i < kHotSlots; i += kThreads) {
+            hkeys[i] = __ldg(hot_keys + i);
+            hacc[i] = 0.f;
+        }
     }
     const uint64_t pol = policy_evict_first();
     const uint32_t count = ps.count;
     const uint32_t enc = ps.entry_encoding;
     constexpr uint32_t wshift = kWeighted ? 1 : 0;
-    PrEmitter em{acc, hkeys, hacc, 0u, 0.f, false};
+    PrEmitter<kDense> em{acc, hkeys, hacc, 0u, 0.f, false};
     double dang = 0.0;
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
@@ -210,10 +222,17 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
         em.flush();
     }
     __syncthreads();
-    for (uint32_t i = tid; i < kHotSlots; i += kThreads) {
-        const uint32_t k = hkeys[i];
-        const float v = hacc[i];
-        if (k != kHotEmpty && v != 0.f) atomicAdd(acc + k, v);
+    if (kDense) {
+        for (uint32_t i = tid; i < n_dense; i += kThreads) {
+            const float v = hacc[i];
+            if (v != 0.f) atomicAdd(acc + i, v);
+        }
+    } else {
+        for (uint32_t i = tid; i < kHotSlots; i += kThreads) {
+            const uint32_t k = hkeys[i];
+            const float v = hacc[i];
+            if (k != kHotEmpty && v != 0.f) atomicAdd(acc + k, v);
+        }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) dang += __shfl_down_sync(0xFFFFFFFFu, dang, o);
@@ -228,24 +247,35 @@ __global__ void pr_init_kernel(float* x, float* acc, uint64_t n, float v0) {
     }
 }
 
-// x_v <- (1-d)/n + d*D/n + acc_v ; acc_v <- 0  (float4 vectorised; buffers are 256-B aligned)
-__global__ void pr_finish_kernel(float* x, float* acc, uint64_t n, double d, const double* dang, double* dang_reset,
-                                 int uniform) {
+// x_v <- (1-d)/n + d*D/n + acc_v ; acc_v <- 0  for v in [lo, hi) (float4 vectorised where aligned).
+// Strategy-S ranks finish only their own WA range and zero the rest of acc.
+__global__ void pr_finish_kernel(float* x, float* acc, uint64_t n, uint64_t lo, uint64_t hi, double d,
+                                 const double* dang, double* dang_reset, int uniform) {
     const double D = *dang;
     const float base = (float)((1.0 - d) / (double)n + (uniform ? d * D / (double)n : 0.0));
-    const uint64_t n4 = n / 4;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    float4* x4 = reinterpret_cast<float4*>(x);
-    float4* a4 = reinterpret_cast<float4*>(acc);
+    const uint64_t t0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
-        float4 a = a4[i];
+    uint64_t a4 = (lo + 3) / 4, b4 = hi / 4;            // aligned float4 span inside [lo, hi)
+    if (b4 < a4) b4 = a4;
+    float4* x4 = reinterpret_cast<float4*>(x);
+    float4* acc4 = reinterpret_cast<float4*>(acc);
+    for (uint64_t i = a4 + t0; i < b4; i += stride) {
+        const float4 a = acc4[i];
         x4[i] = make_float4(base + a.x, base + a.y, base + a.z, base + a.w);
-        a4[i] = z;
+        acc4[i] = z;
     }
-    for (uint64_t i = n4 * 4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-        x[i] = base + acc[i];
-        acc[i] = 0.f;
+    if (t0 < 8) {                                       // unaligned head [lo, 4*a4) and tail [4*b4, hi)
+        const uint64_t i = t0 < 4 ? lo + t0 : 4 * b4 + (t0 - 4);
+        const bool ok = t0 < 4 ? (i < 4 * a4 && i < hi) : (i < hi && i >= 4 * a4);
+        if (ok) {
+            x[i] = base + acc[i];
+            acc[i] = 0.f;
+        }
+    }
+    if (lo > 0 || hi < n) {                             // zero acc outside my range (S)
+        for (uint64_t i = t0; i < n; i += stride)
+            if (i < lo || i >= hi) acc[i] = 0.f;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *dang_reset = 0.0;
 }
@@ -265,9 +295,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     if (!rank_out) return fail(GTS_EINVAL, "NULL output");
     if (!(damping >= 0.0 && damping <= 1.0)) return fail(GTS_EINVAL, "damping must be in [0,1]");
     if (dangling > GTS_DANGLING_DROP) return fail(GTS_EINVAL, "unknown dangling mode %u", dangling);
-    if (rc.strategy == GTS_STRATEGY_S && c->world > 1) return fail(GTS_EUNSUPPORTED, "Strategy-S PageRank not available yet");
     const uint64_t n = g->n;
     const bool streamed = choose_streamed(c, g, rc, 8 * n);
+    const bool strat_s = rc.strategy == GTS_STRATEGY_S && c->world > 1;
     double upload_s = 0;
     GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
     const bool timing = rc.flags & GTS_RUN_TIMING;
@@ -279,10 +309,35 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     GTS_TRY(c->buf(kBufDang, 2 * sizeof(double), (void**)&dang));
     GTS_TRY(c->buf(kBufPrCtr, 4, (void**)&ctr));
     cudaStream_t s = c->stream;
-    auto kern = g->weighted ? pr_scatter_kernel<true> : pr_scatter_kernel<false>;
-    GTS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPrDynSmem));
+    auto kern = g->ordered ? (g->weighted ? pr_scatter_kernel<true, true> : pr_scatter_kernel<false, true>)
+                           : (g->weighted ? pr_scatter_kernel<true, false> : pr_scatter_kernel<false, false>);
+    const size_t dyn = g->ordered ? kPrDynSmemDense : kPrDynSmem;
+    const uint32_t n_dense = (uint32_t)std::min<uint64_t>(n, kHotDense);
+    GTS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
     int grid = 0;
-    GTS_TRY(sms_grid(c, (const void*)kern, kThreads, kPrDynSmem, &grid));
+    GTS_TRY(sms_grid(c, (const void*)kern, kThreads, dyn, &grid));
+    // Optional L2 persistence for the hot head of WA (ordered graphs: the most
+    // updated entries are acc[0, W)).  GTS_L2_PERSIST=<MiB> enables it.
+    bool persist = false;
+    if (g->ordered && getenv("GTS_L2_PERSIST")) {
+        size_t want = (size_t)atol(getenv("GTS_L2_PERSIST")) << 20;
+        cudaDeviceProp prop;
+        GTS_CUDA(cudaGetDeviceProperties(&prop, c->device));
+        want = std::min<size_t>(want, prop.persistingL2CacheMaxSize);
+        want = std::min<size_t>(want, n * 4);
+        if (want > 0) {
+            GTS_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
+            cudaStreamAttrValue at;
+            std::memset(&at, 0, sizeof(at));
+            at.accessPolicyWindow.base_ptr = acc;
+            at.accessPolicyWindow.num_bytes = std::min<size_t>(want, prop.accessPolicyMaxWindowSize);
+            at.accessPolicyWindow.hitRatio = 1.0f;
+            at.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+            at.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+            GTS_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &at));
+            persist = true;
+        }
+    }
     const int eg = c->num_sms * 4;
     pr_init_kernel<<<eg, 256, 0, s>>>(x, acc, n, (float)(1.0 / (double)n));
     GTS_CUDA(cudaMemsetAsync(dang, 0, 2 * sizeof(double), s));
@@ -297,8 +352,8 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                                 GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
                                 std::pair<cudaEvent_t, cudaEvent_t> e2;
                                 if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
-                                kern<<<std::min(grid, cap), kThreads, kPrDynSmem, s>>>(ps, x, acc, c->dg.hot_keys,
-                                                                                     (float)damping, D, ctr);
+                                kern<<<std::min(grid, cap), kThreads, dyn, s>>>(ps, x, acc, c->dg.hot_keys,
+                                                                              (float)damping, D, ctr, n_dense);
                                 if (timing) cudaEventRecord(e2.second, s);
                                 GTS_CUDA(cudaGetLastError());
                                 ++main_launches;
@@ -307,21 +362,45 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         if (c->world > 1) {
             if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
             GTS_NCCL(ncclGroupStart());
-            GTS_NCCL(ncclAllReduce(acc, acc, n, ncclFloat32, ncclSum, c->comm, s));
+            if (strat_s) {      // Strategy-S: rank r receives the sum of WA over its own range only
+                const std::vector<uint64_t>& vr = c->dg.h_vrange;
+                for (int r = 0; r < c->world; ++r)
+                    if (vr[r + 1] > vr[r])
+                        GTS_NCCL(ncclReduce(acc + vr[r], acc + vr[r], vr[r + 1] - vr[r], ncclFloat32, ncclSum, r,
+                                            c->comm, s));
+            } else {            // Strategy-P: every replica receives the full sum
+                GTS_NCCL(ncclAllReduce(acc, acc, n, ncclFloat32, ncclSum, c->comm, s));
+            }
             GTS_NCCL(ncclAllReduce(D, D, 1, ncclFloat64, ncclSum, c->comm, s));
             GTS_NCCL(ncclGroupEnd());
             if (timing) cudaEventRecord(ev.second, s);
             nccl_bytes += n * 4 + 8;
         }
         if (timing) { ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
-        pr_finish_kernel<<<eg, 256, 0, s>>>(x, acc, n, damping, D, dang + ((it + 1) & 1),
-                                             dangling == GTS_DANGLING_UNIFORM ? 1 : 0);
+        pr_finish_kernel<<<eg, 256, 0, s>>>(x, acc, n, strat_s ? c->dg.vlo : 0, strat_s ? c->dg.vhi : n, damping, D,
+                                             dang + ((it + 1) & 1), dangling == GTS_DANGLING_UNIFORM ? 1 : 0);
         if (timing) cudaEventRecord(ev.second, s);
         ++launches;
     }
     launches += main_launches;
+    if (persist) {
+        cudaStreamAttrValue at;
+        std::memset(&at, 0, sizeof(at));
+        at.accessPolicyWindow.num_bytes = 0;
+        GTS_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &at));
+        GTS_CUDA(cudaCtxResetPersistingL2Cache());
+    }
+    if (strat_s) {              // gather every rank's finished range so all ranks return the full vector
+        GTS_NCCL(ncclGroupStart());
+        const std::vector<uint64_t>& vr = c->dg.h_vrange;
+        for (int r = 0; r < c->world; ++r)
+            if (vr[r + 1] > vr[r])
+                GTS_NCCL(ncclBroadcast(x + vr[r], x + vr[r], vr[r + 1] - vr[r], ncclFloat32, r, c->comm, s));
+        GTS_NCCL(ncclGroupEnd());
+        nccl_bytes += n * 4;
+    }
     GTS_CUDA(cudaGetLastError());
-    GTS_TRY(copy_out(c, x, rank_out, n * 4, rc.out_location));
+    GTS_TRY(deliver(c, g, reinterpret_cast<const uint32_t*>(x), rank_out, rc.out_location, false));
     if (st) {
         std::memset(st, 0, sizeof(*st));
         st->wall_s = now_s() - t_start;

@@ -65,12 +65,15 @@ struct DevGraph {
     uint32_t* loc = nullptr;           // [num_pages] local index or UINT32_MAX
     uint32_t* local_list = nullptr;    // [n_local] global page ids owned by this rank
     uint32_t* hot_keys = nullptr;      // [kHotSlots]
+    uint32_t* new_of_old = nullptr;    // ordered graphs: caller VID -> internal ID  [n]
+    uint32_t* old_of_new = nullptr;    // ordered graphs: internal ID -> caller VID  [n]
     uint32_t n_local = 0;
     bool all_local = true;             // every page is local and loc == identity
     bool resident = false;             // pages uploaded
     std::vector<uint32_t> h_local_list;
     std::vector<int32_t> h_owner;
     uint64_t vlo = 0, vhi = 0;         // Strategy-S WA range of this rank
+    std::vector<uint64_t> h_vrange;    // all ranks' WA ranges (world + 1)
 };
 
 struct Timer {               // event pairs around launches; summed after the call synchronises
@@ -89,6 +92,8 @@ struct Context {
     std::vector<DevGraph> parked;  // other graphs kept resident (evicted LRU-first under memory pressure)
     std::vector<std::pair<void*, size_t>> scratch;
     void* h_small = nullptr;   // pinned host scratch (4 KiB)
+    uint8_t* h_stage = nullptr;          // pinned D2H staging (2 x 32 MiB) for pageable outputs
+    cudaEvent_t stage_ev[2] = {nullptr, nullptr};
     Timer t_main, t_finish, t_merge, t_h2d;
     cudaEvent_t ring_ready[64], ring_free[64];
     bool ring_events = false;
@@ -101,6 +106,11 @@ struct Context {
 int ensure_graph(Context* c, const Graph* g, uint32_t strategy, bool need_resident, double* upload_s);
 int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* cfg, gts_run_config* out);
 int copy_out(Context* c, const void* dsrc, void* dst, size_t bytes, uint32_t out_location);
+// Result of a call (internal IDs for ordered graphs) -> caller's buffer in caller VIDs.
+// labels = true: the values are themselves internal VIDs (WCC) and are renamed to
+// the minimum caller VID of their component.
+int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_t out_location, bool labels);
+inline uint64_t map_src(const Graph* g, uint64_t src) { return g->ordered ? g->new_of_old[src] : src; }
 int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid);
 int pinned_register(Graph* g);
 // residency decision (GTS_RESIDENCY_AUTO: resident iff this rank's pages + attributes fit in free HBM)

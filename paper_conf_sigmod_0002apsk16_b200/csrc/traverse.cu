@@ -268,8 +268,6 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     if (!out) return fail(GTS_EINVAL, "NULL output");
     if (src >= g->n) return fail(GTS_EINVAL, "src %llu >= n %llu", (unsigned long long)src, (unsigned long long)g->n);
     if (algo == kSSSP && !g->weighted) return fail(GTS_EUNSUPPORTED, "gts_sssp needs a graph built with weights");
-    if (rc.strategy == GTS_STRATEGY_S && c->world > 1)
-        return fail(GTS_EUNSUPPORTED, "Strategy-S traversal not available yet");
     const uint64_t n = g->n, words = (n + 31) / 32;
     const bool streamed = choose_streamed(c, g, rc, 4 * n + 16 * words);
     double upload_s = 0;
@@ -290,6 +288,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     GTS_CUDA(cudaMemsetAsync(cur, 0, words * 4, s));
     GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
     GTS_CUDA(cudaMemsetAsync(ctr, 0, sizeof(Counters), s));
+    src = map_src(g, src);
     set_source_kernel<<<1, 1, 0, s>>>(value, visited, cur, src);
     uint64_t launches = 1, main_launches = 0;
     std::vector<uint32_t> l0 = pages_of_vertex(g, c->dg, c->rank, src);
@@ -390,7 +389,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         GTS_CUDA(cudaStreamSynchronize(s));
         if (bad) return fail(GTS_EOVERFLOW, "an SSSP distance reaches 2^32-1");
     }
-    GTS_TRY(copy_out(c, value, out, n * 4, rc.out_location));
+    GTS_TRY(deliver(c, g, value, out, rc.out_location, false));
     if (st) {
         std::memset(st, 0, sizeof(*st));
         st->wall_s = now_s() - t_start;

@@ -82,7 +82,6 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     gts_run_config rc;
     GTS_TRY(validate_common(c, g, cfg, &rc));
     if (!label_out) return fail(GTS_EINVAL, "NULL output");
-    if (rc.strategy == GTS_STRATEGY_S && c->world > 1) return fail(GTS_EUNSUPPORTED, "Strategy-S WCC not available yet");
     const uint64_t n = g->n;
     const bool streamed = choose_streamed(c, g, rc, 4 * n);
     double upload_s = 0;
@@ -133,7 +132,7 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
         GTS_CUDA(cudaStreamSynchronize(s));
         if (hs[0] == 0) break;
     }
-    GTS_TRY(copy_out(c, label, label_out, n * 4, rc.out_location));
+    GTS_TRY(deliver(c, g, label, label_out, rc.out_location, true));
     if (st) {
         std::memset(st, 0, sizeof(*st));
         st->wall_s = now_s() - t_start;

@@ -29,10 +29,11 @@ GTS_RESIDENCY_AUTO, GTS_RESIDENT, GTS_STREAMED = 0, 1, 2
 GTS_DANGLING_UNIFORM, GTS_DANGLING_DROP = 0, 1
 GTS_OUT_HOST, GTS_OUT_DEVICE = 0, 1
 GTS_RUN_TIMING = 1
+GTS_BUILD_DEGREE_ORDER = 1
 GTS_UNREACHED = 0xFFFFFFFF
 
 EXPORTED = ["gts_last_error", "gts_version", "gts_build_pages", "gts_plan_pages", "gts_graph_get_stats",
-            "gts_graph_pages", "gts_graph_directory", "gts_graph_free", "gts_get_unique_id",
+            "gts_graph_pages", "gts_graph_directory", "gts_graph_order", "gts_graph_free", "gts_get_unique_id",
             "gts_context_create", "gts_context_free", "gts_context_evict", "gts_context_set_stream",
             "gts_bfs", "gts_pagerank", "gts_sssp", "gts_wcc", "gts_partition_pages"]
 
@@ -51,10 +52,10 @@ class PageConfig(ctypes.Structure):
 class GraphStats(ctypes.Structure):
     _fields_ = [(k, ctypes.c_uint64) for k in ("n", "m", "num_pages", "n_sp", "n_lp", "n_lp_vertices",
                                                "page_bytes", "topo_bytes", "used_bytes", "max_outdeg")] + \
-               [(k, ctypes.c_uint32) for k in ("weighted", "entry_encoding", "n_hot", "reserved")]
+               [(k, ctypes.c_uint32) for k in ("weighted", "entry_encoding", "n_hot", "ordered")]
 
     def as_dict(self):
-        return {k: getattr(self, k) for k, _ in self._fields_ if k != "reserved"}
+        return {k: getattr(self, k) for k, _ in self._fields_}
 
 
 class RunConfig(ctypes.Structure):
@@ -83,6 +84,7 @@ _sig = {
     "gts_graph_get_stats": (_i32, [_vp, ctypes.POINTER(GraphStats)]),
     "gts_graph_pages": (_vp, [_vp]),
     "gts_graph_directory": (_i32, [_vp, _vp, _vp, _vp, _vp, _vp]),
+    "gts_graph_order": (_i32, [_vp, _vp]),
     "gts_graph_free": (None, [_vp]),
     "gts_get_unique_id": (_i32, [_vp]),
     "gts_context_create": (_i32, [_i32, _i32, _i32, _vp, ctypes.POINTER(_vp)]),
@@ -119,8 +121,9 @@ def gts_last_error():
     return _lib.gts_last_error().decode(errors="replace")
 
 
-def _page_config(page_bytes, entry_encoding):
-    return PageConfig(ctypes.sizeof(PageConfig), int(page_bytes), int(entry_encoding), 0)
+def _page_config(page_bytes, entry_encoding, order=False):
+    return PageConfig(ctypes.sizeof(PageConfig), int(page_bytes), int(entry_encoding),
+                      GTS_BUILD_DEGREE_ORDER if order else 0)
 
 
 class Graph:
@@ -157,6 +160,12 @@ class Graph:
                                         _np_ptr(ll)))
         return {"start_vid": sv, "nslots": ns, "kind": kd, "lp_first": lf, "lp_last": ll}
 
+    def order(self):
+        """internal_of[v]: internal ID of caller VID v (identity unless built with order=True)."""
+        a = np.empty(self.n, np.uint32)
+        _check(_lib.gts_graph_order(self.handle, _np_ptr(a)))
+        return a
+
     def free(self):
         if self._h is not None:
             _lib.gts_graph_free(self._h)
@@ -169,14 +178,14 @@ class Graph:
             pass
 
 
-def gts_build_pages(row_ptr, col_idx, weights=None, page_bytes=1 << 20, entry_encoding=GTS_ENTRY_VID32):
+def gts_build_pages(row_ptr, col_idx, weights=None, page_bytes=1 << 20, entry_encoding=GTS_ENTRY_VID32, order=False):
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.uint64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.uint32)
     if weights is not None:
         weights = np.ascontiguousarray(weights, dtype=np.uint32)
     n = row_ptr.shape[0] - 1
     m = col_idx.shape[0]
-    cfg = _page_config(page_bytes, entry_encoding)
+    cfg = _page_config(page_bytes, entry_encoding, order)
     h = ctypes.c_void_p()
     _check(_lib.gts_build_pages(n, m, _np_ptr(row_ptr), _np_ptr(col_idx), _np_ptr(weights), ctypes.byref(cfg),
                                 ctypes.byref(h)))

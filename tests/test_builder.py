@@ -175,3 +175,27 @@ def test_hot_table_holds_top_in_degree():
     indeg = np.bincount(g.col, minlength=g.n)
     # at least the 1,000 hottest vertices have in-degree >= 64 and must all be in the table
     assert st["n_hot"] >= 1000
+
+
+def test_degree_order_build():
+    """GTS_BUILD_DEGREE_ORDER: pages hold the graph renamed by descending in-degree."""
+    g = inputs.rmat(13).with_weights()
+    gr = G.gts_build_pages(g.row_ptr, g.col, g.weights, page_bytes=8192, order=True)
+    st = gr.stats()
+    assert st["ordered"] == 1
+    p = gr.order()
+    assert np.array_equal(np.sort(p), np.arange(g.n))
+    indeg = np.bincount(g.col, minlength=g.n)
+    assert np.all(np.diff(indeg[np.argsort(p)]) <= 0)           # internal order = descending in-degree
+    assert np.array_equal(p, inputs.indegree_order(g))
+    h = inputs.permute(g, p)
+    rp, col, w = oracle.decode_pages(gr.pages(), 8192, g.n, g.m, weighted=True)
+    assert np.array_equal(rp, h.row_ptr) and np.array_equal(col, h.col)
+    # weights travel with their edges: compare (src, dst, w) multisets
+    src = np.repeat(np.arange(g.n), np.diff(g.row_ptr).astype(np.int64))
+    a = sorted(zip(p[src].tolist(), p[g.col].tolist(), g.weights.tolist()))
+    src2 = np.repeat(np.arange(g.n), np.diff(rp).astype(np.int64))
+    b = sorted(zip(src2.tolist(), col.tolist(), w.tolist()))
+    assert a == b
+    plain = G.gts_build_pages(g.row_ptr, g.col, page_bytes=8192)
+    assert np.array_equal(plain.order(), np.arange(g.n))

@@ -243,3 +243,38 @@ def test_streamed_equals_resident_and_oracle(G, ctx, name, ring, batch):
     grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb)
     got, _ = G.gts_sssp(ctx, grw, src, **kw)
     assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, src))
+
+
+# ------------------------------------------------------ degree-ordered pages ---
+
+@pytest.mark.parametrize("name", ["fig1", "multi", "rmat16_4k", "rmat16_1m", "rmat20", "twitter20", "instar", "path"])
+@pytest.mark.parametrize("residency", ["resident", "streamed"])
+def test_degree_ordered_graph(G, ctx, name, residency):
+    """Pages built with GTS_BUILD_DEGREE_ORDER: every result is in the caller's VIDs
+    and equals the oracle on the original graph."""
+    g, pb = graph(name)
+    kw = {} if residency == "resident" else dict(residency=G.GTS_STREAMED, ring_slots=3, batch_pages=4)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+    for src in _sources(g)[:2]:
+        got, _ = G.gts_bfs(ctx, gr, src, **kw)
+        assert np.array_equal(got, oracle.bfs(g.row_ptr, g.col, src))
+    got, _ = G.gts_wcc(ctx, gr, **kw)
+    assert np.array_equal(got, oracle.wcc(g.row_ptr, g.col))
+    got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, **kw)
+    _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, "ordered"))
+    w = inputs.edge_weights(g)
+    grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb, order=True)
+    got, _ = G.gts_sssp(ctx, grw, 0, **kw)
+    assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, 0))
+
+
+def test_degree_ordered_device_outputs(G, ctx):
+    import torch
+    g, pb = graph("rmat16_4k")
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+    d = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    G.gts_wcc(ctx, gr, out=d)
+    assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.wcc(g.row_ptr, g.col))
+    f = torch.empty(g.n, dtype=torch.float32, device="cuda")
+    G.gts_pagerank(ctx, gr, 10, out=f)
+    _pr_check(f.cpu().numpy(), oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, "ordered-device")

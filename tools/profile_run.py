@@ -15,6 +15,7 @@ ap.add_argument("--pr-iters", type=int, default=2)
 ap.add_argument("--page-bytes", type=int, default=1 << 20)
 ap.add_argument("--reps", type=int, default=1)
 ap.add_argument("--relabel", action="store_true")
+ap.add_argument("--order", action="store_true")
 ap.add_argument("--streamed", action="store_true")
 a = ap.parse_args()
 t = time.time()
@@ -26,11 +27,11 @@ if a.relabel:
     g = inputs.permute(g, p)
     print("relabelled", time.time() - t, flush=True)
 w = inputs.edge_weights(g) if "sssp" in a.algos else None
-gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=a.page_bytes)
-grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=a.page_bytes) if w is not None else None
+gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=a.page_bytes, order=a.order)
+grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=a.page_bytes, order=a.order) if w is not None else None
 print("built", time.time() - t, flush=True)
 ctx = G.gts_context_create(0)
-kw = dict(residency=G.GTS_STREAMED, ring_slots=4, batch_pages=16) if a.streamed else {}
+kw = dict(residency=G.GTS_STREAMED) if a.streamed else {}
 for _ in range(a.reps):
     for algo in a.algos.split(","):
         if algo == "bfs":
