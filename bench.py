@@ -165,6 +165,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--algos", default="bfs,pr,sssp,wcc")
+    ap.add_argument("--order", dest="order", action="store_true", default=True,
+                    help="build pages with GTS_BUILD_DEGREE_ORDER (default)")
+    ap.add_argument("--no-order", dest="order", action="store_false")
     args = ap.parse_args()
     if args.ref_scale is None:
         args.ref_scale = min(args.scale, 24)
@@ -197,11 +200,11 @@ def main():
     n, m = g.n, g.m
     log(f"[rank {rank}] RMAT-{args.scale} generated n={n} m={m} in {time.time() - t0:.1f}s")
     t0 = time.time()
-    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=args.page_bytes)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=args.page_bytes, order=args.order)
     grw = None
     if "sssp" in algos:
         w = inputs.edge_weights(g)
-        grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=args.page_bytes)
+        grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=args.page_bytes, order=args.order)
         del w
     gst = gr.stats()
     log(f"[rank {rank}] pages built in {time.time() - t0:.1f}s: {gst}")
@@ -323,8 +326,8 @@ def main():
     # end-to-end through the public API with host buffers (pages re-uploaded from pinned host memory)
     e2e = None
     if not args.no_e2e and "bfs" in algos:
-        hl = np.empty(n, np.uint32)
-        hp = np.empty(n, np.float32)
+        hl = torch.empty(n, dtype=torch.int32, pin_memory=True)      # pinned host result buffers
+        hp = torch.empty(n, dtype=torch.float32, pin_memory=True)
         tb, tp_ = [], []
         for _ in range(max(1, min(K, 3))):
             ctx.evict(gr)
@@ -357,6 +360,7 @@ def main():
                 "config": {"workload": f"rmat{args.scale}_bfs_pr_sssp_wcc", "scale": args.scale, "n": n, "m": m,
                            "edge_factor": 16, "abc": [0.57, 0.19, 0.19], "seed": args.scale, "src": 0,
                            "page_bytes": args.page_bytes, "num_pages": gst["num_pages"], "n_lp": gst["n_lp"],
+                           "vertex_order": "in-degree (GTS_BUILD_DEGREE_ORDER)" if args.order else "VID",
                            "topo_bytes": gst["topo_bytes"], "residency": "resident",
                            "strategy": "P" if world > 1 else "single",
                            "parallelism": f"strategy-P x{world}",
