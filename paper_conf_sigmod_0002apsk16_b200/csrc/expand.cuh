@@ -22,7 +22,8 @@ namespace gts {
 
 constexpr int kThreads = 512;
 constexpr int kTile = 512;
-constexpr int kEdgesPerThread = 4;
+constexpr int kEdgesPerThread = 4;   // must be 4: dense tiles hand one 16-byte group per call
+constexpr int kDenseUnroll = 2;      // 16-byte loads in flight per thread in dense tiles
 constexpr int kWarps = kThreads / 32;
 
 __device__ __forceinline__ uint32_t ld32(const uint8_t* p) { return __ldg(reinterpret_cast<const uint32_t*>(p)); }
@@ -43,6 +44,8 @@ __device__ __forceinline__ bool test_bit(const uint32_t* bm, uint32_t v) {
 }
 
 struct TileSmem {
+    uint32_t soff[kTile + 1];  // word index of every record of the tile (all slots); soff[nv] = end
+    uint8_t sel[kTile];        // dense mode: vertex t of the tile is selected
     uint32_t off[kTile];       // word index of the first ADJLIST entry of item j
     uint32_t deg[kTile];
     uint32_t src[kTile];       // VID of item j
@@ -91,7 +94,8 @@ __device__ __forceinline__ void tile_scan(bool sel, uint32_t deg, uint32_t& pos,
 }
 
 // Op interface:
-//   static constexpr bool kReadWeights;
+//   static constexpr bool kReadWeights;  -- the op needs edge weights
+//   static constexpr bool kWeighted;     -- the pages carry weights (record = sz, adj[sz], w[sz])
 //   bool select(uint32_t vid)                            -- SP vertex expanded?
 //   uint32_t payload(uint32_t vid, uint32_t deg)         -- per selected vertex
 //   bool select_lp(uint32_t vid, uint32_t total_deg, uint32_t chunk_len, uint32_t& payload)
@@ -146,21 +150,89 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             }
         } else {
             const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
+            const uint4* q4 = reinterpret_cast<const uint4*>(data);
             for (uint32_t t0 = 0; t0 < nslots; t0 += kTile) {
                 const uint32_t nv = min((uint32_t)kTile, nslots - t0);
                 const uint32_t v = start + t0 + tid;
                 const bool sel = (uint32_t)tid < nv && op.select(v);
-                uint32_t deg = 0, off = 0;
-                if (sel) {
-                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
-                    off = ld_stream_u32(slot + 4, pol);
-                    deg = ld_stream_u32(data + off, pol);
-                }
                 if (!__syncthreads_or(sel)) continue;   // no frontier vertex in this tile
+                // record offsets of the whole tile (coalesced slot reads); the degree of
+                // a record is the distance to the next record (the last one reads its header)
+                if ((uint32_t)tid < nv) {
+                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
+                    const uint32_t o = ld_stream_u32(slot + 4, pol);
+                    sm.soff[tid] = o >> 2;
+                    if ((uint32_t)tid == nv - 1) {
+                        if (t0 + nv < nslots) sm.soff[nv] = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
+                        else sm.soff[nv] = (o >> 2) + 1 + (ld32(data + o) << (Op::kWeighted ? 1 : 0));
+                    }
+                }
+                __syncthreads();
+                uint32_t deg = 0;
+                if ((uint32_t)tid < nv) deg = (sm.soff[tid + 1] - sm.soff[tid] - 1) >> (Op::kWeighted ? 1 : 0);
                 uint32_t pos, nf, excl, total;
-                tile_scan(sel, deg, pos, nf, excl, total, sm);
+                tile_scan(sel, sel ? deg : 0u, pos, nf, excl, total, sm);
+                const uint32_t W0 = sm.soff[0], W1 = sm.soff[nv];
+                if (2 * total >= W1 - W0) {
+                    // dense tile: stream the whole record region with 16-byte loads and
+                    // act on the words of selected owners (hybrid micro-level, App E)
+                    if ((uint32_t)tid < nv) {
+                        sm.sel[tid] = sel ? 1 : 0;
+                        sm.payload[tid] = sel ? op.payload(v, deg) : 0u;
+                    }
+                    __syncthreads();
+                    const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
+                    for (uint32_t qb = qbeg + tid; qb < qend; qb += kThreads * kDenseUnroll) {
+                        uint4 vv[kDenseUnroll];
+#pragma unroll
+                        for (int u = 0; u < kDenseUnroll; ++u) {
+                            const uint32_t q = qb + u * kThreads;
+                            if (q < qend) vv[u] = ld_stream_v4(q4 + q, pol);
+                        }
+#pragma unroll
+                        for (int u = 0; u < kDenseUnroll; ++u) {
+                            const uint32_t q = qb + u * kThreads;
+                            if (q >= qend) break;
+                            const uint32_t w0 = 4 * q;
+                            uint32_t lo = 0, hi = nv;
+                            while (hi - lo > 1) {
+                                const uint32_t mid = (lo + hi) >> 1;
+                                if (sm.soff[mid] <= w0) lo = mid; else hi = mid;
+                            }
+                            uint32_t j = lo, cur = sm.soff[j], nxt = sm.soff[j + 1];
+                            uint32_t dst[kEdgesPerThread], wt[kEdgesPerThread], pl[kEdgesPerThread],
+                                src[kEdgesPerThread];
+                            bool valid[kEdgesPerThread];
+#pragma unroll
+                            for (int k = 0; k < 4; ++k) {
+                                const uint32_t w = w0 + k;
+                                bool ok = w >= W0 && w < W1;
+                                if (ok) {
+                                    while (w >= nxt) {
+                                        ++j;
+                                        cur = nxt;
+                                        nxt = sm.soff[j + 1];
+                                    }
+                                    const uint32_t rel = w - cur, dj = (nxt - cur - 1) >> (Op::kWeighted ? 1 : 0);
+                                    ok = rel >= 1 && rel <= dj && sm.sel[j];
+                                    wt[k] = (Op::kReadWeights && ok) ? ld_stream_l1_u32(words + w + dj, pol) : 0u;
+                                } else {
+                                    wt[k] = 0u;
+                                }
+                                valid[k] = ok;
+                                dst[k] = decode_entry(ps, word_of(vv[u], k));
+                                pl[k] = sm.payload[j];
+                                src[k] = start + t0 + j;
+                            }
+                            op.edges(dst, wt, pl, src, valid);
+                        }
+                    }
+                    __syncthreads();
+                    continue;
+                }
+                // sparse tile: compacted selected vertices, edge-parallel gather
                 if (sel) {
-                    sm.off[pos] = off / 4 + 1;
+                    sm.off[pos] = sm.soff[tid] + 1;
                     sm.deg[pos] = deg;
                     sm.src[pos] = v;
                     sm.payload[pos] = op.payload(v, deg);

@@ -30,8 +30,10 @@ namespace gts {
 
 // ------------------------------------------------------------------ ops ---
 
+template <bool W>
 struct BfsOp {
     static constexpr bool kReadWeights = false;
+    static constexpr bool kWeighted = W;
     const uint32_t* cur;
     uint32_t* visited;
     uint32_t* next;
@@ -66,8 +68,10 @@ struct BfsOp {
     __device__ void end_page() {}
 };
 
+template <bool W>
 struct SsspOp {
     static constexpr bool kReadWeights = true;
+    static constexpr bool kWeighted = W;
     const uint32_t* cur;
     uint32_t* dist;
     uint32_t* next;
@@ -107,8 +111,10 @@ struct SsspOp {
     __device__ void end_page() {}
 };
 
-struct SsspCheckOp {   // exact overflow test: an edge from a finite vertex into an unreached one
+// exact overflow test: an edge from a finite vertex into an unreached one (weighted pages)
+struct SsspCheckOp {
     static constexpr bool kReadWeights = false;
+    static constexpr bool kWeighted = true;
     const uint32_t* dist;
     bool bad;
     __device__ bool select(uint32_t v) { return __ldg(dist + v) != GTS_UNREACHED; }
@@ -131,11 +137,12 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 
 // -------------------------------------------------------------- kernels ---
 
+template <bool W>
 __global__ void __launch_bounds__(kThreads, 2)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
                   uint32_t* work_ctr, unsigned long long* edges_out) {
     __shared__ TileSmem sm;
-    BfsOp op{cur, visited, next, 0ull};
+    BfsOp<W> op{cur, visited, next, 0ull};
     expand_pages(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
@@ -144,7 +151,7 @@ __global__ void __launch_bounds__(kThreads, 2)
 sssp_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* dist, uint32_t* next,
                    uint32_t* work_ctr, unsigned long long* edges_out, uint32_t* ovf_flag) {
     __shared__ TileSmem sm;
-    SsspOp op{cur, dist, next, 0ull, false};
+    SsspOp<true> op{cur, dist, next, 0ull, false};
     expand_pages(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
     if (__syncthreads_or(op.ovf) && threadIdx.x == 0) *ovf_flag = 1u;
@@ -297,7 +304,9 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     if (!l0.empty()) GTS_CUDA(cudaMemcpyAsync(list, l0.data(), l0.size() * 4, cudaMemcpyHostToDevice, s));
     GTS_CUDA(cudaMemcpyAsync(&ctr->list_count, hs, 4, cudaMemcpyHostToDevice, s));
 
-    const void* kexp = algo == kBFS ? (const void*)bfs_expand_kernel : (const void*)sssp_expand_kernel;
+    const void* kexp = algo == kBFS ? (g->weighted ? (const void*)bfs_expand_kernel<true>
+                                                   : (const void*)bfs_expand_kernel<false>)
+                                    : (const void*)sssp_expand_kernel;
     int grid = 0;
     GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
     const int fin_grid = c->num_sms * 4;
@@ -312,9 +321,12 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-                                if (algo == kBFS)
-                                    bfs_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next,
-                                                                                         &ctr->work, &ctr->edges);
+                                if (algo == kBFS && g->weighted)
+                                    bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(
+                                        ps, cur, visited, next, &ctr->work, &ctr->edges);
+                                else if (algo == kBFS)
+                                    bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(
+                                        ps, cur, visited, next, &ctr->work, &ctr->edges);
                                 else
                                     sssp_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(
                                         ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag);

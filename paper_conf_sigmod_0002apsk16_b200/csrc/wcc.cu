@@ -2,13 +2,13 @@
 //
 // Paper: "connected components" is a PageRank-like algorithm run by GTS
 // (P:308), i.e. whole-topology sweeps (ALL_PAGES, Alg 1 line 7); no
-// kernel is given.  B200 design: min-label propagation, label[v] = v
-// initially; every sweep visits every edge (u,v) of every page and lowers
-// the larger of label[u], label[v] to the smaller with atomicMin (labels only
-// decrease, so the fixpoint labels each weakly connected component with its
-// minimum VID); a pointer-jumping pass label[v] = label[label[v]] follows each
-// sweep.  Stops after a sweep that changes nothing.  Strategy-P: labels are
-// merged with an NCCL all-reduce(min) after each sweep.
+// kernel is given.  B200 design: one sweep over all pages hooks every edge
+// into a concurrent union-find forest whose roots are component minima
+// (ECL-CC-style hooking with atomicCAS, path halving), then a finalize pass
+// points every vertex at its root = the minimum VID of its weakly connected
+// component.  One sweep is exact on one GPU.  Strategy-P/S with N > 1: each
+// rank hooks its own pages, labels are merged with an NCCL all-reduce(min),
+// and the sweep repeats from the merged labels until no rank hooks anything.
 #include <cuda_runtime.h>
 #include <nccl.h>
 
@@ -19,38 +19,68 @@
 
 namespace gts {
 
+// Union-find over the page sweep (ECL-CC style hooking).  Invariant:
+// parent[v] <= v, roots satisfy parent[r] = r, and a hook always points the
+// larger root at the smaller one, so the root of every component is its
+// minimum (internal) VID.  One sweep over all pages hooks every edge; a
+// finalize pass then points every vertex at its root.  Path halving in find
+// writes only ancestors, so concurrent finds/hooks are benign.
+__device__ __forceinline__ uint32_t uf_find(uint32_t* parent, uint32_t x) {
+    uint32_t cur = __ldcg(parent + x);
+    if (cur != x) {
+        uint32_t prev = x, next;
+        while (cur > (next = __ldcg(parent + cur))) {
+            parent[prev] = next;
+            prev = cur;
+            cur = next;
+        }
+    }
+    return cur;
+}
+
+__device__ __forceinline__ bool uf_hook(uint32_t* parent, uint32_t a, uint32_t b) {
+    uint32_t ra = uf_find(parent, a), rb = uf_find(parent, b);
+    bool hooked = false;
+    while (ra != rb) {
+        if (ra < rb) {
+            const uint32_t ret = atomicCAS(parent + rb, rb, ra);
+            if (ret == rb) { hooked = true; break; }
+            rb = ret;
+        } else {
+            const uint32_t ret = atomicCAS(parent + ra, ra, rb);
+            if (ret == ra) { hooked = true; break; }
+            ra = ret;
+        }
+    }
+    return hooked;
+}
+
+template <bool W>
 struct WccOp {
     static constexpr bool kReadWeights = false;
-    uint32_t* label;
+    static constexpr bool kWeighted = W;
+    uint32_t* parent;
     bool changed;
     __device__ bool select(uint32_t) { return true; }
-    __device__ uint32_t payload(uint32_t v, uint32_t deg) { return deg ? __ldcg(label + v) : 0u; }
+    __device__ uint32_t payload(uint32_t v, uint32_t) { return v; }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t& pl) {
-        pl = __ldcg(label + vid);
+        pl = vid;
         return true;
     }
-    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t* lu,
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*,
                                           const uint32_t* src, const bool* valid) {
-        uint32_t lv[kEdgesPerThread];
 #pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q) lv[q] = valid[q] ? __ldcg(label + dst[q]) : 0u;
-#pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q) {
-            if (!valid[q]) continue;
-            if (lu[q] < lv[q]) {
-                if (atomicMin(label + dst[q], lu[q]) > lu[q]) changed = true;
-            } else if (lv[q] < lu[q]) {
-                if (atomicMin(label + src[q], lv[q]) > lv[q]) changed = true;
-            }
-        }
+        for (int q = 0; q < kEdgesPerThread; ++q)
+            if (valid[q] && src[q] != dst[q] && uf_hook(parent, src[q], dst[q])) changed = true;
     }
     __device__ void end_page() {}
 };
 
+template <bool W>
 __global__ void __launch_bounds__(kThreads, 2)
-wcc_sweep_kernel(PageSet ps, uint32_t* label, uint32_t* work_ctr, uint32_t* changed) {
+wcc_sweep_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t* changed) {
     __shared__ TileSmem sm;
-    WccOp op{label, false};
+    WccOp<W> op{parent, false};
     expand_pages(ps, op, sm, work_ctr);
     if (__syncthreads_or(op.changed) && threadIdx.x == 0) *changed = 1u;
 }
@@ -60,12 +90,13 @@ __global__ void wcc_init_kernel(uint32_t* label, uint64_t n) {
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) label[i] = (uint32_t)i;
 }
 
-__global__ void wcc_jump_kernel(uint32_t* label, uint64_t n) {
+// every vertex points at its root (the component's minimum VID)
+__global__ void wcc_finalize_kernel(uint32_t* parent, uint64_t n) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-        const uint32_t l = label[i];
-        const uint32_t ll = __ldcg(label + l);
-        if (ll < l) label[i] = ll;
+        uint32_t r = __ldcg(parent + i);
+        while (r != __ldcg(parent + r)) r = __ldcg(parent + r);
+        parent[i] = r;
     }
 }
 
@@ -94,7 +125,8 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     const int eg = c->num_sms * 4;
     wcc_init_kernel<<<eg, 256, 0, s>>>(label, n);
     int grid = 0;
-    GTS_TRY(sms_grid(c, (const void*)wcc_sweep_kernel, kThreads, 0, &grid));
+    auto sweep_k = g->weighted ? wcc_sweep_kernel<true> : wcc_sweep_kernel<false>;
+    GTS_TRY(sms_grid(c, (const void*)sweep_k, kThreads, 0, &grid));
     uint64_t launches = 1, main_launches = 0, nccl_bytes = 0;
     uint32_t sweeps = 0;
     uint32_t* hs = (uint32_t*)c->h_small;
@@ -108,7 +140,7 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
                                 GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
                                 std::pair<cudaEvent_t, cudaEvent_t> e2;
                                 if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
-                                wcc_sweep_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(ps, label, ctr, ctr + 1);
+                                sweep_k<<<std::min(grid, cap), kThreads, 0, s>>>(ps, label, ctr, ctr + 1);
                                 if (timing) cudaEventRecord(e2.second, s);
                                 GTS_CUDA(cudaGetLastError());
                                 ++main_launches;
@@ -125,9 +157,10 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
             nccl_bytes += n * 4 + 4;
         }
         if (timing) { ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
-        wcc_jump_kernel<<<eg, 256, 0, s>>>(label, n);
+        wcc_finalize_kernel<<<eg, 256, 0, s>>>(label, n);
         if (timing) cudaEventRecord(ev.second, s);
         ++launches;
+        if (c->world == 1) break;              // union-find is exact after one sweep on one GPU
         GTS_CUDA(cudaMemcpyAsync(hs, ctr + 1, 4, cudaMemcpyDeviceToHost, s));
         GTS_CUDA(cudaStreamSynchronize(s));
         if (hs[0] == 0) break;
