@@ -42,6 +42,8 @@ def lib():
         L.gen_rmat.argtypes = [ctypes.c_int, ctypes.c_uint64, ctypes.c_double, ctypes.c_double,
                                ctypes.c_double, ctypes.c_uint64, u64p, u32p]
         L.gen_rmat.restype = ctypes.c_int
+        L.gen_rmat_lean.argtypes = L.gen_rmat.argtypes
+        L.gen_rmat_lean.restype = ctypes.c_int
         L.gen_twitter_like.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_double,
                                        ctypes.c_double, ctypes.c_uint64, u64p, u32p]
         L.gen_twitter_like.restype = ctypes.c_int
@@ -95,15 +97,17 @@ class CSR:
         return f"CSR({self.name!r}, n={self.n}, m={self.m}, weighted={self.weights is not None})"
 
 
-def rmat(scale: int, edge_factor: int = 16, abc=RMAT_ABC, seed: int | None = None) -> CSR:
-    """Unpermuted RMAT (a,b,c) with m = edge_factor * 2^scale; seed defaults to scale."""
+def rmat(scale: int, edge_factor: int = 16, abc=RMAT_ABC, seed: int | None = None, lean: bool = False) -> CSR:
+    """Unpermuted RMAT (a,b,c) with m = edge_factor * 2^scale; seed defaults to scale.
+    lean=True draws the edges twice instead of buffering them (same graph, less memory)."""
     if seed is None:
         seed = scale
     n = 1 << scale
     m = edge_factor * n
     row_ptr = np.empty(n + 1, dtype=np.uint64)
     col = np.empty(m, dtype=np.uint32)
-    rc = lib().gen_rmat(scale, edge_factor, abc[0], abc[1], abc[2], seed, _p64(row_ptr), _p32(col))
+    fn = lib().gen_rmat_lean if lean else lib().gen_rmat
+    rc = fn(scale, edge_factor, abc[0], abc[1], abc[2], seed, _p64(row_ptr), _p32(col))
     if rc != 0:
         raise RuntimeError(f"gen_rmat failed rc={rc}")
     return CSR(row_ptr, col, name=f"rmat{scale}")

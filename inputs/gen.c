@@ -134,6 +134,40 @@ int gen_rmat(int scale, uint64_t edge_factor, double a, double b, double c, uint
     return 0;
 }
 
+/* Same graph as gen_rmat, without the (u, v) pair buffer: the edges are drawn
+ * twice (count pass, fill pass).  For scales whose pair buffer (8 m bytes)
+ * does not fit in host memory next to the CSR. */
+int gen_rmat_lean(int scale, uint64_t edge_factor, double a, double b, double c, uint64_t seed,
+                  uint64_t* row_ptr /* n+1 */, uint32_t* col /* m */) {
+    if (scale < 1 || scale > 32) return -1;
+    uint64_t n = 1ULL << scale, m = edge_factor * n;
+    rmat_p p;
+    const double two32 = 4294967296.0;
+    p.ta = (uint64_t)(a * two32);
+    p.tab = (uint64_t)((a + b) * two32);
+    p.tabc = (uint64_t)((a + b + c) * two32);
+    p.seed_mix = splitmix64(seed ^ 0x524D4154ULL /* "RMAT" */);
+    p.scale = scale;
+    uint64_t* cnt = (uint64_t*)calloc(n, sizeof(uint64_t));
+    if (!cnt) return -2;
+    #pragma omp parallel for schedule(static, 65536)
+    for (int64_t e = 0; e < (int64_t)m; ++e) {
+        uint32_t u, v; rmat_edge(&p, (uint64_t)e, &u, &v);
+        __atomic_fetch_add(&cnt[u], 1, __ATOMIC_RELAXED);
+    }
+    scan_counts(n, cnt, row_ptr);
+    memcpy(cnt, row_ptr, n * sizeof(uint64_t));
+    #pragma omp parallel for schedule(static, 65536)
+    for (int64_t e = 0; e < (int64_t)m; ++e) {
+        uint32_t u, v; rmat_edge(&p, (uint64_t)e, &u, &v);
+        uint64_t pos = __atomic_fetch_add(&cnt[u], 1, __ATOMIC_RELAXED);
+        col[pos] = v;
+    }
+    free(cnt);
+    sort_rows(n, row_ptr, col);
+    return 0;
+}
+
 /* ------------------------------------------------------- Twitter-shaped --- */
 
 /* degree sequence d_i = floor(C (i+i0)^-beta), C chosen so sum d = m; the

@@ -1,28 +1,16 @@
-// Generic page expansion for sm_100a, shared by BFS, SSSP and WCC: persistent
-// CTAs take whole slotted pages from an atomic page queue; inside a page the
-// 16 warps work independently (no CTA barrier between a page's first and last
-// vertex).
+// Generic page expansion for sm_100a: one CTA per slotted page at a time
+// (persistent grid, dynamic page queue), shared by BFS, SSSP, PageRank, WCC.
 //
-// Paper: K_SP / K_LP (Alg 2-5) give each vertex of an SP to one
-// (virtual) warp (VWC) and each ADJLIST entry of an LP to one thread;
-// App E proposes choosing edge- or vertex-centric processing per
-// page by density.  B200 design:
-//  * SP pages are consumed in groups of 32 consecutive slots claimed by warps
-//    from a per-page shared counter.  A lane per slot reads the record offset
-//    (one coalesced slot read); degrees are offset differences; the frontier
-//    test per vertex is folded into __ballot_sync.
-//  * Dense group (selected edges >= half of the group's record words, always
-//    true for PageRank-like sweeps): the group's record region is streamed with
-//    16-byte evict_first loads and each 4-word chunk finds its owner by a
-//    5-step binary search over the 33 group offsets in shared memory.
-//  * Sparse group: the selected vertices are compacted with __popc of the
-//    ballot, their degrees prefix-summed with shuffles, and the warp expands
-//    their edges edge-parallel (4 consecutive edges per lane).
-//  * LP pages (one vertex, up to 262,137 entries at 1 MiB) are swept by all 16
-//    warps of the CTA; a hub spans several LPs and therefore several CTAs.
-// Each op receives 4 edges at a time whose adjacency words were loaded back
-// to back, and issues its own per-edge loads (visited bits, dist, parents) as
-// a batch before acting on them.
+// Paper: K_SP / K_LP (Alg 2-5) assign one warp per vertex of an
+// SP (VWC) and one thread per ADJLIST entry of an LP.  B200 design
+// (DESIGN.md "Kernels"): a CTA takes a whole page; an SP is processed in tiles
+// of kTile consecutive slots: the tile's selected vertices (frontier test, or
+// all for PageRank-like sweeps) are compacted with __ballot_sync/__popc, their
+// degrees prefix-summed, and the tile's edges are then expanded edge-parallel
+// (4 consecutive edges per thread, one binary search per 4 edges), so a
+// degree-13 K vertex and a run of degree-1 vertices are balanced alike.  An LP
+// is swept by the whole CTA; a huge vertex spans several LPs and so several
+// CTAs (high-degree split).
 #pragma once
 
 #include <cstdint>
@@ -33,9 +21,10 @@
 namespace gts {
 
 constexpr int kThreads = 512;
+constexpr int kTile = 512;
+constexpr int kEdgesPerThread = 4;   // must be 4: dense tiles hand one 16-byte group per call
+constexpr int kDenseUnroll = 2;      // 16-byte loads in flight per thread in dense tiles
 constexpr int kWarps = kThreads / 32;
-constexpr int kEdgesPerThread = 4;   // one 16-byte group per op call
-constexpr int kDenseUnroll = 2;      // 16-byte loads in flight per lane in dense groups
 
 __device__ __forceinline__ uint32_t ld32(const uint8_t* p) { return __ldg(reinterpret_cast<const uint32_t*>(p)); }
 
@@ -54,181 +43,79 @@ __device__ __forceinline__ bool test_bit(const uint32_t* bm, uint32_t v) {
     return (__ldg(bm + (v >> 5)) >> (v & 31)) & 1u;
 }
 
-struct WarpSmem {
-    uint32_t off[33];      // dense: record word offsets of the group (off[nv] = end of the last record)
-    uint32_t pay[32];      // payload of each slot (dense) or of each selected vertex (sparse)
-    uint32_t pre[33];      // sparse: exclusive prefix of the selected degrees
-    uint32_t eoff[32];     // sparse: word index of the first ADJLIST entry
-    uint32_t src[32];      // sparse: VID
-    uint32_t deg[32];      // sparse: degree
-    uint32_t selmask;      // dense: ballot of the selected slots
+struct TileSmem {
+    uint32_t soff[kTile + 1];  // word index of every record of the tile (all slots); soff[nv] = end
+    uint8_t sel[kTile];        // dense mode: vertex t of the tile is selected
+    uint32_t off[kTile];       // word index of the first ADJLIST entry of item j
+    uint32_t deg[kTile];
+    uint32_t src[kTile];       // VID of item j
+    uint32_t payload[kTile];
+    uint32_t pre[kTile + 1];   // exclusive prefix of deg over items
+    uint32_t wsum[kWarps];
+    uint32_t wcnt[kWarps];
+    uint32_t item;
 };
 
-struct TileSmem {
-    WarpSmem w[kWarps];
-    uint32_t item;
-    uint32_t gctr;         // next 32-slot group of the current page
-};
+// Tile scan: frontier compaction by __ballot_sync/__popc (position of each
+// selected vertex among the tile's selected vertices) fused with the exclusive
+// prefix sum of the selected vertices' degrees.  Two __syncthreads.
+__device__ __forceinline__ void tile_scan(bool sel, uint32_t deg, uint32_t& pos, uint32_t& nf,
+                                          uint32_t& deg_excl, uint32_t& deg_total, TileSmem& sm) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t mask = __ballot_sync(0xFFFFFFFFu, sel);
+    const uint32_t rank_in_warp = __popc(mask & ((1u << lane) - 1u));
+    uint32_t x = deg;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) {
+        sm.wsum[warp] = x;
+        sm.wcnt[warp] = __popc(mask);
+    }
+    __syncthreads();
+    if (warp == 0) {
+        uint32_t s = lane < kWarps ? sm.wsum[lane] : 0u;
+        uint32_t c = lane < kWarps ? sm.wcnt[lane] : 0u;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint32_t y = __shfl_up_sync(0xFFFFFFFFu, s, o);
+            uint32_t z = __shfl_up_sync(0xFFFFFFFFu, c, o);
+            if (lane >= o) { s += y; c += z; }
+        }
+        if (lane < kWarps) { sm.wsum[lane] = s; sm.wcnt[lane] = c; }   // inclusive warp prefixes
+    }
+    __syncthreads();
+    deg_excl = (warp > 0 ? sm.wsum[warp - 1] : 0u) + x - deg;
+    deg_total = sm.wsum[kWarps - 1];
+    pos = (warp > 0 ? sm.wcnt[warp - 1] : 0u) + rank_in_warp;
+    nf = sm.wcnt[kWarps - 1];
+}
 
 // Op interface:
 //   static constexpr bool kReadWeights;  -- the op needs edge weights
 //   static constexpr bool kWeighted;     -- the pages carry weights (record = sz, adj[sz], w[sz])
 //   bool select(uint32_t vid)                            -- SP vertex expanded?
-//   uint32_t payload(uint32_t vid, uint32_t deg)         -- per selected vertex (called once)
+//   uint32_t payload(uint32_t vid, uint32_t deg)         -- per selected vertex
 //   bool select_lp(uint32_t vid, uint32_t total_deg, uint32_t chunk_len, uint32_t& payload)
-//   void edges(const uint32_t dst[4], const uint32_t w[4], const uint32_t pl[4], const uint32_t src[4],
-//              const bool valid[4])
+//   void edges(const uint32_t dst[E], const uint32_t w[E], const uint32_t pl[E], const uint32_t src[E],
+//              const bool valid[E])                      -- E = kEdgesPerThread edges, loads already issued
 //   void end_page()
-template <class Op>
-__device__ __forceinline__ void expand_group(const PageSet& ps, Op& op, WarpSmem& ws, const uint8_t* data,
-                                             const uint8_t* end, uint32_t start, uint32_t nslots, uint32_t g,
-                                             uint64_t pol) {
-    constexpr uint32_t wsh = Op::kWeighted ? 1 : 0;
-    const int lane = threadIdx.x & 31;
-    const uint32_t* words = reinterpret_cast<const uint32_t*>(data);
-    const uint32_t j = g * 32 + lane;
-    const bool valid = j < nslots;
-    const uint32_t v = start + j;
-    const bool sel = valid && op.select(v);
-    const uint32_t mask = __ballot_sync(0xFFFFFFFFu, sel);
-    if (!mask) return;
-    // record offsets and degrees (offset differences; the page's last record reads its header)
-    uint32_t off = 0;
-    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(j + 1);
-    if (valid) off = ld_stream_u32(slot + 4, pol) >> 2;
-    uint32_t nxt = __shfl_down_sync(0xFFFFFFFFu, off, 1);
-    const uint32_t last = min(31u, nslots - 1 - g * 32);           // lane of the group's last slot
-    if ((uint32_t)lane == last) {
-        if (j + 1 < nslots) nxt = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
-        else nxt = off + 1 + (ld32(data + 4ull * off) << wsh);
-    }
-    const uint32_t deg = valid ? (nxt - off - 1) >> wsh : 0u;
-    const uint32_t sdeg = sel ? deg : 0u;
-    uint32_t incl = sdeg;                                          // warp inclusive scan of selected degrees
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
-        if (lane >= o) incl += y;
-    }
-    const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
-    const uint32_t W0 = __shfl_sync(0xFFFFFFFFu, off, 0), W1 = __shfl_sync(0xFFFFFFFFu, nxt, last);
-    const uint32_t pay = sel ? op.payload(v, deg) : 0u;
-    if (total == 0) return;
-    if (2 * total >= W1 - W0) {
-        // ---- dense group: stream the record words, act on the selected owners
-        ws.off[lane] = off;
-        if (lane == 0) {
-            ws.off[last + 1] = W1;
-            ws.selmask = mask;
-        }
-        ws.pay[lane] = pay;
-        __syncwarp();
-        const uint32_t nv = last + 1;
-        const uint32_t smask = mask;
-        const uint4* q4 = reinterpret_cast<const uint4*>(data);
-        const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
-        for (uint32_t qb = qbeg + lane; qb < qend; qb += 32 * kDenseUnroll) {
-            uint4 vv[kDenseUnroll];
-#pragma unroll
-            for (int u = 0; u < kDenseUnroll; ++u) {
-                const uint32_t q = qb + 32 * u;
-                if (q < qend) vv[u] = ld_stream_v4(q4 + q, pol);
-            }
-#pragma unroll
-            for (int u = 0; u < kDenseUnroll; ++u) {
-                const uint32_t q = qb + 32 * u;
-                if (q >= qend) break;
-                const uint32_t w0 = 4 * q;
-                uint32_t lo = 0, hi = nv;                          // off[lo] <= max(w0, W0) < off[hi]
-                while (hi - lo > 1) {
-                    const uint32_t mid = (lo + hi) >> 1;
-                    if (ws.off[mid] <= w0) lo = mid; else hi = mid;
-                }
-                uint32_t k_ = lo, cur = ws.off[lo], nx = ws.off[lo + 1];
-                uint32_t dst[4], wt[4], pl[4], src[4];
-                bool ok[4];
-#pragma unroll
-                for (int k = 0; k < 4; ++k) {
-                    const uint32_t w = w0 + k;
-                    bool e = w >= W0 && w < W1;
-                    if (e) {
-                        while (w >= nx) {
-                            ++k_;
-                            cur = nx;
-                            nx = ws.off[k_ + 1];
-                        }
-                        const uint32_t rel = w - cur, dj = (nx - cur - 1) >> wsh;
-                        e = rel >= 1 && rel <= dj && ((smask >> k_) & 1u);
-                        wt[k] = (Op::kReadWeights && e) ? ld_stream_l1_u32(words + w + dj, pol) : 0u;
-                    } else {
-                        wt[k] = 0u;
-                    }
-                    ok[k] = e;
-                    dst[k] = decode_entry(ps, word_of(vv[u], k));
-                    pl[k] = ws.pay[k_];
-                    src[k] = start + g * 32 + k_;
-                }
-                op.edges(dst, wt, pl, src, ok);
-            }
-        }
-        __syncwarp();
-        return;
-    }
-    // ---- sparse group: compacted selected vertices, edge-parallel gather
-    const uint32_t pos = __popc(mask & ((1u << lane) - 1u));
-    const uint32_t nf = __popc(mask);
-    if (sel) {
-        ws.eoff[pos] = off + 1;
-        ws.deg[pos] = deg;
-        ws.src[pos] = v;
-        ws.pay[pos] = pay;
-        ws.pre[pos] = incl - sdeg;
-    }
-    if (lane == 0) ws.pre[nf] = total;
-    __syncwarp();
-    for (uint32_t e0 = (uint32_t)lane * 4; e0 < total; e0 += 128) {
-        uint32_t lo = 0, hi = nf;                                  // pre[lo] <= e0 < pre[hi]
-        while (hi - lo > 1) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (ws.pre[mid] <= e0) lo = mid; else hi = mid;
-        }
-        uint32_t k_ = lo, nx = ws.pre[lo + 1];
-        uint32_t dst[4], wt[4], pl[4], src[4];
-        bool ok[4];
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            const uint32_t e = e0 + q;
-            ok[q] = e < total;
-            if (ok[q]) {
-                while (e >= nx) nx = ws.pre[++k_ + 1];
-            }
-            const uint32_t local = e - ws.pre[k_];
-            const uint32_t* adj = words + ws.eoff[k_];
-            dst[q] = ok[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
-            wt[q] = (Op::kReadWeights && ok[q]) ? ld_stream_l1_u32(adj + ws.deg[k_] + local, pol) : 0u;
-            pl[q] = ws.pay[k_];
-            src[q] = ws.src[k_];
-        }
-#pragma unroll
-        for (int q = 0; q < 4; ++q) dst[q] = decode_entry(ps, dst[q]);
-        op.edges(dst, wt, pl, src, ok);
-    }
-    __syncwarp();
-}
-
+// Edges reach the op in groups of kEdgesPerThread whose adjacency words were
+// loaded back to back, so each thread has that many independent loads in
+// flight, and the op can issue its own per-edge loads (visited bits, dist,
+// labels) as a batch before acting on them.
 template <class Op>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
     const uint32_t count = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int tid = threadIdx.x;
     const uint64_t pol = policy_evict_first();
-    WarpSmem& ws = sm.w[warp];
     for (;;) {
-        if (tid == 0) {
-            sm.item = atomicAdd(work_ctr, 1u);
-            sm.gctr = 0;
-        }
+        if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
         __syncthreads();
         const uint32_t i = sm.item;
+        __syncthreads();
         if (i >= count) break;
         uint32_t pid;
         const uint8_t* data;
@@ -263,17 +150,127 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             }
         } else {
             const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
-            const uint32_t ngroups = (nslots + 31) >> 5;
-            for (;;) {
-                uint32_t g = 0;
-                if (lane == 0) g = atomicAdd(&sm.gctr, 1u);
-                g = __shfl_sync(0xFFFFFFFFu, g, 0);
-                if (g >= ngroups) break;
-                expand_group(ps, op, ws, data, end, start, nslots, g, pol);
+            const uint4* q4 = reinterpret_cast<const uint4*>(data);
+            for (uint32_t t0 = 0; t0 < nslots; t0 += kTile) {
+                const uint32_t nv = min((uint32_t)kTile, nslots - t0);
+                const uint32_t v = start + t0 + tid;
+                const bool sel = (uint32_t)tid < nv && op.select(v);
+                if (!__syncthreads_or(sel)) continue;   // no frontier vertex in this tile
+                // record offsets of the whole tile (coalesced slot reads); the degree of
+                // a record is the distance to the next record (the last one reads its header)
+                if ((uint32_t)tid < nv) {
+                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
+                    const uint32_t o = ld_stream_u32(slot + 4, pol);
+                    sm.soff[tid] = o >> 2;
+                    if ((uint32_t)tid == nv - 1) {
+                        if (t0 + nv < nslots) sm.soff[nv] = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
+                        else sm.soff[nv] = (o >> 2) + 1 + (ld32(data + o) << (Op::kWeighted ? 1 : 0));
+                    }
+                }
+                __syncthreads();
+                uint32_t deg = 0;
+                if ((uint32_t)tid < nv) deg = (sm.soff[tid + 1] - sm.soff[tid] - 1) >> (Op::kWeighted ? 1 : 0);
+                uint32_t pos, nf, excl, total;
+                tile_scan(sel, sel ? deg : 0u, pos, nf, excl, total, sm);
+                const uint32_t W0 = sm.soff[0], W1 = sm.soff[nv];
+                if (2 * total >= W1 - W0) {
+                    // dense tile: stream the whole record region with 16-byte loads and
+                    // act on the words of selected owners (hybrid micro-level, App E)
+                    if ((uint32_t)tid < nv) {
+                        sm.sel[tid] = sel ? 1 : 0;
+                        sm.payload[tid] = sel ? op.payload(v, deg) : 0u;
+                    }
+                    __syncthreads();
+                    const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
+                    for (uint32_t qb = qbeg + tid; qb < qend; qb += kThreads * kDenseUnroll) {
+                        uint4 vv[kDenseUnroll];
+#pragma unroll
+                        for (int u = 0; u < kDenseUnroll; ++u) {
+                            const uint32_t q = qb + u * kThreads;
+                            if (q < qend) vv[u] = ld_stream_v4(q4 + q, pol);
+                        }
+#pragma unroll
+                        for (int u = 0; u < kDenseUnroll; ++u) {
+                            const uint32_t q = qb + u * kThreads;
+                            if (q >= qend) break;
+                            const uint32_t w0 = 4 * q;
+                            uint32_t lo = 0, hi = nv;
+                            while (hi - lo > 1) {
+                                const uint32_t mid = (lo + hi) >> 1;
+                                if (sm.soff[mid] <= w0) lo = mid; else hi = mid;
+                            }
+                            uint32_t j = lo, cur = sm.soff[j], nxt = sm.soff[j + 1];
+                            uint32_t dst[kEdgesPerThread], wt[kEdgesPerThread], pl[kEdgesPerThread],
+                                src[kEdgesPerThread];
+                            bool valid[kEdgesPerThread];
+#pragma unroll
+                            for (int k = 0; k < 4; ++k) {
+                                const uint32_t w = w0 + k;
+                                bool ok = w >= W0 && w < W1;
+                                if (ok) {
+                                    while (w >= nxt) {
+                                        ++j;
+                                        cur = nxt;
+                                        nxt = sm.soff[j + 1];
+                                    }
+                                    const uint32_t rel = w - cur, dj = (nxt - cur - 1) >> (Op::kWeighted ? 1 : 0);
+                                    ok = rel >= 1 && rel <= dj && sm.sel[j];
+                                    wt[k] = (Op::kReadWeights && ok) ? ld_stream_l1_u32(words + w + dj, pol) : 0u;
+                                } else {
+                                    wt[k] = 0u;
+                                }
+                                valid[k] = ok;
+                                dst[k] = decode_entry(ps, word_of(vv[u], k));
+                                pl[k] = sm.payload[j];
+                                src[k] = start + t0 + j;
+                            }
+                            op.edges(dst, wt, pl, src, valid);
+                        }
+                    }
+                    __syncthreads();
+                    continue;
+                }
+                // sparse tile: compacted selected vertices, edge-parallel gather
+                if (sel) {
+                    sm.off[pos] = sm.soff[tid] + 1;
+                    sm.deg[pos] = deg;
+                    sm.src[pos] = v;
+                    sm.payload[pos] = op.payload(v, deg);
+                    sm.pre[pos] = excl;
+                }
+                if (tid == 0) sm.pre[nf] = total;
+                __syncthreads();
+                for (uint32_t e0 = (uint32_t)tid * kEdgesPerThread; e0 < total; e0 += kThreads * kEdgesPerThread) {
+                    uint32_t lo = 0, hi = nf;              // pre[lo] <= e0 < pre[hi]
+                    while (hi - lo > 1) {
+                        uint32_t mid = (lo + hi) >> 1;
+                        if (sm.pre[mid] <= e0) lo = mid; else hi = mid;
+                    }
+                    uint32_t j = lo, nxt = sm.pre[lo + 1];
+                    uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
+                    bool valid[kEdgesPerThread];
+#pragma unroll
+                    for (int q = 0; q < kEdgesPerThread; ++q) {
+                        const uint32_t e = e0 + q;
+                        valid[q] = e < total;
+                        if (valid[q]) {
+                            while (e >= nxt) nxt = sm.pre[++j + 1];
+                        }
+                        const uint32_t local = e - sm.pre[j];
+                        const uint32_t* adj = words + sm.off[j];
+                        dst[q] = valid[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
+                        w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_l1_u32(adj + sm.deg[j] + local, pol) : 0u;
+                        pl[q] = sm.payload[j];
+                        src[q] = sm.src[j];
+                    }
+#pragma unroll
+                    for (int q = 0; q < kEdgesPerThread; ++q) dst[q] = decode_entry(ps, dst[q]);
+                    op.edges(dst, w, pl, src, valid);
+                }
+                __syncthreads();
             }
         }
         op.end_page();
-        __syncthreads();                      // sm.item / sm.gctr are rewritten for the next page
     }
 }
 

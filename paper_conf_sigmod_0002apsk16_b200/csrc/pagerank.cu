@@ -78,47 +78,28 @@ struct PrEmitter {
 
 constexpr size_t kPrDynSmem = kHotSlots * (sizeof(uint32_t) + sizeof(float));
 constexpr size_t kPrDynSmemDense = kHotDense * sizeof(float);
-template <bool W, bool kDense>
-struct PrOp {
-    static constexpr bool kReadWeights = false;
-    static constexpr bool kWeighted = W;
-    const float* x;
-    float d;
-    uint64_t pol;
-    double dang;
-    PrEmitter<kDense> em;
+constexpr int kPrUnroll = 4;            // 16-byte loads in flight per thread
 
-    __device__ bool select(uint32_t) { return true; }
-    // c_u = d * x_u / outdeg(u); dangling vertices add x_u to D instead (R3)
-    __device__ uint32_t payload(uint32_t v, uint32_t deg) {
-        const float xv = ld_stream_f32(x + v, pol);
-        if (deg == 0) {
-            dang += (double)xv;
-            return 0u;
-        }
-        return __float_as_uint(d * xv / (float)deg);
-    }
-    // LP: divide by the vertex's TOTAL out-degree (R4)
-    __device__ bool select_lp(uint32_t vid, uint32_t total, uint32_t, uint32_t& pl) {
-        pl = __float_as_uint(d * __ldg(x + vid) / (float)total);
-        return true;
-    }
-    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t* pl, const uint32_t*,
-                                          const bool* ok) {
-#pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q)
-            if (ok[q]) em.edge(dst[q], __uint_as_float(pl[q]));
-    }
-    __device__ void end_page() { em.flush(); }
+struct PrSmem {
+    uint32_t off[kTile + 1];            // page-relative word index of each record of the tile; off[nv] = end
+    float c[kTile];                     // d * x_u / outdeg(u)
+    uint32_t item;
 };
 
-// K_PR_SP / K_PR_LP (Alg 4/5) on the generic warp-centric page engine
-// (expand.cuh); the CTA's shared memory holds the hot-destination partial sums.
+__device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const uint32_t* rvt) {
+    return enc == GTS_ENTRY_VID32 ? e : __ldg(rvt + (e >> 16)) + (e & 0xFFFFu);
+}
+
+// K_PR_SP / K_PR_LP (Alg 4/5) for a persistent CTA.  The record region of a
+// tile of 512 consecutive vertices is one contiguous word range (records are
+// packed in VID order from offset 0), streamed with 16-byte evict_first loads,
+// kPrUnroll in flight per thread; the owner of each 4-word group is found by a
+// binary search over the tile's record offsets in shared memory.
 template <bool kWeighted, bool kDense>
 __global__ void __launch_bounds__(kThreads, 2)
 pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__ hot_keys,
                   float d, double* dang_out, uint32_t* work_ctr, uint32_t n_dense) {
-    __shared__ TileSmem sm;
+    __shared__ PrSmem sm;
     extern __shared__ uint4 dyn_smem[];
     uint32_t* hkeys = reinterpret_cast<uint32_t*>(dyn_smem);
     float* hacc = kDense ? reinterpret_cast<float*>(dyn_smem) : reinterpret_cast<float*>(hkeys + kHotSlots);
@@ -131,9 +112,115 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             hacc[i] = 0.f;
         }
     }
-    __syncthreads();
-    PrOp<kWeighted, kDense> op{x, d, policy_evict_first(), 0.0, {acc, hkeys, hacc, 0u, 0.f, false}};
-    expand_pages(ps, op, sm, work_ctr);
+    const uint64_t pol = policy_evict_first();
+    const uint32_t count = ps.count;
+    const uint32_t enc = ps.entry_encoding;
+    constexpr uint32_t wshift = kWeighted ? 1 : 0;
+    PrEmitter<kDense> em{acc, hkeys, hacc, 0u, 0.f, false};
+    double dang = 0.0;
+    for (;;) {
+        if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
+        __syncthreads();
+        const uint32_t it = sm.item;
+        __syncthreads();                     // sm.item is rewritten by thread 0 next round
+        if (it >= count) break;
+        uint32_t pid;
+        const uint8_t* data;
+        page_at(ps, it, pid, data);
+        const uint8_t* end = data + ps.page_bytes;
+        const uint32_t kind = ld32(end - 4);
+        const uint32_t nslots = ld32(end - 8);
+        const uint4* q4 = reinterpret_cast<const uint4*>(data);
+        if (kind == GTS_PAGE_LP) {
+            const uint32_t vid = ld32(end - kLpFooter - kSlotBytes);
+            const uint32_t total = ld32(end - 16);
+            const uint32_t len = ld32(data);
+            const float c = d * __ldg(x + vid) / (float)total;
+            const uint32_t wend = 1 + len, qend = (wend + 3) >> 2;
+            for (uint32_t qb = tid; qb < qend; qb += kThreads * kPrUnroll) {
+                uint4 v[kPrUnroll];
+#pragma unroll
+                for (int u = 0; u < kPrUnroll; ++u) {
+                    const uint32_t q = qb + u * kThreads;
+                    if (q < qend) v[u] = ld_stream_v4(q4 + q, pol);
+                }
+#pragma unroll
+                for (int u = 0; u < kPrUnroll; ++u) {
+                    const uint32_t q = qb + u * kThreads;
+                    if (q >= qend) break;
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        const uint32_t w = 4 * q + k;
+                        if (w >= 1 && w < wend) em.edge(pr_decode(word_of(v[u], k), enc, ps.rvt_start), c);
+                    }
+                }
+            }
+        } else {
+            const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
+            for (uint32_t t0 = 0; t0 < nslots; t0 += kTile) {
+                const uint32_t nv = min((uint32_t)kTile, nslots - t0);
+                if ((uint32_t)tid < nv) {
+                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
+                    sm.off[tid] = ld_stream_u32(slot + 4, pol) >> 2;
+                    if ((uint32_t)tid == nv - 1) {                 // end of the tile's last record
+                        if (t0 + nv < nslots) {
+                            sm.off[nv] = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
+                        } else {
+                            const uint32_t o = ld_stream_u32(slot + 4, pol);
+                            sm.off[nv] = (o >> 2) + 1 + (ld32(data + o) << wshift);
+                        }
+                    }
+                }
+                __syncthreads();
+                if ((uint32_t)tid < nv) {
+                    const uint32_t deg = (sm.off[tid + 1] - sm.off[tid] - 1) >> wshift;
+                    const float xv = ld_stream_f32(x + start + t0 + tid, pol);
+                    float c = 0.f;
+                    if (deg == 0) dang += (double)xv;
+                    else c = d * xv / (float)deg;
+                    sm.c[tid] = c;
+                }
+                __syncthreads();
+                const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
+                const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
+                for (uint32_t qb = qbeg + tid; qb < qend; qb += kThreads * kPrUnroll) {
+                    uint4 v[kPrUnroll];
+#pragma unroll
+                    for (int u = 0; u < kPrUnroll; ++u) {
+                        const uint32_t q = qb + u * kThreads;
+                        if (q < qend) v[u] = ld_stream_v4(q4 + q, pol);
+                    }
+#pragma unroll
+                    for (int u = 0; u < kPrUnroll; ++u) {
+                        const uint32_t q = qb + u * kThreads;
+                        if (q >= qend) break;
+                        const uint32_t w0 = 4 * q;
+                        uint32_t lo = 0, hi = nv;               // off[lo] <= max(w0, W0) < off[hi]
+                        while (hi - lo > 1) {
+                            const uint32_t mid = (lo + hi) >> 1;
+                            if (sm.off[mid] <= w0) lo = mid; else hi = mid;
+                        }
+                        uint32_t j = lo, cur = sm.off[j], nxt = sm.off[j + 1];
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            const uint32_t w = w0 + k;
+                            if (w < W0 || w >= W1) continue;
+                            while (w >= nxt) {
+                                ++j;
+                                cur = nxt;
+                                nxt = sm.off[j + 1];
+                            }
+                            const uint32_t rel = w - cur;     // 0 = ADJLIST_SZ word; > deg = weight words
+                            if (rel == 0 || rel > ((nxt - cur - 1) >> wshift)) continue;
+                            em.edge(pr_decode(word_of(v[u], k), enc, ps.rvt_start), sm.c[j]);
+                        }
+                    }
+                }
+                __syncthreads();
+            }
+        }
+        em.flush();
+    }
     __syncthreads();
     if (kDense) {
         for (uint32_t i = tid; i < n_dense; i += kThreads) {
@@ -147,7 +234,6 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             if (k != kHotEmpty && v != 0.f) atomicAdd(acc + k, v);
         }
     }
-    double dang = op.dang;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) dang += __shfl_down_sync(0xFFFFFFFFu, dang, o);
     if ((tid & 31) == 0 && dang != 0.0) atomicAdd(dang_out, dang);
@@ -230,11 +316,13 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     GTS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
     int grid = 0;
     GTS_TRY(sms_grid(c, (const void*)kern, kThreads, dyn, &grid));
-    // Optional L2 persistence for the hot head of WA (ordered graphs: the most
-    // updated entries are acc[0, W)).  GTS_L2_PERSIST=<MiB> enables it.
+    // L2 persistence for the hot head of WA: on a degree-ordered graph the most
+    // updated entries are acc[0, W) (W = 96 MiB by default, clipped to the
+    // device's persisting-L2 limit); GTS_L2_PERSIST=<MiB> overrides, 0 disables.
     bool persist = false;
-    if (g->ordered && getenv("GTS_L2_PERSIST")) {
-        size_t want = (size_t)atol(getenv("GTS_L2_PERSIST")) << 20;
+    const char* pe = getenv("GTS_L2_PERSIST");
+    if (g->ordered && (!pe || atol(pe) > 0)) {
+        size_t want = (size_t)(pe ? atol(pe) : 96) << 20;
         cudaDeviceProp prop;
         GTS_CUDA(cudaGetDeviceProperties(&prop, c->device));
         want = std::min<size_t>(want, prop.persistingL2CacheMaxSize);

@@ -138,3 +138,9 @@ def test_bfs_rejects_bad_src():
     g = inputs.path(3)
     with pytest.raises(ValueError):
         oracle.bfs(g.row_ptr, g.col, 3)
+
+
+def test_generator_lean_mode_same_graph():
+    a = inputs.rmat(13)
+    b = inputs.rmat(13, lean=True)
+    assert np.array_equal(a.row_ptr, b.row_ptr) and np.array_equal(a.col, b.col)
