@@ -310,8 +310,10 @@ __global__ void gather_kernel(uint32_t* out, const uint32_t* __restrict__ vals, 
 __global__ void label_min_kernel(uint32_t* minorig, const uint32_t* __restrict__ label,
                                  const uint32_t* __restrict__ old_of_new, uint64_t n) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
-        atomicMin(minorig + label[i], old_of_new[i]);
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const uint32_t l = label[i], o = old_of_new[i];
+        if (o < __ldcg(minorig + l)) atomicMin(minorig + l, o);   // test first: giant components share one label
+    }
 }
 
 __global__ void label_map_kernel(uint32_t* tmp, const uint32_t* __restrict__ label, const uint32_t* __restrict__ minorig,

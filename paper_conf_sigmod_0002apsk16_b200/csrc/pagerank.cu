@@ -31,21 +31,46 @@
 
 namespace gts {
 
+// Hot-destination modes of the scatter:
+//   kHash    : natural VID order; the builder's top-4096 in-degree vertices in a
+//              bucketed two-choice hash table in shared memory
+//   kDense   : degree-ordered pages; hot = internal IDs [0, kHotDense), one
+//              shared-memory array per CTA
+//   kCluster : degree-ordered pages; hot = [0, kClusterCTAs * kClusterSlice),
+//              spread over the distributed shared memory of a thread-block
+//              cluster (red.shared::cluster on the owner CTA's slice)
+enum PrMode : int { kHash = 0, kDense = 1, kCluster = 2 };
+constexpr int kClusterCTAs = 4;
+constexpr uint32_t kClusterSlice = 51200;          // floats per CTA (200 KiB)
+constexpr uint32_t kClusterHot = kClusterCTAs * kClusterSlice;
+
+__device__ __forceinline__ void dsmem_red_add(float* local_base, uint32_t rank, uint32_t idx, float c) {
+    const uint32_t la = (uint32_t)__cvta_generic_to_shared(local_base + idx);
+    uint32_t ra;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(la), "r"(rank));
+    asm volatile("red.shared::cluster.add.f32 [%0], %1;" ::"r"(ra), "f"(c) : "memory");
+}
+
 // Per-thread destination emitter: combines runs of equal destinations (rows
-// are sorted), routes hot destinations to the CTA's shared-memory partial sums
-// and everything else to a fire-and-forget fp32 red.add into acc.
-template <bool kDense>
+// are sorted), routes hot destinations to shared-memory partial sums and
+// everything else to a fire-and-forget fp32 red.add into acc.
+template <int kMode>
 struct PrEmitter {
     float* acc;
-    const uint32_t* hkeys;   // shared memory, kHotSlots (hash-table mode)
-    float* hacc;             // shared memory, kHotSlots (hash) or kHotDense (dense) partial sums
+    const uint32_t* hkeys;   // kHash: shared memory keys
+    float* hacc;             // shared memory partial sums (this CTA's slice in kCluster)
     uint32_t last;
     float sum;
     bool has;
 
     __device__ __forceinline__ void emit(uint32_t dst, float c) {
-        if (kDense) {                                   // degree-ordered graph: hot = [0, kHotDense)
+        if (kMode == kDense) {
             if (dst < kHotDense) atomicAdd(hacc + dst, c);
+            else atomicAdd(acc + dst, c);
+            return;
+        }
+        if (kMode == kCluster) {
+            if (dst < kClusterHot) dsmem_red_add(hacc, dst / kClusterSlice, dst % kClusterSlice, c);
             else atomicAdd(acc + dst, c);
             return;
         }
@@ -76,47 +101,59 @@ struct PrEmitter {
     }
 };
 
-constexpr size_t kPrDynSmem = kHotSlots * (sizeof(uint32_t) + sizeof(float));
-constexpr size_t kPrDynSmemDense = kHotDense * sizeof(float);
 constexpr int kPrUnroll = 4;            // 16-byte loads in flight per thread
 
+template <int T>
 struct PrSmem {
-    uint32_t off[kTile + 1];            // page-relative word index of each record of the tile; off[nv] = end
-    float c[kTile];                     // d * x_u / outdeg(u)
+    uint32_t off[T + 1];                // page-relative word index of each record of the tile; off[nv] = end
+    float c[T];                         // d * x_u / outdeg(u)
     uint32_t item;
 };
+
+template <int kMode>
+constexpr size_t pr_dyn_smem() {
+    return kMode == kHash ? kHotSlots * (sizeof(uint32_t) + sizeof(float))
+                          : (kMode == kDense ? kHotDense * sizeof(float) : kClusterSlice * sizeof(float));
+}
 
 __device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const uint32_t* rvt) {
     return enc == GTS_ENTRY_VID32 ? e : __ldg(rvt + (e >> 16)) + (e & 0xFFFFu);
 }
 
-// K_PR_SP / K_PR_LP (Alg 4/5) for a persistent CTA.  The record region of a
-// tile of 512 consecutive vertices is one contiguous word range (records are
-// packed in VID order from offset 0), streamed with 16-byte evict_first loads,
-// kPrUnroll in flight per thread; the owner of each 4-word group is found by a
-// binary search over the tile's record offsets in shared memory.
-template <bool kWeighted, bool kDense>
-__global__ void __launch_bounds__(kThreads, 2)
+__device__ __forceinline__ void cluster_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+// K_PR_SP / K_PR_LP (Alg 4/5) for a persistent CTA of T threads.  The record
+// region of a tile of T consecutive vertices is one contiguous word range
+// (records are packed in VID order from offset 0), streamed with 16-byte
+// evict_first loads, kPrUnroll in flight per thread; the owner of each 4-word
+// group is found by a binary search over the tile's record offsets.
+template <bool kWeighted, int kMode, int T, int kMinBlocks>
+__global__ void __launch_bounds__(T, kMinBlocks)
 pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__ hot_keys,
-                  float d, double* dang_out, uint32_t* work_ctr, uint32_t n_dense) {
-    __shared__ PrSmem sm;
+                  float d, double* dang_out, uint32_t* work_ctr, uint32_t n_hot) {
+    __shared__ PrSmem<T> sm;
     extern __shared__ uint4 dyn_smem[];
     uint32_t* hkeys = reinterpret_cast<uint32_t*>(dyn_smem);
-    float* hacc = kDense ? reinterpret_cast<float*>(dyn_smem) : reinterpret_cast<float*>(hkeys + kHotSlots);
+    float* hacc = kMode == kHash ? reinterpret_cast<float*>(hkeys + kHotSlots) : reinterpret_cast<float*>(dyn_smem);
     const int tid = threadIdx.x;
-    if (kDense) {
-        for (uint32_t i = tid; i < kHotDense; i += kThreads) hacc[i] = 0.f;
-    } else {
-        for (uint32_t i = tid; i < kHotSlots; i += kThreads) {
+    if (kMode == kHash) {
+        for (uint32_t i = tid; i < kHotSlots; i += T) {
             hkeys[i] = __ldg(hot_keys + i);
             hacc[i] = 0.f;
         }
+    } else {
+        const uint32_t nh = kMode == kDense ? kHotDense : kClusterSlice;
+        for (uint32_t i = tid; i < nh; i += T) hacc[i] = 0.f;
     }
+    if (kMode == kCluster) cluster_sync();   // every slice is zeroed before any remote add
+    else __syncthreads();
     const uint64_t pol = policy_evict_first();
     const uint32_t count = ps.count;
     const uint32_t enc = ps.entry_encoding;
     constexpr uint32_t wshift = kWeighted ? 1 : 0;
-    PrEmitter<kDense> em{acc, hkeys, hacc, 0u, 0.f, false};
+    PrEmitter<kMode> em{acc, hkeys, hacc, 0u, 0.f, false};
     double dang = 0.0;
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
@@ -137,16 +174,16 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             const uint32_t len = ld32(data);
             const float c = d * __ldg(x + vid) / (float)total;
             const uint32_t wend = 1 + len, qend = (wend + 3) >> 2;
-            for (uint32_t qb = tid; qb < qend; qb += kThreads * kPrUnroll) {
+            for (uint32_t qb = tid; qb < qend; qb += T * kPrUnroll) {
                 uint4 v[kPrUnroll];
 #pragma unroll
                 for (int u = 0; u < kPrUnroll; ++u) {
-                    const uint32_t q = qb + u * kThreads;
+                    const uint32_t q = qb + u * T;
                     if (q < qend) v[u] = ld_stream_v4(q4 + q, pol);
                 }
 #pragma unroll
                 for (int u = 0; u < kPrUnroll; ++u) {
-                    const uint32_t q = qb + u * kThreads;
+                    const uint32_t q = qb + u * T;
                     if (q >= qend) break;
 #pragma unroll
                     for (int k = 0; k < 4; ++k) {
@@ -157,8 +194,8 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             }
         } else {
             const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
-            for (uint32_t t0 = 0; t0 < nslots; t0 += kTile) {
-                const uint32_t nv = min((uint32_t)kTile, nslots - t0);
+            for (uint32_t t0 = 0; t0 < nslots; t0 += T) {
+                const uint32_t nv = min((uint32_t)T, nslots - t0);
                 if ((uint32_t)tid < nv) {
                     const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
                     sm.off[tid] = ld_stream_u32(slot + 4, pol) >> 2;
@@ -183,16 +220,16 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                 __syncthreads();
                 const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
                 const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
-                for (uint32_t qb = qbeg + tid; qb < qend; qb += kThreads * kPrUnroll) {
+                for (uint32_t qb = qbeg + tid; qb < qend; qb += T * kPrUnroll) {
                     uint4 v[kPrUnroll];
 #pragma unroll
                     for (int u = 0; u < kPrUnroll; ++u) {
-                        const uint32_t q = qb + u * kThreads;
+                        const uint32_t q = qb + u * T;
                         if (q < qend) v[u] = ld_stream_v4(q4 + q, pol);
                     }
 #pragma unroll
                     for (int u = 0; u < kPrUnroll; ++u) {
-                        const uint32_t q = qb + u * kThreads;
+                        const uint32_t q = qb + u * T;
                         if (q >= qend) break;
                         const uint32_t w0 = 4 * q;
                         uint32_t lo = 0, hi = nv;               // off[lo] <= max(w0, W0) < off[hi]
@@ -221,17 +258,25 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
         }
         em.flush();
     }
-    __syncthreads();
-    if (kDense) {
-        for (uint32_t i = tid; i < n_dense; i += kThreads) {
-            const float v = hacc[i];
-            if (v != 0.f) atomicAdd(acc + i, v);
-        }
-    } else {
-        for (uint32_t i = tid; i < kHotSlots; i += kThreads) {
+    if (kMode == kCluster) cluster_sync();   // all remote adds into my slice are done
+    else __syncthreads();
+    if (kMode == kHash) {
+        for (uint32_t i = tid; i < kHotSlots; i += T) {
             const uint32_t k = hkeys[i];
             const float v = hacc[i];
             if (k != kHotEmpty && v != 0.f) atomicAdd(acc + k, v);
+        }
+    } else {
+        uint32_t base = 0;
+        if (kMode == kCluster) {
+            uint32_t r;
+            asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+            base = r * kClusterSlice;
+        }
+        const uint32_t nh = kMode == kDense ? kHotDense : kClusterSlice;
+        for (uint32_t i = tid; i < nh && base + i < n_hot; i += T) {
+            const float v = hacc[i];
+            if (v != 0.f) atomicAdd(acc + base + i, v);
         }
     }
 #pragma unroll
@@ -309,13 +354,34 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     GTS_TRY(c->buf(kBufDang, 2 * sizeof(double), (void**)&dang));
     GTS_TRY(c->buf(kBufPrCtr, 4, (void**)&ctr));
     cudaStream_t s = c->stream;
-    auto kern = g->ordered ? (g->weighted ? pr_scatter_kernel<true, true> : pr_scatter_kernel<false, true>)
-                           : (g->weighted ? pr_scatter_kernel<true, false> : pr_scatter_kernel<false, false>);
-    const size_t dyn = g->ordered ? kPrDynSmemDense : kPrDynSmem;
-    const uint32_t n_dense = (uint32_t)std::min<uint64_t>(n, kHotDense);
+    // scatter variant: degree-ordered graphs use the dense hot set, or (GTS_PR_CLUSTER=1)
+    // the cluster-distributed one; natural-order graphs the hash table
+    const char* pc = getenv("GTS_PR_CLUSTER");
+    const int mode = !g->ordered ? kHash : ((pc && atoi(pc) > 0) ? kCluster : kDense);
+    const void* kern;
+    size_t dyn;
+    int threads;
+    if (mode == kHash) {
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kHash, 512, 2> : (const void*)pr_scatter_kernel<false, kHash, 512, 2>;
+        dyn = pr_dyn_smem<kHash>();
+        threads = 512;
+    } else if (mode == kDense) {
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, 512, 2> : (const void*)pr_scatter_kernel<false, kDense, 512, 2>;
+        dyn = pr_dyn_smem<kDense>();
+        threads = 512;
+    } else {
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kCluster, 1024, 1> : (const void*)pr_scatter_kernel<false, kCluster, 1024, 1>;
+        dyn = pr_dyn_smem<kCluster>();
+        threads = 1024;
+    }
+    const uint32_t n_hot = (uint32_t)std::min<uint64_t>(n, mode == kCluster ? kClusterHot : kHotDense);
     GTS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
     int grid = 0;
-    GTS_TRY(sms_grid(c, (const void*)kern, kThreads, dyn, &grid));
+    if (mode == kCluster) {
+        grid = (c->num_sms / kClusterCTAs) * kClusterCTAs;
+    } else {
+        GTS_TRY(sms_grid(c, kern, threads, dyn, &grid));
+    }
     // L2 persistence for the hot head of WA: on a degree-ordered graph the most
     // updated entries are acc[0, W) (W = 96 MiB by default, clipped to the
     // device's persisting-L2 limit); GTS_L2_PERSIST=<MiB> overrides, 0 disables.
@@ -354,8 +420,28 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                                 GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
                                 std::pair<cudaEvent_t, cudaEvent_t> e2;
                                 if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
-                                kern<<<std::min(grid, cap), kThreads, dyn, s>>>(ps, x, acc, c->dg.hot_keys,
-                                                                              (float)damping, D, ctr, n_dense);
+                                float dmp = (float)damping;
+                                const uint32_t* hk = c->dg.hot_keys;
+                                void* args[] = {(void*)&ps, (void*)&x, (void*)&acc, (void*)&hk, (void*)&dmp, (void*)&D,
+                                                (void*)&ctr, (void*)&n_hot};
+                                cudaLaunchConfig_t lc;
+                                std::memset(&lc, 0, sizeof(lc));
+                                int gsz = std::min(grid, cap);
+                                cudaLaunchAttribute at[1];
+                                if (mode == kCluster) {                 // whole clusters only
+                                    gsz = ((gsz + kClusterCTAs - 1) / kClusterCTAs) * kClusterCTAs;
+                                    at[0].id = cudaLaunchAttributeClusterDimension;
+                                    at[0].val.clusterDim.x = kClusterCTAs;
+                                    at[0].val.clusterDim.y = 1;
+                                    at[0].val.clusterDim.z = 1;
+                                    lc.attrs = at;
+                                    lc.numAttrs = 1;
+                                }
+                                lc.gridDim = dim3(gsz);
+                                lc.blockDim = dim3(threads);
+                                lc.dynamicSmemBytes = dyn;
+                                lc.stream = s;
+                                GTS_CUDA(cudaLaunchKernelExC(&lc, kern, args));
                                 if (timing) cudaEventRecord(e2.second, s);
                                 GTS_CUDA(cudaGetLastError());
                                 ++main_launches;
