@@ -307,13 +307,28 @@ __global__ void gather_kernel(uint32_t* out, const uint32_t* __restrict__ vals, 
     for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) out[v] = vals[idx[v]];
 }
 
+// min caller VID per component.  Each thread folds runs of equal labels in a
+// register before touching memory (a giant component shares one label, and a
+// read or atomic per vertex on that one address serialises on one L2 slice).
+__device__ __forceinline__ void label_min_flush(uint32_t* minorig, uint32_t l, uint32_t o) {
+    if (o < __ldcg(minorig + l)) atomicMin(minorig + l, o);
+}
+
 __global__ void label_min_kernel(uint32_t* minorig, const uint32_t* __restrict__ label,
                                  const uint32_t* __restrict__ old_of_new, uint64_t n) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    uint32_t cl = 0xFFFFFFFFu, cm = 0xFFFFFFFFu;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
         const uint32_t l = label[i], o = old_of_new[i];
-        if (o < __ldcg(minorig + l)) atomicMin(minorig + l, o);   // test first: giant components share one label
+        if (l == cl) {
+            cm = min(cm, o);
+        } else {
+            if (cl != 0xFFFFFFFFu) label_min_flush(minorig, cl, cm);
+            cl = l;
+            cm = o;
+        }
     }
+    if (cl != 0xFFFFFFFFu) label_min_flush(minorig, cl, cm);
 }
 
 __global__ void label_map_kernel(uint32_t* tmp, const uint32_t* __restrict__ label, const uint32_t* __restrict__ minorig,

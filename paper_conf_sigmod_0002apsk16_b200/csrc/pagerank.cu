@@ -36,20 +36,10 @@ namespace gts {
 //              bucketed two-choice hash table in shared memory
 //   kDense   : degree-ordered pages; hot = internal IDs [0, kHotDense), one
 //              shared-memory array per CTA
-//   kCluster : degree-ordered pages; hot = [0, kClusterCTAs * kClusterSlice),
-//              spread over the distributed shared memory of a thread-block
-//              cluster (red.shared::cluster on the owner CTA's slice)
-enum PrMode : int { kHash = 0, kDense = 1, kCluster = 2 };
-constexpr int kClusterCTAs = 4;
-constexpr uint32_t kClusterSlice = 51200;          // floats per CTA (200 KiB)
-constexpr uint32_t kClusterHot = kClusterCTAs * kClusterSlice;
-
-__device__ __forceinline__ void dsmem_red_add(float* local_base, uint32_t rank, uint32_t idx, float c) {
-    const uint32_t la = (uint32_t)__cvta_generic_to_shared(local_base + idx);
-    uint32_t ra;
-    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(la), "r"(rank));
-    asm volatile("red.shared::cluster.add.f32 [%0], %1;" ::"r"(ra), "f"(c) : "memory");
-}
+// (A third mode that spread a 4x larger hot set over the distributed shared
+// memory of a 4-CTA cluster with red.shared::cluster was built and measured:
+// 2.2x slower on RMAT-27 and a larger fp32 error at the hub; removed.)
+enum PrMode : int { kHash = 0, kDense = 1 };
 
 // Per-thread destination emitter: combines runs of equal destinations (rows
 // are sorted), routes hot destinations to shared-memory partial sums and
@@ -58,7 +48,7 @@ template <int kMode>
 struct PrEmitter {
     float* acc;
     const uint32_t* hkeys;   // kHash: shared memory keys
-    float* hacc;             // shared memory partial sums (this CTA's slice in kCluster)
+    float* hacc;             // shared memory partial sums
     uint32_t last;
     float sum;
     bool has;
@@ -66,11 +56,6 @@ struct PrEmitter {
     __device__ __forceinline__ void emit(uint32_t dst, float c) {
         if (kMode == kDense) {
             if (dst < kHotDense) atomicAdd(hacc + dst, c);
-            else atomicAdd(acc + dst, c);
-            return;
-        }
-        if (kMode == kCluster) {
-            if (dst < kClusterHot) dsmem_red_add(hacc, dst / kClusterSlice, dst % kClusterSlice, c);
             else atomicAdd(acc + dst, c);
             return;
         }
@@ -112,16 +97,11 @@ struct PrSmem {
 
 template <int kMode>
 constexpr size_t pr_dyn_smem() {
-    return kMode == kHash ? kHotSlots * (sizeof(uint32_t) + sizeof(float))
-                          : (kMode == kDense ? kHotDense * sizeof(float) : kClusterSlice * sizeof(float));
+    return kMode == kHash ? kHotSlots * (sizeof(uint32_t) + sizeof(float)) : kHotDense * sizeof(float);
 }
 
 __device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const uint32_t* rvt) {
     return enc == GTS_ENTRY_VID32 ? e : __ldg(rvt + (e >> 16)) + (e & 0xFFFFu);
-}
-
-__device__ __forceinline__ void cluster_sync() {
-    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
 // K_PR_SP / K_PR_LP (Alg 4/5) for a persistent CTA of T threads.  The record
@@ -144,11 +124,9 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             hacc[i] = 0.f;
         }
     } else {
-        const uint32_t nh = kMode == kDense ? kHotDense : kClusterSlice;
-        for (uint32_t i = tid; i < nh; i += T) hacc[i] = 0.f;
+        for (uint32_t i = tid; i < kHotDense; i += T) hacc[i] = 0.f;
     }
-    if (kMode == kCluster) cluster_sync();   // every slice is zeroed before any remote add
-    else __syncthreads();
+    __syncthreads();
     const uint64_t pol = policy_evict_first();
     const uint32_t count = ps.count;
     const uint32_t enc = ps.entry_encoding;
@@ -258,8 +236,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
         }
         em.flush();
     }
-    if (kMode == kCluster) cluster_sync();   // all remote adds into my slice are done
-    else __syncthreads();
+    __syncthreads();
     if (kMode == kHash) {
         for (uint32_t i = tid; i < kHotSlots; i += T) {
             const uint32_t k = hkeys[i];
@@ -267,16 +244,9 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             if (k != kHotEmpty && v != 0.f) atomicAdd(acc + k, v);
         }
     } else {
-        uint32_t base = 0;
-        if (kMode == kCluster) {
-            uint32_t r;
-            asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-            base = r * kClusterSlice;
-        }
-        const uint32_t nh = kMode == kDense ? kHotDense : kClusterSlice;
-        for (uint32_t i = tid; i < nh && base + i < n_hot; i += T) {
+        for (uint32_t i = tid; i < n_hot; i += T) {
             const float v = hacc[i];
-            if (v != 0.f) atomicAdd(acc + base + i, v);
+            if (v != 0.f) atomicAdd(acc + i, v);
         }
     }
 #pragma unroll
@@ -354,34 +324,21 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     GTS_TRY(c->buf(kBufDang, 2 * sizeof(double), (void**)&dang));
     GTS_TRY(c->buf(kBufPrCtr, 4, (void**)&ctr));
     cudaStream_t s = c->stream;
-    // scatter variant: degree-ordered graphs use the dense hot set, or (GTS_PR_CLUSTER=1)
-    // the cluster-distributed one; natural-order graphs the hash table
-    const char* pc = getenv("GTS_PR_CLUSTER");
-    const int mode = !g->ordered ? kHash : ((pc && atoi(pc) > 0) ? kCluster : kDense);
+    // scatter variant: degree-ordered graphs use the dense hot set, natural-order graphs the hash table
+    const int mode = g->ordered ? kDense : kHash;
     const void* kern;
-    size_t dyn;
-    int threads;
-    if (mode == kHash) {
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kHash, 512, 2> : (const void*)pr_scatter_kernel<false, kHash, 512, 2>;
-        dyn = pr_dyn_smem<kHash>();
-        threads = 512;
-    } else if (mode == kDense) {
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, 512, 2> : (const void*)pr_scatter_kernel<false, kDense, 512, 2>;
-        dyn = pr_dyn_smem<kDense>();
-        threads = 512;
-    } else {
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kCluster, 1024, 1> : (const void*)pr_scatter_kernel<false, kCluster, 1024, 1>;
-        dyn = pr_dyn_smem<kCluster>();
-        threads = 1024;
-    }
-    const uint32_t n_hot = (uint32_t)std::min<uint64_t>(n, mode == kCluster ? kClusterHot : kHotDense);
+    if (mode == kHash)
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kHash, kThreads, 2>
+                           : (const void*)pr_scatter_kernel<false, kHash, kThreads, 2>;
+    else
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, kThreads, 2>
+                           : (const void*)pr_scatter_kernel<false, kDense, kThreads, 2>;
+    const size_t dyn = mode == kHash ? pr_dyn_smem<kHash>() : pr_dyn_smem<kDense>();
+    const int threads = kThreads;
+    const uint32_t n_hot = (uint32_t)std::min<uint64_t>(n, kHotDense);
     GTS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
     int grid = 0;
-    if (mode == kCluster) {
-        grid = (c->num_sms / kClusterCTAs) * kClusterCTAs;
-    } else {
-        GTS_TRY(sms_grid(c, kern, threads, dyn, &grid));
-    }
+    GTS_TRY(sms_grid(c, kern, threads, dyn, &grid));
     // L2 persistence for the hot head of WA: on a degree-ordered graph the most
     // updated entries are acc[0, W) (W = 96 MiB by default, clipped to the
     // device's persisting-L2 limit); GTS_L2_PERSIST=<MiB> overrides, 0 disables.
@@ -427,16 +384,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                                 cudaLaunchConfig_t lc;
                                 std::memset(&lc, 0, sizeof(lc));
                                 int gsz = std::min(grid, cap);
-                                cudaLaunchAttribute at[1];
-                                if (mode == kCluster) {                 // whole clusters only
-                                    gsz = ((gsz + kClusterCTAs - 1) / kClusterCTAs) * kClusterCTAs;
-                                    at[0].id = cudaLaunchAttributeClusterDimension;
-                                    at[0].val.clusterDim.x = kClusterCTAs;
-                                    at[0].val.clusterDim.y = 1;
-                                    at[0].val.clusterDim.z = 1;
-                                    lc.attrs = at;
-                                    lc.numAttrs = 1;
-                                }
                                 lc.gridDim = dim3(gsz);
                                 lc.blockDim = dim3(threads);
                                 lc.dynamicSmemBytes = dyn;

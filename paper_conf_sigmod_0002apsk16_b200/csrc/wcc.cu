@@ -38,10 +38,8 @@ __device__ __forceinline__ uint32_t uf_find(uint32_t* parent, uint32_t x) {
     return cur;
 }
 
-// ra: the source's root as found when its record was opened (a hint: if it has
-// been hooked since, the failed CAS returns its new parent and the loop goes on)
-__device__ __forceinline__ bool uf_hook(uint32_t* parent, uint32_t ra, uint32_t b) {
-    uint32_t rb = uf_find(parent, b);
+__device__ __forceinline__ bool uf_hook(uint32_t* parent, uint32_t a, uint32_t b) {
+    uint32_t ra = uf_find(parent, a), rb = uf_find(parent, b);
     bool hooked = false;
     while (ra != rb) {
         if (ra < rb) {
@@ -64,16 +62,16 @@ struct WccOp {
     uint32_t* parent;
     bool changed;
     __device__ bool select(uint32_t) { return true; }
-    __device__ uint32_t payload(uint32_t v, uint32_t deg) { return deg ? uf_find(parent, v) : v; }
+    __device__ uint32_t payload(uint32_t v, uint32_t) { return v; }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t& pl) {
-        pl = uf_find(parent, vid);
+        pl = vid;
         return true;
     }
-    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t* pl,
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*,
                                           const uint32_t* src, const bool* valid) {
 #pragma unroll
         for (int q = 0; q < kEdgesPerThread; ++q)
-            if (valid[q] && src[q] != dst[q] && uf_hook(parent, pl[q], dst[q])) changed = true;
+            if (valid[q] && src[q] != dst[q] && uf_hook(parent, src[q], dst[q])) changed = true;
     }
     __device__ void end_page() {}
 };

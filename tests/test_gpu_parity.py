@@ -281,31 +281,13 @@ def test_degree_ordered_device_outputs(G, ctx):
 
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "instar", "multi"])
-@pytest.mark.parametrize("mode", ["cluster", "nopersist"])
+@pytest.mark.parametrize("mode", ["persist", "nopersist"])
 def test_pagerank_ordered_variants(G, ctx, name, mode, monkeypatch):
-    """Degree-ordered PageRank with the cluster-DSMEM hot set (GTS_PR_CLUSTER=1)
-    and without the L2 persistence window (GTS_L2_PERSIST=0)."""
-    if mode == "cluster":
-        monkeypatch.setenv("GTS_PR_CLUSTER", "1")
-    else:
+    """Degree-ordered PageRank with and without the L2 persistence window (GTS_L2_PERSIST=0)."""
+    if mode == "nopersist":
         monkeypatch.setenv("GTS_L2_PERSIST", "0")
     g, pb = graph(name)
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
     for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3)):
         got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, **kw)
         _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, mode, kw))
-
-
-@pytest.mark.parametrize("k", [4_600_000])
-def test_pagerank_in_star_hub_cluster(G, ctx, k, monkeypatch):
-    monkeypatch.setenv("GTS_PR_CLUSTER", "1")
-    n = k + 1
-    row_ptr = np.concatenate([[0, 0], np.arange(1, k + 1)]).astype(np.uint64)
-    gr = G.gts_build_pages(row_ptr, np.zeros(k, np.uint32), order=True)
-    got, _ = G.gts_pagerank(ctx, gr, 10, 0.85)
-    d = 0.85
-    leaf = eta = 1.0 / n
-    for _ in range(10):
-        leaf, eta = (1 - d) / n + d * eta / n, (1 - d) / n + d * (k * leaf + eta / n)
-    assert abs(got[0] - eta) / eta <= PR_MAX_REL
-    assert np.max(np.abs(got[1:] - leaf) / leaf) <= PR_MAX_REL
