@@ -43,9 +43,13 @@ __device__ __forceinline__ bool test_bit(const uint32_t* bm, uint32_t v) {
     return (__ldg(bm + (v >> 5)) >> (v & 31)) & 1u;
 }
 
+constexpr uint32_t kMaxTileWords = 8;   // tile mask words: up to 256 tiles (131,072 slots) per page
+
 struct TileSmem {
     uint32_t soff[kTile + 1];  // word index of every record of the tile (all slots); soff[nv] = end
     uint8_t sel[kTile];        // dense mode: vertex t of the tile is selected
+    uint32_t paytile[kTile];   // dense mode: payload of vertex t of the tile
+    uint32_t tmask[kMaxTileWords];   // tiles of the current page holding a frontier vertex
     uint32_t off[kTile];       // word index of the first ADJLIST entry of item j
     uint32_t deg[kTile];
     uint32_t src[kTile];       // VID of item j
@@ -96,6 +100,7 @@ __device__ __forceinline__ void tile_scan(bool sel, uint32_t deg, uint32_t& pos,
 // Op interface:
 //   static constexpr bool kReadWeights;  -- the op needs edge weights
 //   static constexpr bool kWeighted;     -- the pages carry weights (record = sz, adj[sz], w[sz])
+//   const uint32_t* frontier()                           -- bitmap behind select(), or nullptr (all)
 //   bool select(uint32_t vid)                            -- SP vertex expanded?
 //   uint32_t payload(uint32_t vid, uint32_t deg)         -- per selected vertex
 //   bool select_lp(uint32_t vid, uint32_t total_deg, uint32_t chunk_len, uint32_t& payload)
@@ -151,11 +156,32 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
         } else {
             const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
             const uint4* q4 = reinterpret_cast<const uint4*>(data);
-            for (uint32_t t0 = 0; t0 < nslots; t0 += kTile) {
+            const uint32_t ntiles = (nslots + kTile - 1) / kTile;
+            // Frontier-driven ops: one pass over the page's frontier-bitmap words marks
+            // the tiles that hold a selected vertex, so inactive tiles cost nothing.
+            const uint32_t* fbm = ntiles <= 32 * kMaxTileWords ? op.frontier() : nullptr;
+            if (fbm) {
+                for (uint32_t k = tid; k < kMaxTileWords; k += kThreads) sm.tmask[k] = 0u;
+                __syncthreads();
+                const uint32_t w0 = start >> 5, w1 = (start + nslots - 1) >> 5;
+                for (uint32_t w = w0 + tid; w <= w1; w += kThreads) {
+                    uint32_t bits = __ldg(fbm + w);
+                    if (w == w0) bits &= 0xFFFFFFFFu << (start & 31);
+                    if (w == w1 && ((start + nslots) & 31)) bits &= 0xFFFFFFFFu >> (32 - ((start + nslots) & 31));
+                    if (bits) {
+                        const uint32_t a = w * 32 + (__ffs(bits) - 1) - start;
+                        const uint32_t b = w * 32 + (31 - __clz(bits)) - start;
+                        for (uint32_t t = a / kTile; t <= b / kTile; ++t) atomicOr(&sm.tmask[t >> 5], 1u << (t & 31));
+                    }
+                }
+                __syncthreads();
+            }
+            for (uint32_t ti = 0; ti < ntiles; ++ti) {
+                if (fbm && !((sm.tmask[ti >> 5] >> (ti & 31)) & 1u)) continue;   // uniform: no frontier vertex
+                const uint32_t t0 = ti * kTile;
                 const uint32_t nv = min((uint32_t)kTile, nslots - t0);
                 const uint32_t v = start + t0 + tid;
                 const bool sel = (uint32_t)tid < nv && op.select(v);
-                if (!__syncthreads_or(sel)) continue;   // no frontier vertex in this tile
                 // record offsets of the whole tile (coalesced slot reads); the degree of
                 // a record is the distance to the next record (the last one reads its header)
                 if ((uint32_t)tid < nv) {
@@ -167,20 +193,20 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                         else sm.soff[nv] = (o >> 2) + 1 + (ld32(data + o) << (Op::kWeighted ? 1 : 0));
                     }
                 }
-                __syncthreads();
+                if (!__syncthreads_or(sel)) continue;   // (also publishes soff)
                 uint32_t deg = 0;
                 if ((uint32_t)tid < nv) deg = (sm.soff[tid + 1] - sm.soff[tid] - 1) >> (Op::kWeighted ? 1 : 0);
+                const uint32_t pay = sel ? op.payload(v, deg) : 0u;
+                if ((uint32_t)tid < nv) {               // published by tile_scan's barriers
+                    sm.sel[tid] = sel ? 1 : 0;
+                    sm.paytile[tid] = pay;
+                }
                 uint32_t pos, nf, excl, total;
                 tile_scan(sel, sel ? deg : 0u, pos, nf, excl, total, sm);
                 const uint32_t W0 = sm.soff[0], W1 = sm.soff[nv];
                 if (2 * total >= W1 - W0) {
                     // dense tile: stream the whole record region with 16-byte loads and
                     // act on the words of selected owners (hybrid micro-level, App E)
-                    if ((uint32_t)tid < nv) {
-                        sm.sel[tid] = sel ? 1 : 0;
-                        sm.payload[tid] = sel ? op.payload(v, deg) : 0u;
-                    }
-                    __syncthreads();
                     const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
                     for (uint32_t qb = qbeg + tid; qb < qend; qb += kThreads * kDenseUnroll) {
                         uint4 vv[kDenseUnroll];
@@ -221,7 +247,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                                 }
                                 valid[k] = ok;
                                 dst[k] = decode_entry(ps, word_of(vv[u], k));
-                                pl[k] = sm.payload[j];
+                                pl[k] = sm.paytile[j];
                                 src[k] = start + t0 + j;
                             }
                             op.edges(dst, wt, pl, src, valid);
@@ -235,7 +261,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     sm.off[pos] = sm.soff[tid] + 1;
                     sm.deg[pos] = deg;
                     sm.src[pos] = v;
-                    sm.payload[pos] = op.payload(v, deg);
+                    sm.payload[pos] = pay;
                     sm.pre[pos] = excl;
                 }
                 if (tid == 0) sm.pre[nf] = total;

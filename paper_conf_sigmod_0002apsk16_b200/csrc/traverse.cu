@@ -38,6 +38,7 @@ struct BfsOp {
     uint32_t* visited;
     uint32_t* next;
     unsigned long long nedges;
+    __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
         nedges += deg;
@@ -77,6 +78,7 @@ struct SsspOp {
     uint32_t* next;
     unsigned long long nedges;
     bool ovf;
+    __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t v, uint32_t deg) {
         nedges += deg;
@@ -117,6 +119,7 @@ struct SsspCheckOp {
     static constexpr bool kWeighted = true;
     const uint32_t* dist;
     bool bad;
+    __device__ const uint32_t* frontier() const { return nullptr; }
     __device__ bool select(uint32_t v) { return __ldg(dist + v) != GTS_UNREACHED; }
     __device__ uint32_t payload(uint32_t, uint32_t) { return 0u; }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t&) { return __ldg(dist + vid) != GTS_UNREACHED; }

@@ -61,6 +61,7 @@ struct WccOp {
     static constexpr bool kWeighted = W;
     uint32_t* parent;
     bool changed;
+    __device__ const uint32_t* frontier() const { return nullptr; }
     __device__ bool select(uint32_t) { return true; }
     __device__ uint32_t payload(uint32_t v, uint32_t) { return v; }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t& pl) {
