@@ -85,14 +85,24 @@ void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t
     vrange[world] = g->n;
 }
 
+// Pin the graph's host pages (and, for ordered graphs, the VID maps) once, so
+// uploads and streamed sweeps run at the link rate.  Failure is not an error:
+// pageable sources are still correct, only slower.
 int pinned_register(Graph* g) {
     if (g->host_registered || g->pages_alloc == 0) return GTS_OK;
     cudaError_t e = cudaHostRegister(g->pages, (g->pages_alloc + 4095) & ~(size_t)4095, cudaHostRegisterPortable);
     if (e != cudaSuccess) {
-        cudaGetLastError();   // pageable fallback for the copy source is still correct, only slower
+        cudaGetLastError();
         return GTS_OK;
     }
     g->host_registered = true;
+    if (g->ordered) {
+        if (cudaHostRegister(g->new_of_old.data(), g->n * 4, cudaHostRegisterPortable) == cudaSuccess &&
+            cudaHostRegister(g->old_of_new.data(), g->n * 4, cudaHostRegisterPortable) == cudaSuccess)
+            g->maps_registered = true;
+        else
+            cudaGetLastError();
+    }
     return GTS_OK;
 }
 
@@ -157,6 +167,7 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
                                      c->stream));
         GTS_CUDA(cudaMemcpyAsync(d.hot_keys, g->hot_keys.data(), kHotSlots * 4, cudaMemcpyHostToDevice, c->stream));
         if (g->ordered) {
+            GTS_TRY(pinned_register(g));
             GTS_CUDA(cudaMalloc(&d.new_of_old, g->n * 4));
             GTS_CUDA(cudaMalloc(&d.old_of_new, g->n * 4));
             GTS_CUDA(cudaMemcpyAsync(d.new_of_old, g->new_of_old.data(), g->n * 4, cudaMemcpyHostToDevice, c->stream));
@@ -477,6 +488,10 @@ extern "C" int gts_context_set_stream(gts_context* c, void* s) {
 extern "C" void gts_graph_free(gts_graph* g) {
     if (!g) return;
     if (g->host_registered) cudaHostUnregister(g->pages);
+    if (g->maps_registered) {
+        cudaHostUnregister(g->new_of_old.data());
+        cudaHostUnregister(g->old_of_new.data());
+    }
     std::free(g->pages);
     delete g;
 }

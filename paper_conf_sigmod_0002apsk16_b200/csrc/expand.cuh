@@ -44,6 +44,7 @@ __device__ __forceinline__ bool test_bit(const uint32_t* bm, uint32_t v) {
 }
 
 constexpr uint32_t kMaxTileWords = 8;   // tile mask words: up to 256 tiles (131,072 slots) per page
+constexpr uint32_t kListWords = 128;    // sparse pages: frontier bitmap words compacted per pass
 
 struct TileSmem {
     uint32_t soff[kTile + 1];  // word index of every record of the tile (all slots); soff[nv] = end
@@ -58,6 +59,8 @@ struct TileSmem {
     uint32_t wsum[kWarps];
     uint32_t wcnt[kWarps];
     uint32_t item;
+    uint32_t pcount;                 // frontier vertices of the current page
+    uint32_t list[kListWords * 32];  // sparse pages: compacted frontier vertices (slot indices)
 };
 
 // Tile scan: frontier compaction by __ballot_sync/__popc (position of each
@@ -111,6 +114,97 @@ __device__ __forceinline__ void tile_scan(bool sel, uint32_t deg, uint32_t& pos,
 // loaded back to back, so each thread has that many independent loads in
 // flight, and the op can issue its own per-edge loads (visited bits, dist,
 // labels) as a batch before acting on them.
+// Edge-parallel expansion of nf compacted items (sm.off/deg/src/payload/pre):
+// 4 consecutive edges per thread, one binary search per 4 edges.
+template <class Op>
+__device__ __forceinline__ void gather_items(const PageSet& ps, Op& op, TileSmem& sm, const uint32_t* words,
+                                             uint32_t nf, uint32_t total, uint64_t pol) {
+    const int tid = threadIdx.x;
+    for (uint32_t e0 = (uint32_t)tid * kEdgesPerThread; e0 < total; e0 += kThreads * kEdgesPerThread) {
+        uint32_t lo = 0, hi = nf;              // pre[lo] <= e0 < pre[hi]
+        while (hi - lo > 1) {
+            uint32_t mid = (lo + hi) >> 1;
+            if (sm.pre[mid] <= e0) lo = mid; else hi = mid;
+        }
+        uint32_t j = lo, nxt = sm.pre[lo + 1];
+        uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
+        bool valid[kEdgesPerThread];
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            const uint32_t e = e0 + q;
+            valid[q] = e < total;
+            if (valid[q]) {
+                while (e >= nxt) nxt = sm.pre[++j + 1];
+            }
+            const uint32_t local = e - sm.pre[j];
+            const uint32_t* adj = words + sm.off[j];
+            dst[q] = valid[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
+            w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_l1_u32(adj + sm.deg[j] + local, pol) : 0u;
+            pl[q] = sm.payload[j];
+            src[q] = sm.src[j];
+        }
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) dst[q] = decode_entry(ps, dst[q]);
+        op.edges(dst, w, pl, src, valid);
+    }
+}
+
+// Sparse page (frontier-driven ops, < 1/4 of the page's vertices selected):
+// compact the page's frontier vertices from the bitmap in passes of
+// kListWords words, then expand them in batches of kTile with gather_items.
+template <class Op>
+__device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, const uint8_t* data,
+                                   const uint8_t* end, uint32_t start, uint32_t nslots, const uint32_t* fbm,
+                                   uint64_t pol) {
+    const int tid = threadIdx.x;
+    const uint32_t* words = reinterpret_cast<const uint32_t*>(data);
+    const uint32_t w0 = start >> 5, w1 = (start + nslots - 1) >> 5;
+    for (uint32_t wb = w0; wb <= w1; wb += kListWords) {
+        const uint32_t w = wb + tid;
+        uint32_t bits = 0;
+        if ((uint32_t)tid < kListWords && w <= w1) {
+            bits = __ldg(fbm + w);
+            if (w == w0) bits &= 0xFFFFFFFFu << (start & 31);
+            if (w == w1 && ((start + nslots) & 31)) bits &= 0xFFFFFFFFu >> (32 - ((start + nslots) & 31));
+        }
+        uint32_t pos, nw, excl, tot;
+        tile_scan(bits != 0, __popc(bits), pos, nw, excl, tot, sm);
+        uint32_t k = excl;
+        while (bits) {
+            const uint32_t b = __ffs(bits) - 1;
+            sm.list[k++] = w * 32 + b - start;
+            bits &= bits - 1;
+        }
+        __syncthreads();
+        for (uint32_t b0 = 0; b0 < tot; b0 += kTile) {
+            const uint32_t kk = b0 + tid;
+            const bool sel = kk < tot;
+            uint32_t j = 0, off = 0, deg = 0;
+            if (sel) {
+                j = sm.list[kk];
+                const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(j + 1);
+                off = ld_stream_u32(slot + 4, pol);
+                deg = ld_stream_u32(data + off, pol) ;
+            }
+            const uint32_t v = start + j;
+            const uint32_t pay = sel ? op.payload(v, deg) : 0u;
+            uint32_t p2, nf, ex2, total;
+            tile_scan(sel, deg, p2, nf, ex2, total, sm);
+            if (sel) {
+                sm.off[p2] = off / 4 + 1;
+                sm.deg[p2] = deg;
+                sm.src[p2] = v;
+                sm.payload[p2] = pay;
+                sm.pre[p2] = ex2;
+            }
+            if (tid == 0) sm.pre[nf] = total;
+            __syncthreads();
+            gather_items(ps, op, sm, words, nf, total, pol);
+            __syncthreads();
+        }
+    }
+}
+
 template <class Op>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
     const uint32_t count = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
@@ -162,19 +256,28 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             const uint32_t* fbm = ntiles <= 32 * kMaxTileWords ? op.frontier() : nullptr;
             if (fbm) {
                 for (uint32_t k = tid; k < kMaxTileWords; k += kThreads) sm.tmask[k] = 0u;
+                if (tid == 0) sm.pcount = 0;
                 __syncthreads();
+                uint32_t cnt = 0;
                 const uint32_t w0 = start >> 5, w1 = (start + nslots - 1) >> 5;
                 for (uint32_t w = w0 + tid; w <= w1; w += kThreads) {
                     uint32_t bits = __ldg(fbm + w);
                     if (w == w0) bits &= 0xFFFFFFFFu << (start & 31);
                     if (w == w1 && ((start + nslots) & 31)) bits &= 0xFFFFFFFFu >> (32 - ((start + nslots) & 31));
+                    cnt += __popc(bits);
                     if (bits) {
                         const uint32_t a = w * 32 + (__ffs(bits) - 1) - start;
                         const uint32_t b = w * 32 + (31 - __clz(bits)) - start;
                         for (uint32_t t = a / kTile; t <= b / kTile; ++t) atomicOr(&sm.tmask[t >> 5], 1u << (t & 31));
                     }
                 }
+                if (cnt) atomicAdd(&sm.pcount, cnt);
                 __syncthreads();
+                if (4 * sm.pcount < nslots) {          // uniform: sparse page -> compacted batches
+                    expand_sparse_page(ps, op, sm, data, end, start, nslots, fbm, pol);
+                    op.end_page();
+                    continue;
+                }
             }
             for (uint32_t ti = 0; ti < ntiles; ++ti) {
                 if (fbm && !((sm.tmask[ti >> 5] >> (ti & 31)) & 1u)) continue;   // uniform: no frontier vertex
@@ -266,33 +369,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 }
                 if (tid == 0) sm.pre[nf] = total;
                 __syncthreads();
-                for (uint32_t e0 = (uint32_t)tid * kEdgesPerThread; e0 < total; e0 += kThreads * kEdgesPerThread) {
-                    uint32_t lo = 0, hi = nf;              // pre[lo] <= e0 < pre[hi]
-                    while (hi - lo > 1) {
-                        uint32_t mid = (lo + hi) >> 1;
-                        if (sm.pre[mid] <= e0) lo = mid; else hi = mid;
-                    }
-                    uint32_t j = lo, nxt = sm.pre[lo + 1];
-                    uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
-                    bool valid[kEdgesPerThread];
-#pragma unroll
-                    for (int q = 0; q < kEdgesPerThread; ++q) {
-                        const uint32_t e = e0 + q;
-                        valid[q] = e < total;
-                        if (valid[q]) {
-                            while (e >= nxt) nxt = sm.pre[++j + 1];
-                        }
-                        const uint32_t local = e - sm.pre[j];
-                        const uint32_t* adj = words + sm.off[j];
-                        dst[q] = valid[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
-                        w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_l1_u32(adj + sm.deg[j] + local, pol) : 0u;
-                        pl[q] = sm.payload[j];
-                        src[q] = sm.src[j];
-                    }
-#pragma unroll
-                    for (int q = 0; q < kEdgesPerThread; ++q) dst[q] = decode_entry(ps, dst[q]);
-                    op.edges(dst, w, pl, src, valid);
-                }
+                gather_items(ps, op, sm, words, nf, total, pol);
                 __syncthreads();
             }
         }

@@ -62,7 +62,8 @@ struct Graph {
     bool ordered = false;              // GTS_BUILD_DEGREE_ORDER: pages hold internal IDs
     std::vector<uint32_t> new_of_old;  // caller VID -> internal ID (ordered graphs)
     std::vector<uint32_t> old_of_new;  // internal ID -> caller VID
-    bool host_registered = false;      // cudaHostRegister'ed by a context
+    bool host_registered = false;      // pages cudaHostRegister'ed by a context
+    bool maps_registered = false;      // new_of_old / old_of_new registered too
 };
 
 struct PagePlanEntry {
