@@ -160,6 +160,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="gts", choices=["gts", "reference"])
     ap.add_argument("--scale", type=int, default=27)
+    ap.add_argument("--workload", default="rmat", choices=["rmat", "twitter"],
+                    help="rmat: RMAT-<scale> (configs[2]); twitter: Twitter-shaped (configs[1])")
     ap.add_argument("--ref-scale", type=int, default=None)
     ap.add_argument("--page-bytes", type=int, default=1 << 20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -196,9 +198,11 @@ def main():
     algos = args.algos.split(",")
 
     t0 = time.time()
-    g = inputs.rmat(args.scale)
+    g = inputs.rmat(args.scale) if args.workload == "rmat" else inputs.twitter_like()
     n, m = g.n, g.m
-    log(f"[rank {rank}] RMAT-{args.scale} generated n={n} m={m} in {time.time() - t0:.1f}s")
+    src = 0 if args.workload == "rmat" else int(np.argmax(np.diff(g.row_ptr)))
+    wname = f"rmat{args.scale}" if args.workload == "rmat" else "twitter_shaped"
+    log(f"[rank {rank}] {wname} generated n={n} m={m} in {time.time() - t0:.1f}s")
     t0 = time.time()
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=args.page_bytes, order=args.order)
     grw = None
@@ -232,11 +236,11 @@ def main():
             e1 = torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             if a == "bfs":
-                _, st = G.gts_bfs(ctx, gr, 0, out=lv, timing=True)
+                _, st = G.gts_bfs(ctx, gr, src, out=lv, timing=True)
             elif a == "pr":
                 _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=pr, timing=True)
             elif a == "sssp":
-                _, st = G.gts_sssp(ctx, grw, 0, out=ds, timing=True)
+                _, st = G.gts_sssp(ctx, grw, src, out=ds, timing=True)
             else:
                 _, st = G.gts_wcc(ctx, gr, out=lab, timing=True)
             e1.record(stream)
@@ -315,13 +319,20 @@ def main():
         ks, kl, bytes_per_launch = cand[dom]
         avg = ks / max(1, kl)
         ach = bytes_per_launch / avg / 1e9 if avg > 0 else 0.0
-        traffic = None
+        traffic, tj = None, {}
         tp = os.path.join(ROOT, "profiles", "traffic.json")
         if os.path.exists(tp):
-            traffic = json.load(open(tp)).get(dom)
+            tj = json.load(open(tp))
+            traffic = tj.get(dom)
         roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
                 "traffic": traffic, "algorithmic_bytes_per_launch": bytes_per_launch, "avg_launch_s": avg,
                 "share_of_step": ks / total_s if total_s else None, "peak_source": peak_src}
+        red = tj.get(dom + "_lts_red_sectors")
+        if red and avg > 0:   # the scatter's real ceiling: L2 atomic throughput
+            roof["l2_red"] = {"ops_per_launch_ncu": red, "achieved_gops": red / avg / 1e9,
+                              "ceiling_gops": tj.get("l2_red_ceiling_gops"),
+                              "frac": red / avg / 1e9 / tj.get("l2_red_ceiling_gops", 1.0),
+                              "ceiling_source": tj.get("_l2_red_source")}
 
     # end-to-end through the public API with host buffers (pages re-uploaded from pinned host memory)
     e2e = None
@@ -333,7 +344,7 @@ def main():
             ctx.evict(gr)
             barrier()
             t0 = time.perf_counter()
-            _, st = G.gts_bfs(ctx, gr, 0, out=hl)
+            _, st = G.gts_bfs(ctx, gr, src, out=hl)
             tb.append(maxred(time.perf_counter() - t0))
             ctx.evict(gr)
             barrier()
@@ -357,8 +368,10 @@ def main():
         line = {"metric": METRIC, "value": bfs_gteps, "unit": "GTEPS", "n_gpus": world, "steps": K,
                 "warmup": args.warmup, "ms_per_step": 1e3 * total_s / K, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-                "config": {"workload": f"rmat{args.scale}_bfs_pr_sssp_wcc", "scale": args.scale, "n": n, "m": m,
-                           "edge_factor": 16, "abc": [0.57, 0.19, 0.19], "seed": args.scale, "src": 0,
+                "config": {"workload": f"{wname}_bfs_pr_sssp_wcc", "scale": args.scale if args.workload == "rmat" else None,
+                           "n": n, "m": m, "edge_factor": 16 if args.workload == "rmat" else None,
+                           "abc": [0.57, 0.19, 0.19] if args.workload == "rmat" else None,
+                           "seed": args.scale if args.workload == "rmat" else inputs.TWITTER_SEED, "src": src,
                            "page_bytes": args.page_bytes, "num_pages": gst["num_pages"], "n_lp": gst["n_lp"],
                            "vertex_order": "in-degree (GTS_BUILD_DEGREE_ORDER)" if args.order else "VID",
                            "topo_bytes": gst["topo_bytes"], "residency": "resident",

@@ -112,3 +112,30 @@ def test_pagerank_full_properties(big):
     want = (1 - dmp) / n + dmp * (acc + D / n)
     rel = np.abs(a10[sample] - want) / want
     assert rel.max() <= 1e-4, (float(rel.max()), int(sample[np.argmax(rel)]))
+
+
+def test_twitter_shaped_full_size(gpu):
+    """BASELINE configs[1]: Twitter-shaped graph at full size (n = 41.65 M,
+    m = 1.47 B, degree-ordered 1 MiB pages): BFS and WCC bit-exact, PageRank
+    sum and lower-bound invariants."""
+    import torch
+    import paper_conf_sigmod_0002apsk16_b200 as G
+    g = inputs.twitter_like()
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=1 << 20, order=True)
+    st = gr.stats()
+    assert st["n_lp"] > 0
+    ctx = G.gts_context_create(0)
+    try:
+        src = int(np.argmax(np.diff(g.row_ptr)))
+        out = torch.empty(g.n, dtype=torch.int32, device="cuda")
+        G.gts_bfs(ctx, gr, src, out=out)
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), oracle.bfs(g.row_ptr, g.col, src))
+        G.gts_wcc(ctx, gr, out=out)
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), oracle.wcc(g.row_ptr, g.col))
+        x = torch.empty(g.n, dtype=torch.float32, device="cuda")
+        G.gts_pagerank(ctx, gr, 10, 0.85, out=x)
+        a = x.cpu().numpy().astype(np.float64)
+        assert abs(np.sum(np.sort(a)) - 1.0) <= 1e-4
+        assert np.all(a >= 0.15 / g.n * (1 - 1e-4))
+    finally:
+        ctx.free()
