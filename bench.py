@@ -319,15 +319,16 @@ def main():
         ks, kl, bytes_per_launch = cand[dom]
         avg = ks / max(1, kl)
         ach = bytes_per_launch / avg / 1e9 if avg > 0 else 0.0
-        traffic, tj = None, {}
+        traffic, tj, tw = None, {}, {}
         tp = os.path.join(ROOT, "profiles", "traffic.json")
-        if os.path.exists(tp):
+        if os.path.exists(tp):        # ncu --set full captures, per workload (profiles/)
             tj = json.load(open(tp))
-            traffic = tj.get(dom)
+            tw = tj.get(f"{wname}_bfs_pr_sssp_wcc", {}) if world == 1 else {}
+            traffic = tw.get(dom)
         roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
                 "traffic": traffic, "algorithmic_bytes_per_launch": bytes_per_launch, "avg_launch_s": avg,
                 "share_of_step": ks / total_s if total_s else None, "peak_source": peak_src}
-        red = tj.get(dom + "_lts_red_sectors")
+        red = tw.get(dom + "_lts_red_sectors")
         if red and avg > 0:   # the scatter's real ceiling: L2 atomic throughput
             roof["l2_red"] = {"ops_per_launch_ncu": red, "achieved_gops": red / avg / 1e9,
                               "ceiling_gops": tj.get("l2_red_ceiling_gops"),

@@ -174,7 +174,8 @@ typedef struct {
     uint32_t batch_pages;     /* streamed: pages per H2D batch (0 -> 8) */
     uint32_t out_location;    /* GTS_OUT_HOST (default) | GTS_OUT_DEVICE (out pointer is device memory on this rank's GPU) */
     uint32_t flags;           /* GTS_RUN_TIMING */
-    uint32_t reserved;
+    uint32_t cache_mib;       /* streamed BFS/SSSP: device LRU cache of topology pages across levels,
+                                 in MiB (cachedPIDMap, Alg 1 lines 8/16/29); 0 = none */
 } gts_run_config;
 
 typedef struct {
@@ -192,6 +193,8 @@ typedef struct {
     uint64_t main_kernel_launches;
     uint32_t levels_or_iters;
     uint32_t reserved;
+    uint64_t cache_hits;      /* streamed + cache: page visits served from the device cache */
+    uint64_t cache_misses;    /* streamed + cache: page visits copied from host memory */
 } gts_run_stats;
 
 /* BFS (App B.1, Alg 2/3 P:1494-1514; Alg 1 BFS-like path P:330-334).

@@ -106,6 +106,12 @@ int pinned_register(Graph* g) {
     return GTS_OK;
 }
 
+void free_cache(PageCache& pc) {
+    cudaFree(pc.buf);
+    cudaFree(pc.d_loc);
+    pc = PageCache();
+}
+
 static void free_devgraph(DevGraph& d) {
     cudaFree(d.pages);
     cudaFree(d.rvt_start);
@@ -217,6 +223,7 @@ int ensure_ring(Context* c, const Graph* g, uint32_t slots, uint32_t batch_pages
         }
         c->ring_events = true;
     }
+    if (!ring) return GTS_OK;    // events only
     return c->buf(60 /* kBufRing */, (size_t)slots * batch_pages * g->page_bytes, (void**)ring);
 }
 
@@ -443,6 +450,7 @@ extern "C" void gts_context_free(gts_context* c) {
     cudaDeviceSynchronize();
     free_devgraph(c->dg);
     for (auto& d : c->parked) free_devgraph(d);
+    free_cache(c->cache);
     for (auto& b : c->scratch) cudaFree(b.first);
     for (Timer* t : {&c->t_main, &c->t_finish, &c->t_merge, &c->t_h2d})
         for (auto& p : t->pairs) {
@@ -470,6 +478,7 @@ extern "C" int gts_context_evict(gts_context* c, const gts_graph* g) {
     cudaSetDevice(c->device);
     cudaStreamSynchronize(c->stream);
     if (!g || c->dg.uid == g->uid) free_devgraph(c->dg);
+    if (!g || c->cache.uid == g->uid) free_cache(c->cache);
     for (size_t i = c->parked.size(); i-- > 0;)
         if (!g || c->parked[i].uid == g->uid) {
             free_devgraph(c->parked[i]);

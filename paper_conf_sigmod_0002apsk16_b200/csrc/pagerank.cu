@@ -351,7 +351,10 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         want = std::min<size_t>(want, prop.persistingL2CacheMaxSize);
         want = std::min<size_t>(want, n * 4);
         if (want > 0) {
-            GTS_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
+            if (c->persist_limit != want) {           // set once per context (a device-wide limit)
+                GTS_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
+                c->persist_limit = want;
+            }
             cudaStreamAttrValue at;
             std::memset(&at, 0, sizeof(at));
             at.accessPolicyWindow.base_ptr = acc;
@@ -423,7 +426,8 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         std::memset(&at, 0, sizeof(at));
         at.accessPolicyWindow.num_bytes = 0;
         GTS_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &at));
-        GTS_CUDA(cudaCtxResetPersistingL2Cache());
+        const char* rs = getenv("GTS_L2_RESET");
+        if (!rs || atoi(rs) != 0) GTS_CUDA(cudaCtxResetPersistingL2Cache());   // release the lines for other work
     }
     if (strat_s) {              // gather every rank's finished range so all ranks return the full vector
         GTS_NCCL(ncclGroupStart());

@@ -76,6 +76,20 @@ struct DevGraph {
     std::vector<uint64_t> h_vrange;    // all ranks' WA ranges (world + 1)
 };
 
+// LRU cache of topology pages in device memory for streamed BFS-like sweeps
+// (cachedPIDMap; Alg 1 lines 8, 16, 29).
+struct PageCache {
+    uint64_t uid = 0;                  // graph the cache holds pages of
+    uint32_t cap = 0;                  // slots
+    uint32_t page_bytes = 0;
+    uint8_t* buf = nullptr;            // cap * page_bytes
+    uint32_t* d_loc = nullptr;         // [num_pages] page -> slot (UINT32_MAX = not cached)
+    std::vector<uint32_t> loc;         // host mirror of d_loc
+    std::vector<uint32_t> pid_of;      // slot -> page (UINT32_MAX = free)
+    std::vector<uint64_t> stamp;       // slot -> tick of last use
+    uint64_t tick = 0;
+};
+
 struct Timer {               // event pairs around launches; summed after the call synchronises
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> pairs;
     size_t used = 0;
@@ -89,6 +103,7 @@ struct Context {
     cudaStream_t own_stream = nullptr, stream = nullptr, copy_stream = nullptr;
     ncclComm_t comm = nullptr;
     DevGraph dg;                   // the graph of the current call
+    PageCache cache;               // streamed BFS/SSSP page cache
     std::vector<DevGraph> parked;  // other graphs kept resident (evicted LRU-first under memory pressure)
     std::vector<std::pair<void*, size_t>> scratch;
     void* h_small = nullptr;   // pinned host scratch (4 KiB)
@@ -98,6 +113,7 @@ struct Context {
     cudaEvent_t ring_ready[64], ring_free[64];
     bool ring_events = false;
     uint64_t launches = 0, main_launches = 0;
+    size_t persist_limit = 0;      // cudaLimitPersistingL2CacheSize set by this context
 
     int buf(int slot, size_t bytes, void** out);   // grow-only scratch device buffer
 };
@@ -113,6 +129,7 @@ int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_
 inline uint64_t map_src(const Graph* g, uint64_t src) { return g->ordered ? g->new_of_old[src] : src; }
 int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid);
 int pinned_register(Graph* g);
+void free_cache(PageCache& pc);
 // residency decision (GTS_RESIDENCY_AUTO: resident iff this rank's pages + attributes fit in free HBM)
 bool choose_streamed(Context* c, const Graph* g, const gts_run_config& rc, uint64_t attr_bytes);
 

@@ -23,6 +23,8 @@ constexpr int kBufRing = 60;
 struct SweepStats {
     uint64_t h2d_bytes = 0;
     uint64_t launches = 0;
+    uint64_t cache_hits = 0;
+    uint64_t cache_misses = 0;
 };
 
 int ensure_ring(Context* c, const Graph* g, uint32_t slots, uint32_t batch_pages, uint8_t** ring);
@@ -91,6 +93,120 @@ int sweep_pages(Context* c, const Graph* g, const gts_run_config& rc, bool strea
         GTS_CUDA(cudaEventRecord(c->ring_free[slot], c->stream));
         ss->h2d_bytes += (uint64_t)nb * pb;
         ss->launches++;
+    }
+    return GTS_OK;
+}
+
+constexpr int kBufCacheList = 61;
+
+// Streamed sweep through the LRU page cache: pages of L already cached are
+// processed in place (no copy); missing pages are copied into free or least
+// recently used slots (never one used in this sweep) in batches of B, each
+// batch's kernel waiting for its copy; pages that find no slot take the ring
+// path of sweep_pages.
+template <class F>
+int sweep_pages_cached(Context* c, const Graph* g, const gts_run_config& rc, const std::vector<uint32_t>& L,
+                       const uint32_t* d_L, F&& launch, SweepStats* ss) {
+    PageCache& pc = c->cache;
+    const size_t pb = g->page_bytes;
+    const uint32_t want = (uint32_t)std::min<uint64_t>(((uint64_t)rc.cache_mib << 20) / pb, g->num_pages);
+    if (pc.uid != g->uid || pc.cap != want || pc.page_bytes != g->page_bytes) {
+        free_cache(pc);
+        if (want == 0) return sweep_pages(c, g, rc, true, &L, d_L, (uint32_t)L.size(), nullptr, launch, ss);
+        cudaError_t e = cudaMalloc(&pc.buf, (size_t)want * pb);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(GTS_ENOMEM, "page cache: cudaMalloc(%zu) failed", (size_t)want * pb);
+        }
+        GTS_CUDA(cudaMalloc(&pc.d_loc, g->num_pages * 4));
+        pc.uid = g->uid;
+        pc.cap = want;
+        pc.page_bytes = g->page_bytes;
+        pc.loc.assign(g->num_pages, UINT32_MAX);
+        pc.pid_of.assign(want, UINT32_MAX);
+        pc.stamp.assign(want, 0);
+        pc.tick = 0;
+    }
+    const uint64_t tick = ++pc.tick;
+    std::vector<uint32_t> hits, miss;
+    for (uint32_t p : L) {
+        const uint32_t sl = pc.loc[p];
+        if (sl != UINT32_MAX) {
+            hits.push_back(p);
+            pc.stamp[sl] = tick;
+        } else {
+            miss.push_back(p);
+        }
+    }
+    // victims: free slots first, then least recently used slots not touched in this sweep
+    std::vector<uint32_t> cand;
+    for (uint32_t sl = 0; sl < pc.cap; ++sl)
+        if (pc.stamp[sl] < tick || pc.pid_of[sl] == UINT32_MAX) cand.push_back(sl);
+    const size_t ncached = std::min(cand.size(), miss.size());
+    if (ncached < cand.size())
+        std::nth_element(cand.begin(), cand.begin() + ncached, cand.end(), [&](uint32_t a, uint32_t b) {
+            const bool fa = pc.pid_of[a] == UINT32_MAX, fb = pc.pid_of[b] == UINT32_MAX;
+            return fa != fb ? fa : pc.stamp[a] < pc.stamp[b];
+        });
+    for (size_t k = 0; k < ncached; ++k) {
+        const uint32_t sl = cand[k], p = miss[k];
+        if (pc.pid_of[sl] != UINT32_MAX) pc.loc[pc.pid_of[sl]] = UINT32_MAX;
+        pc.pid_of[sl] = p;
+        pc.loc[p] = sl;
+        pc.stamp[sl] = tick;
+    }
+    ss->cache_hits += hits.size();
+    ss->cache_misses += miss.size();
+    // device list = [hits | cached misses]; the loc map goes up with it (the host synchronised
+    // after the previous level, so no kernel still reads the slots or the map)
+    std::vector<uint32_t> order(hits);
+    order.insert(order.end(), miss.begin(), miss.begin() + ncached);
+    uint32_t* d_list = nullptr;
+    GTS_TRY(c->buf(kBufCacheList, std::max<size_t>(order.size(), 1) * 4, (void**)&d_list));
+    if (!order.empty())
+        GTS_CUDA(cudaMemcpyAsync(d_list, order.data(), order.size() * 4, cudaMemcpyHostToDevice, c->stream));
+    GTS_CUDA(cudaMemcpyAsync(pc.d_loc, pc.loc.data(), g->num_pages * 4, cudaMemcpyHostToDevice, c->stream));
+    GTS_CUDA(cudaStreamSynchronize(c->stream));   // host vectors are reused below
+    auto cached_set = [&](uint32_t first, uint32_t cnt) {
+        PageSet ps;
+        ps.base = pc.buf;
+        ps.list = d_list + first;
+        ps.loc = pc.d_loc;
+        ps.d_count = nullptr;
+        ps.count = cnt;
+        ps.page_bytes = g->page_bytes;
+        ps.mode = kAddrByLoc;
+        ps.entry_encoding = g->entry_encoding;
+        ps.rvt_start = c->dg.rvt_start;
+        return ps;
+    };
+    if (!hits.empty()) {                          // overlaps the miss copies below
+        GTS_TRY(launch(cached_set(0, (uint32_t)hits.size()), (int)hits.size()));
+        ss->launches++;
+    }
+    GTS_TRY(ensure_ring(c, g, rc.ring_slots, rc.batch_pages, nullptr));
+    const uint32_t B = rc.batch_pages;
+    for (size_t b0 = 0, bi = 0; b0 < ncached; b0 += B, ++bi) {
+        const uint32_t nb = (uint32_t)std::min<size_t>(B, ncached - b0);
+        const uint32_t ev = bi % rc.ring_slots;
+        for (uint32_t k = 0; k < nb; ++k) {
+            const uint32_t p = miss[b0 + k];
+            GTS_CUDA(cudaMemcpyAsync(pc.buf + (size_t)pc.loc[p] * pb, g->pages + (size_t)p * pb, pb,
+                                     cudaMemcpyHostToDevice, c->copy_stream));
+        }
+        GTS_CUDA(cudaEventRecord(c->ring_ready[ev], c->copy_stream));
+        GTS_CUDA(cudaStreamWaitEvent(c->stream, c->ring_ready[ev], 0));
+        GTS_TRY(launch(cached_set((uint32_t)(hits.size() + b0), nb), (int)nb));
+        ss->h2d_bytes += (uint64_t)nb * pb;
+        ss->launches++;
+    }
+    if (ncached < miss.size()) {                  // no slot left: stream the rest through the ring
+        std::vector<uint32_t> rest(miss.begin() + ncached, miss.end());
+        uint32_t* d_rest = nullptr;
+        GTS_TRY(c->buf(kBufCacheList + 1, rest.size() * 4, (void**)&d_rest));
+        GTS_CUDA(cudaMemcpyAsync(d_rest, rest.data(), rest.size() * 4, cudaMemcpyHostToDevice, c->stream));
+        GTS_CUDA(cudaStreamSynchronize(c->stream));
+        GTS_TRY(sweep_pages(c, g, rc, true, &rest, d_rest, (uint32_t)rest.size(), nullptr, launch, ss));
     }
     return GTS_OK;
 }

@@ -38,8 +38,6 @@ struct BfsOp {
     uint32_t* visited;
     uint32_t* next;
     unsigned long long nedges;
-    const uint32_t* svis;      // shared-memory copy of visited[0, nsvis) taken at kernel start
-    uint32_t nsvis;
     __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
@@ -59,13 +57,7 @@ struct BfsOp {
                                           const bool* valid) {
         uint32_t vis[kEdgesPerThread];
 #pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q) {
-            // the start-of-level copy is a conservative filter: a set bit is final,
-            // a clear one falls through to the global test-and-set
-            const uint32_t wi = dst[q] >> 5;
-            const uint32_t sv = (valid[q] && wi < nsvis) ? svis[wi] : 0u;
-            vis[q] = !valid[q] ? ~0u : ((sv >> (dst[q] & 31)) & 1u) ? sv : __ldca(visited + wi);
-        }
+        for (int q = 0; q < kEdgesPerThread; ++q) vis[q] = valid[q] ? __ldca(visited + (dst[q] >> 5)) : ~0u;
 #pragma unroll
         for (int q = 0; q < kEdgesPerThread; ++q) {
             const uint32_t wi = dst[q] >> 5, b = 1u << (dst[q] & 31);
@@ -151,12 +143,9 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 template <bool W>
 __global__ void __launch_bounds__(kThreads, 2)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
-                  uint32_t* work_ctr, unsigned long long* edges_out, uint32_t nsvis) {
+                  uint32_t* work_ctr, unsigned long long* edges_out) {
     __shared__ TileSmem sm;
-    extern __shared__ uint32_t svis[];   // visited bits of the hottest (lowest-ID) vertices
-    for (uint32_t i = threadIdx.x; i < nsvis; i += kThreads) svis[i] = __ldcg(visited + i);
-    __syncthreads();
-    BfsOp<W> op{cur, visited, next, 0ull, svis, nsvis};
+    BfsOp<W> op{cur, visited, next, 0ull};
     expand_pages(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
@@ -246,8 +235,6 @@ struct Counters {               // device scratch, slot kCtr
     uint32_t flag2;
 };
 
-constexpr uint32_t kSharedVisitedWords = 16384;   // 64 KiB
-
 enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather };
 
 // pages holding vertex v among this rank's pages (Alg 1 line 5: "page ID containing start vertex")
@@ -323,31 +310,26 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     const void* kexp = algo == kBFS ? (g->weighted ? (const void*)bfs_expand_kernel<true>
                                                    : (const void*)bfs_expand_kernel<false>)
                                     : (const void*)sssp_expand_kernel;
-    // BFS: a shared-memory copy of the first visited words (64 KiB = the 512 K
-    // lowest IDs: on a degree-ordered graph the most-referenced vertices)
-    const uint32_t nsvis = algo == kBFS ? (uint32_t)std::min<uint64_t>(words, kSharedVisitedWords) : 0u;
-    const size_t svis_bytes = (size_t)nsvis * 4;
-    if (algo == kBFS) GTS_CUDA(cudaFuncSetAttribute(kexp, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)svis_bytes));
     int grid = 0;
-    GTS_TRY(sms_grid(c, kexp, kThreads, svis_bytes, &grid));
+    GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
     const int fin_grid = c->num_sms * 4;
     uint64_t pages_processed = l0.size(), nccl_bytes = 0;
     uint32_t levels = 0;
     Counters h;
     SweepStats ss;
     std::vector<uint32_t> h_list = l0;             // streamed mode: this level's pages on the host (ascending)
+    const bool cached = streamed && rc.cache_mib > 0;
     for (uint32_t L = 0;; ++L) {
-        GTS_TRY(sweep_pages(c, g, rc, streamed, &h_list, list, (uint32_t)h_list.size(), &ctr->list_count,
-                            [&](const PageSet& ps, int cap) -> int {
+        auto launch = [&](const PageSet& ps, int cap) -> int {
                                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
                                 if (algo == kBFS && g->weighted)
-                                    bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, svis_bytes, s>>>(
-                                        ps, cur, visited, next, &ctr->work, &ctr->edges, nsvis);
+                                    bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(
+                                        ps, cur, visited, next, &ctr->work, &ctr->edges);
                                 else if (algo == kBFS)
-                                    bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, svis_bytes, s>>>(
-                                        ps, cur, visited, next, &ctr->work, &ctr->edges, nsvis);
+                                    bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(
+                                        ps, cur, visited, next, &ctr->work, &ctr->edges);
                                 else
                                     sssp_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(
                                         ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag);
@@ -355,7 +337,10 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                 GTS_CUDA(cudaGetLastError());
                                 ++main_launches;
                                 return GTS_OK;
-                            }, &ss));
+                            };
+        if (cached) GTS_TRY(sweep_pages_cached(c, g, rc, h_list, list, launch, &ss));
+        else GTS_TRY(sweep_pages(c, g, rc, streamed, &h_list, list, (uint32_t)h_list.size(), &ctr->list_count,
+                                 launch, &ss));
         std::pair<cudaEvent_t, cudaEvent_t> ev;
         if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
         if (c->world > 1) {
@@ -434,6 +419,8 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         }
         st->pages_processed = pages_processed;
         st->h2d_bytes = ss.h2d_bytes;
+        st->cache_hits = ss.cache_hits;
+        st->cache_misses = ss.cache_misses;
         if (timing) st->h2d_s = c->t_h2d.sum_s();
         st->edges_traversed = h.edges;
         st->nccl_bytes = nccl_bytes;

@@ -60,7 +60,7 @@ class GraphStats(ctypes.Structure):
 
 class RunConfig(ctypes.Structure):
     _fields_ = [(k, ctypes.c_uint32) for k in ("struct_size", "strategy", "residency", "ring_slots",
-                                               "batch_pages", "out_location", "flags", "reserved")]
+                                               "batch_pages", "out_location", "flags", "cache_mib")]
 
 
 class RunStats(ctypes.Structure):
@@ -68,7 +68,8 @@ class RunStats(ctypes.Structure):
                                                "h2d_s")] + \
                [(k, ctypes.c_uint64) for k in ("h2d_bytes", "nccl_bytes", "pages_processed", "edges_traversed",
                                                "launches", "main_kernel_launches")] + \
-               [(k, ctypes.c_uint32) for k in ("levels_or_iters", "reserved")]
+               [(k, ctypes.c_uint32) for k in ("levels_or_iters", "reserved")] + \
+               [(k, ctypes.c_uint64) for k in ("cache_hits", "cache_misses")]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_ if k != "reserved"}
@@ -254,9 +255,9 @@ def gts_context_create(device=0, rank=0, world_size=1, unique_id: bytes | None =
     return Context(h, device, rank, world_size)
 
 
-def _run_config(strategy, residency, ring_slots, batch_pages, out_location, timing):
+def _run_config(strategy, residency, ring_slots, batch_pages, out_location, timing, cache_mib=0):
     return RunConfig(ctypes.sizeof(RunConfig), strategy, residency, ring_slots, batch_pages, out_location,
-                     GTS_RUN_TIMING if timing else 0, 0)
+                     GTS_RUN_TIMING if timing else 0, int(cache_mib))
 
 
 def _out(out, n, dtype):
@@ -277,10 +278,10 @@ def _out(out, n, dtype):
 
 
 def gts_bfs(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-            batch_pages=0, timing=False):
+            batch_pages=0, timing=False, cache_mib=0):
     """Returns (levels, stats dict)."""
     out, ptr, loc = _out(out, graph.n, np.uint32)
-    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing)
+    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib)
     st = RunStats()
     _check(_lib.gts_bfs(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()
@@ -297,9 +298,9 @@ def gts_pagerank(ctx, graph, iters=10, damping=0.85, dangling=GTS_DANGLING_UNIFO
 
 
 def gts_sssp(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-             batch_pages=0, timing=False):
+             batch_pages=0, timing=False, cache_mib=0):
     out, ptr, loc = _out(out, graph.n, np.uint32)
-    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing)
+    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib)
     st = RunStats()
     _check(_lib.gts_sssp(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()

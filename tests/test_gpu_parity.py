@@ -291,3 +291,33 @@ def test_pagerank_ordered_variants(G, ctx, name, mode, monkeypatch):
     for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3)):
         got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, **kw)
         _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, mode, kw))
+
+
+# ------------------------------------------------- streamed + LRU page cache ---
+
+@pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "path", "bintree"])
+@pytest.mark.parametrize("cache_pages", [1, 3, 16, 1 << 20])
+def test_streamed_page_cache(G, ctx, name, cache_pages):
+    """cachedPIDMap: pages of earlier levels stay in a device LRU cache; a
+    cache smaller than one level's page set spills to the ring.  Results are
+    identical to the oracle; with a cache that holds everything every page
+    crosses the link at most once."""
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
+    mib = max(1, (cache_pages * pb) >> 20) if cache_pages * pb >= (1 << 20) else 0
+    if mib == 0:
+        pytest.skip("cache granularity is 1 MiB")
+    kw = dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=2, cache_mib=mib)
+    src = int(np.argmax(np.diff(g.row_ptr)))
+    got, st = G.gts_bfs(ctx, gr, src, **kw)
+    assert np.array_equal(got, oracle.bfs(g.row_ptr, g.col, src))
+    assert st["cache_hits"] + st["cache_misses"] == st["pages_processed"]
+    npages = gr.stats()["num_pages"]
+    if mib * (1 << 20) >= npages * pb:
+        assert st["h2d_bytes"] <= npages * pb
+    got2, st2 = G.gts_bfs(ctx, gr, src, **kw)     # warm cache: reuse across calls
+    assert np.array_equal(got2, got)
+    w = inputs.edge_weights(g)
+    grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb)
+    got, _ = G.gts_sssp(ctx, grw, src, **kw)
+    assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, src))
