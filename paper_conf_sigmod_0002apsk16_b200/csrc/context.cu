@@ -427,6 +427,8 @@ extern "C" int gts_context_create(int device, int rank, int world_size, const ui
     cudaDeviceProp prop;
     GTS_CUDA(cudaGetDeviceProperties(&prop, device));
     c->num_sms = prop.multiProcessorCount;
+    c->persist_max = prop.persistingL2CacheMaxSize;
+    c->window_max = prop.accessPolicyMaxWindowSize;
     GTS_CUDA(cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking));
     GTS_CUDA(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
     c->stream = c->own_stream;

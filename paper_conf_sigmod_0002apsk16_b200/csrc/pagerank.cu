@@ -44,7 +44,7 @@ enum PrMode : int { kHash = 0, kDense = 1 };
 // Per-thread destination emitter: combines runs of equal destinations (rows
 // are sorted), routes hot destinations to shared-memory partial sums and
 // everything else to a fire-and-forget fp32 red.add into acc.
-template <int kMode>
+template <int kMode, uint32_t H>
 struct PrEmitter {
     float* acc;
     const uint32_t* hkeys;   // kHash: shared memory keys
@@ -55,7 +55,7 @@ struct PrEmitter {
 
     __device__ __forceinline__ void emit(uint32_t dst, float c) {
         if (kMode == kDense) {
-            if (dst < kHotDense) atomicAdd(hacc + dst, c);
+            if (dst < H) atomicAdd(hacc + dst, c);
             else atomicAdd(acc + dst, c);
             return;
         }
@@ -95,10 +95,14 @@ struct PrSmem {
     uint32_t item;
 };
 
-template <int kMode>
+template <int kMode, uint32_t H>
 constexpr size_t pr_dyn_smem() {
-    return kMode == kHash ? kHotSlots * (sizeof(uint32_t) + sizeof(float)) : kHotDense * sizeof(float);
+    return kMode == kHash ? kHotSlots * (sizeof(uint32_t) + sizeof(float)) : H * sizeof(float);
 }
+
+// dense hot-set sizes: 512-thread CTAs (2 per SM) hold kHotDense floats each;
+// 1024-thread CTAs (1 per SM) hold kHotDenseBig
+constexpr uint32_t kHotDenseBig = 53248;
 
 __device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const uint32_t* rvt) {
     return enc == GTS_ENTRY_VID32 ? e : __ldg(rvt + (e >> 16)) + (e & 0xFFFFu);
@@ -109,7 +113,7 @@ __device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const ui
 // (records are packed in VID order from offset 0), streamed with 16-byte
 // evict_first loads, kPrUnroll in flight per thread; the owner of each 4-word
 // group is found by a binary search over the tile's record offsets.
-template <bool kWeighted, int kMode, int T, int kMinBlocks>
+template <bool kWeighted, int kMode, int T, int kMinBlocks, uint32_t H>
 __global__ void __launch_bounds__(T, kMinBlocks)
 pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__ hot_keys,
                   float d, double* dang_out, uint32_t* work_ctr, uint32_t n_hot) {
@@ -124,14 +128,14 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             hacc[i] = 0.f;
         }
     } else {
-        for (uint32_t i = tid; i < kHotDense; i += T) hacc[i] = 0.f;
+        for (uint32_t i = tid; i < H; i += T) hacc[i] = 0.f;
     }
     __syncthreads();
     const uint64_t pol = policy_evict_first();
     const uint32_t count = ps.count;
     const uint32_t enc = ps.entry_encoding;
     constexpr uint32_t wshift = kWeighted ? 1 : 0;
-    PrEmitter<kMode> em{acc, hkeys, hacc, 0u, 0.f, false};
+    PrEmitter<kMode, H> em{acc, hkeys, hacc, 0u, 0.f, false};
     double dang = 0.0;
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
@@ -324,18 +328,34 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     GTS_TRY(c->buf(kBufDang, 2 * sizeof(double), (void**)&dang));
     GTS_TRY(c->buf(kBufPrCtr, 4, (void**)&ctr));
     cudaStream_t s = c->stream;
-    // scatter variant: degree-ordered graphs use the dense hot set, natural-order graphs the hash table
+    // scatter variant: degree-ordered graphs use the dense hot set, natural-order graphs the hash table;
+    // GTS_PR_BIG=1 selects 1024-thread CTAs (one per SM) with a 2.2x larger dense hot set
+    const char* pbig = getenv("GTS_PR_BIG");
+    const bool big = g->ordered && pbig && atoi(pbig) > 0;
     const int mode = g->ordered ? kDense : kHash;
     const void* kern;
-    if (mode == kHash)
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kHash, kThreads, 2>
-                           : (const void*)pr_scatter_kernel<false, kHash, kThreads, 2>;
-    else
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, kThreads, 2>
-                           : (const void*)pr_scatter_kernel<false, kDense, kThreads, 2>;
-    const size_t dyn = mode == kHash ? pr_dyn_smem<kHash>() : pr_dyn_smem<kDense>();
-    const int threads = kThreads;
-    const uint32_t n_hot = (uint32_t)std::min<uint64_t>(n, kHotDense);
+    size_t dyn;
+    int threads;
+    uint32_t n_hot;
+    if (mode == kHash) {
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kHash, kThreads, 2, 0>
+                           : (const void*)pr_scatter_kernel<false, kHash, kThreads, 2, 0>;
+        dyn = pr_dyn_smem<kHash, 0>();
+        threads = kThreads;
+        n_hot = 0;
+    } else if (!big) {
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, kThreads, 2, kHotDense>
+                           : (const void*)pr_scatter_kernel<false, kDense, kThreads, 2, kHotDense>;
+        dyn = pr_dyn_smem<kDense, kHotDense>();
+        threads = kThreads;
+        n_hot = (uint32_t)std::min<uint64_t>(n, kHotDense);
+    } else {
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, 1024, 1, kHotDenseBig>
+                           : (const void*)pr_scatter_kernel<false, kDense, 1024, 1, kHotDenseBig>;
+        dyn = pr_dyn_smem<kDense, kHotDenseBig>();
+        threads = 1024;
+        n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
+    }
     GTS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
     int grid = 0;
     GTS_TRY(sms_grid(c, kern, threads, dyn, &grid));
@@ -346,9 +366,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     const char* pe = getenv("GTS_L2_PERSIST");
     if (g->ordered && (!pe || atol(pe) > 0)) {
         size_t want = (size_t)(pe ? atol(pe) : 96) << 20;
-        cudaDeviceProp prop;
-        GTS_CUDA(cudaGetDeviceProperties(&prop, c->device));
-        want = std::min<size_t>(want, prop.persistingL2CacheMaxSize);
+        want = std::min<size_t>(want, c->persist_max);
         want = std::min<size_t>(want, n * 4);
         if (want > 0) {
             if (c->persist_limit != want) {           // set once per context (a device-wide limit)
@@ -358,7 +376,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
             cudaStreamAttrValue at;
             std::memset(&at, 0, sizeof(at));
             at.accessPolicyWindow.base_ptr = acc;
-            at.accessPolicyWindow.num_bytes = std::min<size_t>(want, prop.accessPolicyMaxWindowSize);
+            at.accessPolicyWindow.num_bytes = std::min<size_t>(want, c->window_max);
             at.accessPolicyWindow.hitRatio = 1.0f;
             at.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
             at.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;

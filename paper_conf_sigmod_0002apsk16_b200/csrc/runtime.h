@@ -114,6 +114,8 @@ struct Context {
     bool ring_events = false;
     uint64_t launches = 0, main_launches = 0;
     size_t persist_limit = 0;      // cudaLimitPersistingL2CacheSize set by this context
+    size_t persist_max = 0;        // device attributes, queried once
+    size_t window_max = 0;
 
     int buf(int slot, size_t bytes, void** out);   // grow-only scratch device buffer
 };

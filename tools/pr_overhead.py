@@ -14,7 +14,7 @@ gr = G.gts_build_pages(g.row_ptr, g.col, order=True)
 ctx = G.gts_context_create(0)
 x = torch.empty(g.n, dtype=torch.float32, device="cuda")
 G.gts_pagerank(ctx, gr, 1, out=x)
-for env in ({}, {"GTS_L2_RESET": "0"}, {"GTS_L2_PERSIST": "0"}):
+for env in ({}, {"GTS_L2_RESET": "0"}, {"GTS_L2_PERSIST": "0"}, {"GTS_PR_BIG": "1"}, {"GTS_PR_BIG": "1", "GTS_L2_RESET": "0"}):
     for k, v in env.items():
         os.environ[k] = v
     for it in (1, 10):
