@@ -153,6 +153,36 @@ def cpu_baseline(args):
             "bfs_s": t_bfs, "pagerank_s_per_iter": t_pr, "sample_m": g.m}
 
 
+def make_graph(args, rank, world, dist):
+    """The workload graph.  With N > 1 ranks on one node, rank 0 draws it once
+    and shares the CSR through /dev/shm (each rank then builds its own pages)."""
+    import inputs
+    gen = (lambda: inputs.rmat(args.scale)) if args.workload == "rmat" else inputs.twitter_like
+    if world == 1:
+        return gen()
+    tag = f"/dev/shm/gts_bench_{args.workload}_{args.scale}_{os.environ.get('MASTER_PORT', '0')}"
+    if rank == 0:
+        g = gen()
+        np.save(tag + "_rp.npy", g.row_ptr)
+        np.save(tag + "_col.npy", g.col)
+    dist.barrier()
+    if rank != 0:
+        g = inputs.CSR(np.load(tag + "_rp.npy", mmap_mode="r"), np.load(tag + "_col.npy", mmap_mode="r"))
+    return g
+
+
+def drop_shared_graph(args, rank, world, dist):
+    if world > 1:
+        dist.barrier()
+        if rank == 0:
+            tag = f"/dev/shm/gts_bench_{args.workload}_{args.scale}_{os.environ.get('MASTER_PORT', '0')}"
+            for suf in ("_rp.npy", "_col.npy"):
+                try:
+                    os.remove(tag + suf)
+                except OSError:
+                    pass
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -198,7 +228,7 @@ def main():
     algos = args.algos.split(",")
 
     t0 = time.time()
-    g = inputs.rmat(args.scale) if args.workload == "rmat" else inputs.twitter_like()
+    g = make_graph(args, rank, world, dist)
     n, m = g.n, g.m
     src = 0 if args.workload == "rmat" else int(np.argmax(np.diff(g.row_ptr)))
     wname = f"rmat{args.scale}" if args.workload == "rmat" else "twitter_shaped"
@@ -213,6 +243,7 @@ def main():
     gst = gr.stats()
     log(f"[rank {rank}] pages built in {time.time() - t0:.1f}s: {gst}")
     del g
+    drop_shared_graph(args, rank, world, dist)
 
     uid = None
     if world > 1:

@@ -1,0 +1,62 @@
+"""bench.py host logic on CPU: the N > 1 graph sharing through /dev/shm (gloo,
+world_size 2) and the reference arm's JSON line."""
+import json
+import os
+import socket
+import subprocess
+import sys
+
+import numpy as np
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, port, out):
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=2)
+    import bench
+    import inputs
+
+    class A:
+        workload = "rmat"
+        scale = 10
+
+    g = bench.make_graph(A, rank, 2, dist)
+    ref = inputs.rmat(10)
+    ok = bool(np.array_equal(g.col, ref.col) and np.array_equal(g.row_ptr, ref.row_ptr))
+    bench.drop_shared_graph(A, rank, 2, dist)
+    out[rank] = ok
+    dist.destroy_process_group()
+
+
+def test_graph_shared_across_ranks():
+    ctx = mp.get_context("spawn")
+    out = ctx.Manager().dict()
+    port = _port()
+    ps = [ctx.Process(target=_worker, args=(r, port, out)) for r in range(2)]
+    for p in ps:
+        p.start()
+    for p in ps:
+        p.join(120)
+    assert all(p.exitcode == 0 for p in ps) and out[0] and out[1]
+    assert not os.path.exists(f"/dev/shm/gts_bench_rmat_10_{port}_rp.npy")
+
+
+def test_reference_arm_line():
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--scale", "14",
+                        "--steps", "2", "--warmup", "1"], capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr
+    line = json.loads(r.stdout.strip().splitlines()[-1])
+    assert line["impl"] == "reference" and line["value"] > 0 and line["unit"] == "GTEPS"
+    assert line["cpu_baseline"]["kind"] == "oracle" and line["e2e"]["h2d_bytes_per_step"] == 0
