@@ -328,10 +328,11 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     GTS_TRY(c->buf(kBufDang, 2 * sizeof(double), (void**)&dang));
     GTS_TRY(c->buf(kBufPrCtr, 4, (void**)&ctr));
     cudaStream_t s = c->stream;
-    // scatter variant: degree-ordered graphs use the dense hot set, natural-order graphs the hash table;
-    // GTS_PR_BIG=1 selects 1024-thread CTAs (one per SM) with a 2.2x larger dense hot set
+    // scatter variant: degree-ordered graphs use the dense hot set held by one 1024-thread CTA per
+    // SM (53,248 floats; GTS_PR_BIG=0 selects two 512-thread CTAs with 24,576 each, 3% slower
+    // on RMAT-27); natural-order graphs the hash table
     const char* pbig = getenv("GTS_PR_BIG");
-    const bool big = g->ordered && pbig && atoi(pbig) > 0;
+    const bool big = g->ordered && (!pbig || atoi(pbig) > 0);
     const int mode = g->ordered ? kDense : kHash;
     const void* kern;
     size_t dyn;
