@@ -39,7 +39,50 @@ namespace gts {
 // (A third mode that spread a 4x larger hot set over the distributed shared
 // memory of a 4-CTA cluster with red.shared::cluster was built and measured:
 // 2.2x slower on RMAT-27 and a larger fp32 error at the hub; removed.)
-enum PrMode : int { kHash = 0, kDense = 1 };
+//   kRoute   : Strategy-S with routed updates (SURVEY 8(e) "S-route"): dense hot set
+//              as kDense; destinations in this rank's WA range [lo, hi) are added
+//              locally, all others are packed into per-owner (dst, value) buffers
+//              that the driver exchanges with NCCL send/recv; hot partial sums for
+//              non-local hot vertices go to a dense per-rank buffer reduced onto
+//              their owners.
+enum PrMode : int { kHash = 0, kDense = 1, kRoute = 2 };
+
+constexpr int kMaxRanks = 8;
+
+struct RouteParams {
+    float* acc_loc;                    // local WA: acc_loc[v - lo]
+    float* hot_out;                    // [n_hot] hot partials of vertices outside [lo, hi)
+    uint2* send;                       // (dst, float bits) pairs, peer p's region at send_off[p]
+    uint32_t* send_cnt;                // [nranks] pairs appended per peer
+    uint32_t* overflow;                // set if a peer region is full (capacity is an upper bound)
+    uint64_t vr[kMaxRanks + 1];        // WA ranges: rank p owns [vr[p], vr[p+1])
+    uint32_t send_off[kMaxRanks];
+    uint32_t send_cap[kMaxRanks];
+    uint64_t lo, hi;
+    int nranks;
+};
+
+__device__ __forceinline__ int route_owner(const RouteParams& rp, uint32_t v) {
+    int p = 0;
+    while (p < rp.nranks - 1 && (uint64_t)v >= rp.vr[p + 1]) ++p;
+    return p;
+}
+
+// append (dst, c) to the owner's buffer; lanes of a warp bound for the same
+// owner share one atomic on its counter
+__device__ __forceinline__ void route_push(const RouteParams& rp, uint32_t dst, float c) {
+    const int p = route_owner(rp, dst);
+    const uint32_t active = __activemask();
+    const uint32_t peers = __match_any_sync(active, p);
+    const int lane = threadIdx.x & 31;
+    const int leader = __ffs(peers) - 1;
+    uint32_t base = 0;
+    if (lane == leader) base = atomicAdd(rp.send_cnt + p, (uint32_t)__popc(peers));
+    base = __shfl_sync(peers, base, leader);
+    const uint32_t slot = base + __popc(peers & ((1u << lane) - 1u));
+    if (slot < rp.send_cap[p]) rp.send[rp.send_off[p] + slot] = make_uint2(dst, __float_as_uint(c));
+    else *rp.overflow = 1u;
+}
 
 // Per-thread destination emitter: combines runs of equal destinations (rows
 // are sorted), routes hot destinations to shared-memory partial sums and
@@ -49,11 +92,18 @@ struct PrEmitter {
     float* acc;
     const uint32_t* hkeys;   // kHash: shared memory keys
     float* hacc;             // shared memory partial sums
+    const RouteParams* rp;   // kRoute
     uint32_t last;
     float sum;
     bool has;
 
     __device__ __forceinline__ void emit(uint32_t dst, float c) {
+        if (kMode == kRoute) {
+            if (dst < H) atomicAdd(hacc + dst, c);
+            else if ((uint64_t)dst >= rp->lo && (uint64_t)dst < rp->hi) atomicAdd(rp->acc_loc + (dst - rp->lo), c);
+            else route_push(*rp, dst, c);
+            return;
+        }
         if (kMode == kDense) {
             if (dst < H) atomicAdd(hacc + dst, c);
             else atomicAdd(acc + dst, c);
@@ -97,7 +147,7 @@ struct PrSmem {
 
 template <int kMode, uint32_t H>
 constexpr size_t pr_dyn_smem() {
-    return kMode == kHash ? kHotSlots * (sizeof(uint32_t) + sizeof(float)) : H * sizeof(float);
+    return kMode == kHash ? kHotSlots * (sizeof(uint32_t) + sizeof(float)) : H * sizeof(float);   // kDense, kRoute
 }
 
 // dense hot-set sizes: 512-thread CTAs (2 per SM) hold kHotDense floats each;
@@ -116,7 +166,7 @@ __device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const ui
 template <bool kWeighted, int kMode, int T, int kMinBlocks, uint32_t H>
 __global__ void __launch_bounds__(T, kMinBlocks)
 pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__ hot_keys,
-                  float d, double* dang_out, uint32_t* work_ctr, uint32_t n_hot) {
+                  float d, double* dang_out, uint32_t* work_ctr, uint32_t n_hot, const RouteParams rp) {
     __shared__ PrSmem<T> sm;
     extern __shared__ uint4 dyn_smem[];
     uint32_t* hkeys = reinterpret_cast<uint32_t*>(dyn_smem);
@@ -135,7 +185,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
     const uint32_t count = ps.count;
     const uint32_t enc = ps.entry_encoding;
     constexpr uint32_t wshift = kWeighted ? 1 : 0;
-    PrEmitter<kMode, H> em{acc, hkeys, hacc, 0u, 0.f, false};
+    PrEmitter<kMode, H> em{acc, hkeys, hacc, &rp, 0u, 0.f, false};
     double dang = 0.0;
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
@@ -247,6 +297,13 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             const float v = hacc[i];
             if (k != kHotEmpty && v != 0.f) atomicAdd(acc + k, v);
         }
+    } else if (kMode == kRoute) {
+        for (uint32_t i = tid; i < n_hot; i += T) {
+            const float v = hacc[i];
+            if (v == 0.f) continue;
+            if ((uint64_t)i >= rp.lo && (uint64_t)i < rp.hi) atomicAdd(rp.acc_loc + (i - rp.lo), v);
+            else atomicAdd(rp.hot_out + i, v);
+        }
     } else {
         for (uint32_t i = tid; i < n_hot; i += T) {
             const float v = hacc[i];
@@ -269,7 +326,7 @@ __global__ void pr_init_kernel(float* x, float* acc, uint64_t n, float v0) {
 // x_v <- (1-d)/n + d*D/n + acc_v ; acc_v <- 0  for v in [lo, hi) (float4 vectorised where aligned).
 // Strategy-S ranks finish only their own WA range and zero the rest of acc.
 __global__ void pr_finish_kernel(float* x, float* acc, uint64_t n, uint64_t lo, uint64_t hi, double d,
-                                 const double* dang, double* dang_reset, int uniform) {
+                                 const double* dang, double* dang_reset, int uniform, int zero_outside) {
     const double D = *dang;
     const float base = (float)((1.0 - d) / (double)n + (uniform ? d * D / (double)n : 0.0));
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
@@ -292,14 +349,82 @@ __global__ void pr_finish_kernel(float* x, float* acc, uint64_t n, uint64_t lo, 
             acc[i] = 0.f;
         }
     }
-    if (lo > 0 || hi < n) {                             // zero acc outside my range (S)
+    if (zero_outside && (lo > 0 || hi < n)) {           // zero acc outside my range
         for (uint64_t i = t0; i < n; i += stride)
             if (i < lo || i >= hi) acc[i] = 0.f;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *dang_reset = 0.0;
 }
 
-enum { kBufX = 20, kBufAcc, kBufDang, kBufPrCtr };
+// ---- Strategy-S with routed updates: capacity count, apply -----------------
+
+template <bool W>
+struct RouteCountOp {   // per-owner count of this rank's remote cold edges (send capacities)
+    static constexpr bool kReadWeights = false;
+    static constexpr bool kWeighted = W;
+    const RouteParams* rp;
+    uint32_t n_hot;
+    uint32_t cnt[kMaxRanks];
+    __device__ const uint32_t* frontier() const { return nullptr; }
+    __device__ bool select(uint32_t) { return true; }
+    __device__ uint32_t payload(uint32_t, uint32_t) { return 0u; }
+    __device__ bool select_lp(uint32_t, uint32_t, uint32_t, uint32_t&) { return true; }
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*, const uint32_t*,
+                                          const bool* ok) {
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            const uint32_t v = dst[q];
+            if (ok[q] && v >= n_hot && !((uint64_t)v >= rp->lo && (uint64_t)v < rp->hi)) {
+                const int p = route_owner(*rp, v);
+#pragma unroll
+                for (int k = 0; k < kMaxRanks; ++k) cnt[k] += (k == p);
+            }
+        }
+    }
+    __device__ void end_page() {}
+};
+
+template <bool W>
+__global__ void __launch_bounds__(kThreads, 2)
+route_count_kernel(PageSet ps, const RouteParams rp, uint32_t n_hot, unsigned long long* out, uint32_t* work_ctr) {
+    __shared__ TileSmem sm;
+    RouteCountOp<W> op{&rp, n_hot, {0, 0, 0, 0, 0, 0, 0, 0}};
+    expand_pages(ps, op, sm, work_ctr);
+#pragma unroll
+    for (int k = 0; k < kMaxRanks; ++k) {
+        unsigned long long v = op.cnt[k];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
+        if ((threadIdx.x & 31) == 0 && v) atomicAdd(out + k, v);
+    }
+}
+
+// acc_loc[dst - lo] += val for the received (dst, val) pairs of every peer region
+__global__ void route_apply_kernel(const uint2* __restrict__ pairs, const uint32_t* __restrict__ off,
+                                   const uint32_t* __restrict__ cnt, int nranks, float* acc_loc, uint32_t lo) {
+    for (int p = 0; p < nranks; ++p) {
+        const uint32_t c = cnt[p], o = off[p];
+        for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < c; i += gridDim.x * blockDim.x) {
+            const uint2 e = pairs[o + i];
+            atomicAdd(acc_loc + (e.x - lo), __uint_as_float(e.y));
+        }
+    }
+}
+
+// acc[i] += hot[i], hot[i] = 0 over [a, b)
+__global__ void dense_add_kernel(float* acc, float* hot, uint64_t a, uint64_t b) {
+    for (uint64_t i = a + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < b;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        const float v = hot[i];
+        if (v != 0.f) {
+            acc[i] += v;
+            hot[i] = 0.f;
+        }
+    }
+}
+
+enum { kBufX = 20, kBufAcc, kBufDang, kBufPrCtr, kBufRouteSend, kBufRouteRecv, kBufRouteHot, kBufRouteHotIn,
+       kBufRouteCnt, kBufRouteList };
 
 }  // namespace gts
 
@@ -316,7 +441,14 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     if (dangling > GTS_DANGLING_DROP) return fail(GTS_EINVAL, "unknown dangling mode %u", dangling);
     const uint64_t n = g->n;
     const bool streamed = choose_streamed(c, g, rc, 8 * n);
-    const bool strat_s = rc.strategy == GTS_STRATEGY_S && c->world > 1;
+    // Strategy-S with routed updates: N > 1 ranks, or (tests, one GPU) GTS_VIRTUAL_RANKS=V
+    // virtual ranks run one after another on this GPU with an in-memory exchange
+    const char* vre = getenv("GTS_VIRTUAL_RANKS");
+    const int vranks = (rc.strategy == GTS_STRATEGY_S && c->world == 1 && vre) ? std::max(1, atoi(vre)) : 1;
+    const bool virt = vranks > 1;
+    const bool route = rc.strategy == GTS_STRATEGY_S && (c->world > 1 || virt);
+    const int R = virt ? vranks : c->world;
+    if (route && R > kMaxRanks) return fail(GTS_EUNSUPPORTED, "Strategy-S routing supports at most %d ranks", kMaxRanks);
     double upload_s = 0;
     GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
     const bool timing = rc.flags & GTS_RUN_TIMING;
@@ -330,10 +462,10 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     cudaStream_t s = c->stream;
     // scatter variant: degree-ordered graphs use the dense hot set held by one 1024-thread CTA per
     // SM (53,248 floats; GTS_PR_BIG=0 selects two 512-thread CTAs with 24,576 each, 3% slower
-    // on RMAT-27); natural-order graphs the hash table
+    // on RMAT-27); natural-order graphs the hash table; routed Strategy-S always the dense set
     const char* pbig = getenv("GTS_PR_BIG");
-    const bool big = g->ordered && (!pbig || atoi(pbig) > 0);
-    const int mode = g->ordered ? kDense : kHash;
+    const bool big = (g->ordered || route) && (!pbig || atoi(pbig) > 0);
+    const int mode = route ? kRoute : (g->ordered ? kDense : kHash);
     const void* kern;
     size_t dyn;
     int threads;
@@ -344,6 +476,12 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         dyn = pr_dyn_smem<kHash, 0>();
         threads = kThreads;
         n_hot = 0;
+    } else if (mode == kRoute) {
+        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kRoute, 1024, 1, kHotDenseBig>
+                           : (const void*)pr_scatter_kernel<false, kRoute, 1024, 1, kHotDenseBig>;
+        dyn = pr_dyn_smem<kRoute, kHotDenseBig>();
+        threads = 1024;
+        n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
     } else if (!big) {
         kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, kThreads, 2, kHotDense>
                            : (const void*)pr_scatter_kernel<false, kDense, kThreads, 2, kHotDense>;
@@ -365,7 +503,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     // device's persisting-L2 limit); GTS_L2_PERSIST=<MiB> overrides, 0 disables.
     bool persist = false;
     const char* pe = getenv("GTS_L2_PERSIST");
-    if (g->ordered && (!pe || atol(pe) > 0)) {
+    if (g->ordered && !route && (!pe || atol(pe) > 0)) {
         size_t want = (size_t)(pe ? atol(pe) : 96) << 20;
         want = std::min<size_t>(want, c->persist_max);
         want = std::min<size_t>(want, n * 4);
@@ -390,54 +528,240 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     GTS_CUDA(cudaMemsetAsync(dang, 0, 2 * sizeof(double), s));
     uint64_t launches = 1, main_launches = 0, nccl_bytes = 0;
     SweepStats ss;
-    const uint32_t* d_list = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
-    for (uint32_t it = 0; it < iters; ++it) {
-        double* D = dang + (it & 1);
-        std::pair<cudaEvent_t, cudaEvent_t> ev;
-        GTS_TRY(sweep_pages(c, g, rc, streamed, &c->dg.h_local_list, d_list, c->dg.n_local, nullptr,
-                            [&](const PageSet& ps, int cap) -> int {
-                                GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
-                                std::pair<cudaEvent_t, cudaEvent_t> e2;
-                                if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
-                                float dmp = (float)damping;
-                                const uint32_t* hk = c->dg.hot_keys;
-                                void* args[] = {(void*)&ps, (void*)&x, (void*)&acc, (void*)&hk, (void*)&dmp, (void*)&D,
-                                                (void*)&ctr, (void*)&n_hot};
-                                cudaLaunchConfig_t lc;
-                                std::memset(&lc, 0, sizeof(lc));
-                                int gsz = std::min(grid, cap);
-                                lc.gridDim = dim3(gsz);
-                                lc.blockDim = dim3(threads);
-                                lc.dynamicSmemBytes = dyn;
-                                lc.stream = s;
-                                GTS_CUDA(cudaLaunchKernelExC(&lc, kern, args));
-                                if (timing) cudaEventRecord(e2.second, s);
-                                GTS_CUDA(cudaGetLastError());
-                                ++main_launches;
-                                return GTS_OK;
-                            }, &ss));
-        if (c->world > 1) {
-            if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
-            GTS_NCCL(ncclGroupStart());
-            if (strat_s) {      // Strategy-S: rank r receives the sum of WA over its own range only
-                const std::vector<uint64_t>& vr = c->dg.h_vrange;
-                for (int r = 0; r < c->world; ++r)
-                    if (vr[r + 1] > vr[r])
-                        GTS_NCCL(ncclReduce(acc + vr[r], acc + vr[r], vr[r + 1] - vr[r], ncclFloat32, ncclSum, r,
-                                            c->comm, s));
-            } else {            // Strategy-P: every replica receives the full sum
+    float dmp = (float)damping;
+    const uint32_t* hk = c->dg.hot_keys;
+    auto scatter = [&](const PageSet& ps, int cap, double* D, const RouteParams& rp) -> int {
+        GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
+        std::pair<cudaEvent_t, cudaEvent_t> e2;
+        if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
+        void* args[] = {(void*)&ps, (void*)&x, (void*)&acc, (void*)&hk, (void*)&dmp, (void*)&D,
+                        (void*)&ctr, (void*)&n_hot, (void*)&rp};
+        cudaLaunchConfig_t lc;
+        std::memset(&lc, 0, sizeof(lc));
+        lc.gridDim = dim3(std::min(grid, cap));
+        lc.blockDim = dim3(threads);
+        lc.dynamicSmemBytes = dyn;
+        lc.stream = s;
+        GTS_CUDA(cudaLaunchKernelExC(&lc, kern, args));
+        if (timing) cudaEventRecord(e2.second, s);
+        GTS_CUDA(cudaGetLastError());
+        ++main_launches;
+        return GTS_OK;
+    };
+    RouteParams rp0;
+    std::memset(&rp0, 0, sizeof(rp0));
+    if (!route) {
+        const uint32_t* d_list = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
+        for (uint32_t it = 0; it < iters; ++it) {
+            double* D = dang + (it & 1);
+            std::pair<cudaEvent_t, cudaEvent_t> ev;
+            GTS_TRY(sweep_pages(c, g, rc, streamed, &c->dg.h_local_list, d_list, c->dg.n_local, nullptr,
+                                [&](const PageSet& ps, int cap) -> int { return scatter(ps, cap, D, rp0); }, &ss));
+            if (c->world > 1) {         // Strategy-P: every replica receives the full sum
+                if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
+                GTS_NCCL(ncclGroupStart());
                 GTS_NCCL(ncclAllReduce(acc, acc, n, ncclFloat32, ncclSum, c->comm, s));
+                GTS_NCCL(ncclAllReduce(D, D, 1, ncclFloat64, ncclSum, c->comm, s));
+                GTS_NCCL(ncclGroupEnd());
+                if (timing) cudaEventRecord(ev.second, s);
+                nccl_bytes += n * 4 + 8;
             }
-            GTS_NCCL(ncclAllReduce(D, D, 1, ncclFloat64, ncclSum, c->comm, s));
-            GTS_NCCL(ncclGroupEnd());
+            if (timing) { ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
+            pr_finish_kernel<<<eg, 256, 0, s>>>(x, acc, n, 0, n, damping, D, dang + ((it + 1) & 1),
+                                                 dangling == GTS_DANGLING_UNIFORM ? 1 : 0, 0);
             if (timing) cudaEventRecord(ev.second, s);
-            nccl_bytes += n * 4 + 8;
+            ++launches;
         }
-        if (timing) { ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
-        pr_finish_kernel<<<eg, 256, 0, s>>>(x, acc, n, strat_s ? c->dg.vlo : 0, strat_s ? c->dg.vhi : n, damping, D,
-                                             dang + ((it + 1) & 1), dangling == GTS_DANGLING_UNIFORM ? 1 : 0);
-        if (timing) cudaEventRecord(ev.second, s);
-        ++launches;
+    } else {
+        // ---- Strategy-S, routed: rank r owns WA [vr[r], vr[r+1]) and the pages whose sources lie in it
+        std::vector<int32_t> owner;
+        std::vector<uint64_t> vr;
+        partition(g, GTS_STRATEGY_S, R, owner, vr);
+        std::vector<std::vector<uint32_t>> plist(R);          // pages of each (virtual) rank
+        for (uint64_t j = 0; j < g->num_pages; ++j) plist[owner[j]].push_back((uint32_t)j);
+        const int me = virt ? -1 : c->rank;
+        const int r0 = virt ? 0 : me, r1 = virt ? R : me + 1;  // ranks simulated by this process
+        uint32_t* d_plist = nullptr;
+        GTS_TRY(c->buf(kBufRouteList, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&d_plist));
+        std::vector<uint32_t> pl_off(R + 1, 0);
+        for (int r = 0; r < R; ++r) pl_off[r + 1] = pl_off[r] + (uint32_t)plist[r].size();
+        {
+            std::vector<uint32_t> flat;
+            for (int r = 0; r < R; ++r) flat.insert(flat.end(), plist[r].begin(), plist[r].end());
+            GTS_CUDA(cudaMemcpyAsync(d_plist, flat.data(), flat.size() * 4, cudaMemcpyHostToDevice, s));
+            GTS_CUDA(cudaStreamSynchronize(s));
+        }
+        auto make_rp = [&](int r) {
+            RouteParams rp;
+            std::memset(&rp, 0, sizeof(rp));
+            for (int k = 0; k <= R; ++k) rp.vr[k] = vr[k];
+            rp.lo = vr[r];
+            rp.hi = vr[r + 1];
+            rp.nranks = R;
+            rp.acc_loc = acc + vr[r];
+            return rp;
+        };
+        auto pages_of = [&](int r, const uint32_t*& d, uint32_t& cnt) {
+            d = d_plist + pl_off[r];
+            cnt = pl_off[r + 1] - pl_off[r];
+        };
+        // send capacities: remote cold edges per (sender, owner), counted once per call
+        unsigned long long* d_cnt64;
+        // u64 capacities [kMaxRanks^2] | u32 flags[8] | send counts [kMaxRanks^2] | recv counts [kMaxRanks]
+        GTS_TRY(c->buf(kBufRouteCnt, sizeof(unsigned long long) * kMaxRanks * kMaxRanks +
+                                         (8 + kMaxRanks * kMaxRanks + kMaxRanks) * 4, (void**)&d_cnt64));
+        GTS_CUDA(cudaMemsetAsync(d_cnt64, 0, sizeof(unsigned long long) * kMaxRanks * kMaxRanks, s));
+        const void* kcount = g->weighted ? (const void*)route_count_kernel<true> : (const void*)route_count_kernel<false>;
+        int cgrid = 0;
+        GTS_TRY(sms_grid(c, kcount, kThreads, 0, &cgrid));
+        for (int r = r0; r < r1; ++r) {
+            RouteParams rp = make_rp(r);
+            const uint32_t* dl;
+            uint32_t cnt;
+            pages_of(r, dl, cnt);
+            std::vector<uint32_t> hl(plist[r]);
+            GTS_TRY(sweep_pages(c, g, rc, streamed, &hl, dl, cnt, nullptr, [&](const PageSet& ps, int cap) -> int {
+                GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
+                unsigned long long* out = d_cnt64 + (size_t)r * kMaxRanks;
+                void* args[] = {(void*)&ps, (void*)&rp, (void*)&n_hot, (void*)&out, (void*)&ctr};
+                GTS_CUDA(cudaLaunchKernel(kcount, dim3(std::min(cgrid, cap)), dim3(kThreads), args, 0, s));
+                ++launches;
+                return GTS_OK;
+            }, &ss));
+        }
+        std::vector<unsigned long long> cap64((size_t)kMaxRanks * kMaxRanks, 0);
+        GTS_CUDA(cudaMemcpyAsync(cap64.data(), d_cnt64, cap64.size() * 8, cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+        uint32_t* d_flags = reinterpret_cast<uint32_t*>(d_cnt64 + (size_t)kMaxRanks * kMaxRanks);  // [0] overflow
+        uint32_t* d_scnt = d_flags + 8;            // send counts [R] per simulated rank (R x R in virtual mode)
+        uint32_t* d_rcnt = d_flags + 8 + kMaxRanks * kMaxRanks;
+        if (!virt) {   // everyone learns what it will receive: all-gather the capacity rows
+            uint32_t* d_caprow;
+            uint32_t* d_capall;
+            GTS_TRY(c->buf(kBufRouteHotIn + 10, (size_t)(R + R * R) * 4, (void**)&d_caprow));
+            d_capall = d_caprow + R;
+            std::vector<uint32_t> row(R);
+            for (int p = 0; p < R; ++p) row[p] = (uint32_t)cap64[(size_t)me * kMaxRanks + p];
+            GTS_CUDA(cudaMemcpyAsync(d_caprow, row.data(), R * 4, cudaMemcpyHostToDevice, s));
+            GTS_NCCL(ncclAllGather(d_caprow, d_capall, R, ncclUint32, c->comm, s));
+            std::vector<uint32_t> all((size_t)R * R);
+            GTS_CUDA(cudaMemcpyAsync(all.data(), d_capall, all.size() * 4, cudaMemcpyDeviceToHost, s));
+            GTS_CUDA(cudaStreamSynchronize(s));
+            for (int a = 0; a < R; ++a)
+                for (int p = 0; p < R; ++p) cap64[(size_t)a * kMaxRanks + p] = all[(size_t)a * R + p];
+        }
+        // buffers: send regions of each simulated rank; receive regions (real ranks)
+        std::vector<uint32_t> soff((size_t)R * kMaxRanks, 0), roff(kMaxRanks, 0);
+        uint64_t stot = 0, rtot = 0;
+        for (int r = r0; r < r1; ++r)
+            for (int p = 0; p < R; ++p) {
+                soff[(size_t)r * kMaxRanks + p] = (uint32_t)stot;
+                stot += cap64[(size_t)r * kMaxRanks + p];
+            }
+        if (!virt)
+            for (int p = 0; p < R; ++p) {
+                roff[p] = (uint32_t)rtot;
+                rtot += cap64[(size_t)p * kMaxRanks + me];
+            }
+        if (stot >= (1ull << 32) || rtot >= (1ull << 32)) return fail(GTS_EOVERFLOW, "route buffers exceed 2^32 pairs");
+        uint2 *d_send, *d_recv = nullptr;
+        float *d_hot, *d_hot_in = nullptr;
+        GTS_TRY(c->buf(kBufRouteSend, std::max<uint64_t>(stot, 1) * 8, (void**)&d_send));
+        if (!virt) GTS_TRY(c->buf(kBufRouteRecv, std::max<uint64_t>(rtot, 1) * 8, (void**)&d_recv));
+        GTS_TRY(c->buf(kBufRouteHot, (size_t)(r1 - r0) * std::max<uint32_t>(n_hot, 1) * 4, (void**)&d_hot));
+        if (!virt) GTS_TRY(c->buf(kBufRouteHotIn, std::max<uint32_t>(n_hot, 1) * 4, (void**)&d_hot_in));
+        GTS_CUDA(cudaMemsetAsync(d_hot, 0, (size_t)(r1 - r0) * std::max<uint32_t>(n_hot, 1) * 4, s));
+        GTS_CUDA(cudaMemsetAsync(d_flags, 0, 4, s));
+        uint32_t* d_soff;                          // device copy of the send offsets (for apply)
+        GTS_TRY(c->buf(kBufRouteHotIn + 11, (size_t)(R * kMaxRanks + kMaxRanks) * 4, (void**)&d_soff));
+        GTS_CUDA(cudaMemcpyAsync(d_soff, soff.data(), soff.size() * 4, cudaMemcpyHostToDevice, s));
+        GTS_CUDA(cudaMemcpyAsync(d_soff + R * kMaxRanks, roff.data(), kMaxRanks * 4, cudaMemcpyHostToDevice, s));
+        std::vector<uint32_t> h_scnt(kMaxRanks * kMaxRanks), h_rcnt(kMaxRanks);
+        for (uint32_t it = 0; it < iters; ++it) {
+            double* D = dang + (it & 1);
+            std::pair<cudaEvent_t, cudaEvent_t> ev;
+            GTS_CUDA(cudaMemsetAsync(d_scnt, 0, (size_t)kMaxRanks * kMaxRanks * 4, s));
+            for (int r = r0; r < r1; ++r) {
+                RouteParams rp = make_rp(r);
+                rp.hot_out = d_hot + (size_t)(r - r0) * n_hot;
+                rp.send = d_send;
+                rp.send_cnt = d_scnt + (size_t)r * kMaxRanks;
+                rp.overflow = d_flags;
+                for (int p = 0; p < R; ++p) {
+                    rp.send_off[p] = soff[(size_t)r * kMaxRanks + p];
+                    rp.send_cap[p] = (uint32_t)cap64[(size_t)r * kMaxRanks + p];
+                }
+                const uint32_t* dl;
+                uint32_t cnt;
+                pages_of(r, dl, cnt);
+                std::vector<uint32_t> hl(plist[r]);
+                GTS_TRY(sweep_pages(c, g, rc, streamed, &hl, dl, cnt, nullptr,
+                                    [&](const PageSet& ps, int cap) -> int { return scatter(ps, cap, D, rp); }, &ss));
+            }
+            if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
+            if (virt) {                // in-memory exchange: every sender's pairs and hot partials land in acc
+                for (int r = 0; r < R; ++r) {
+                    route_apply_kernel<<<eg, 256, 0, s>>>(d_send, d_soff + (size_t)r * kMaxRanks,
+                                                          d_scnt + (size_t)r * kMaxRanks, R, acc, 0);
+                    dense_add_kernel<<<eg, 256, 0, s>>>(acc, d_hot + (size_t)r * n_hot, 0, n_hot);
+                    launches += 2;
+                }
+            } else {
+                const uint32_t* scnt_me = d_scnt + (size_t)me * kMaxRanks;
+                GTS_NCCL(ncclGroupStart());
+                for (int p = 0; p < R; ++p) {
+                    if (p == me) continue;
+                    GTS_NCCL(ncclSend(scnt_me + p, 1, ncclUint32, p, c->comm, s));
+                    GTS_NCCL(ncclRecv(d_rcnt + p, 1, ncclUint32, p, c->comm, s));
+                }
+                for (int q = 0; q < R; ++q) {  // hot partials: reduce each owner's slice of [0, n_hot)
+                    const uint64_t a = std::min<uint64_t>(vr[q], n_hot), b = std::min<uint64_t>(vr[q + 1], n_hot);
+                    if (b > a)
+                        GTS_NCCL(ncclReduce(d_hot + a, d_hot_in + a, b - a, ncclFloat32, ncclSum, q, c->comm, s));
+                }
+                GTS_NCCL(ncclGroupEnd());
+                GTS_CUDA(cudaMemcpyAsync(h_scnt.data(), scnt_me, R * 4, cudaMemcpyDeviceToHost, s));
+                GTS_CUDA(cudaMemcpyAsync(h_rcnt.data(), d_rcnt, R * 4, cudaMemcpyDeviceToHost, s));
+                GTS_CUDA(cudaStreamSynchronize(s));
+                GTS_NCCL(ncclGroupStart());
+                for (int p = 0; p < R; ++p) {
+                    if (p == me) continue;
+                    if (h_scnt[p])
+                        GTS_NCCL(ncclSend(d_send + soff[(size_t)me * kMaxRanks + p], (size_t)h_scnt[p] * 2, ncclUint32,
+                                          p, c->comm, s));
+                    if (h_rcnt[p])
+                        GTS_NCCL(ncclRecv(d_recv + roff[p], (size_t)h_rcnt[p] * 2, ncclUint32, p, c->comm, s));
+                    nccl_bytes += (uint64_t)h_scnt[p] * 8;
+                }
+                GTS_NCCL(ncclGroupEnd());
+                GTS_CUDA(cudaMemsetAsync(d_rcnt + me, 0, 4, s));
+                route_apply_kernel<<<eg, 256, 0, s>>>(d_recv, d_soff + R * kMaxRanks, d_rcnt, R, acc, 0);
+                const uint64_t a = std::min<uint64_t>(vr[me], n_hot), b = std::min<uint64_t>(vr[me + 1], n_hot);
+                if (b > a) dense_add_kernel<<<eg, 256, 0, s>>>(acc, d_hot_in, a, b);
+                GTS_CUDA(cudaMemsetAsync(d_hot, 0, std::max<uint32_t>(n_hot, 1) * 4, s));
+                GTS_NCCL(ncclAllReduce(D, D, 1, ncclFloat64, ncclSum, c->comm, s));
+                launches += 2;
+                nccl_bytes += n_hot * 4 + 8;
+            }
+            if (timing) { cudaEventRecord(ev.second, s); ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
+            const uint64_t flo = virt ? 0 : vr[me], fhi = virt ? n : vr[me + 1];
+            pr_finish_kernel<<<eg, 256, 0, s>>>(x, acc, n, flo, fhi, damping, D, dang + ((it + 1) & 1),
+                                                 dangling == GTS_DANGLING_UNIFORM ? 1 : 0, 0);
+            if (timing) cudaEventRecord(ev.second, s);
+            ++launches;
+        }
+        uint32_t ovf = 0;
+        GTS_CUDA(cudaMemcpyAsync(&ovf, d_flags, 4, cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+        if (ovf) return fail(GTS_ECUDA, "Strategy-S route buffer overflow (capacity count mismatch)");
+        if (!virt) {               // gather every rank's finished range so all ranks return the full vector
+            GTS_NCCL(ncclGroupStart());
+            for (int r = 0; r < R; ++r)
+                if (vr[r + 1] > vr[r])
+                    GTS_NCCL(ncclBroadcast(x + vr[r], x + vr[r], vr[r + 1] - vr[r], ncclFloat32, r, c->comm, s));
+            GTS_NCCL(ncclGroupEnd());
+            nccl_bytes += n * 4;
+        }
     }
     launches += main_launches;
     if (persist) {
@@ -447,15 +771,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         GTS_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &at));
         const char* rs = getenv("GTS_L2_RESET");
         if (!rs || atoi(rs) != 0) GTS_CUDA(cudaCtxResetPersistingL2Cache());   // release the lines for other work
-    }
-    if (strat_s) {              // gather every rank's finished range so all ranks return the full vector
-        GTS_NCCL(ncclGroupStart());
-        const std::vector<uint64_t>& vr = c->dg.h_vrange;
-        for (int r = 0; r < c->world; ++r)
-            if (vr[r + 1] > vr[r])
-                GTS_NCCL(ncclBroadcast(x + vr[r], x + vr[r], vr[r + 1] - vr[r], ncclFloat32, r, c->comm, s));
-        GTS_NCCL(ncclGroupEnd());
-        nccl_bytes += n * 4;
     }
     GTS_CUDA(cudaGetLastError());
     GTS_TRY(deliver(c, g, reinterpret_cast<const uint32_t*>(x), rank_out, rc.out_location, false));

@@ -321,3 +321,24 @@ def test_streamed_page_cache(G, ctx, name, cache_pages):
     grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb)
     got, _ = G.gts_sssp(ctx, grw, src, **kw)
     assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, src))
+
+
+# ------------------------------------- Strategy-S with routed updates (virtual ranks) ---
+
+@pytest.mark.parametrize("name", ["fig1", "rmat16_4k", "rmat20", "twitter20", "instar", "outstar"])
+@pytest.mark.parametrize("vranks", [2, 3, 8])
+@pytest.mark.parametrize("order", [False, True])
+def test_pagerank_strategy_s_routed(G, ctx, name, vranks, order, monkeypatch):
+    """Strategy-S with range-partitioned WA and routed updates: V
+    virtual ranks run one after another on this GPU (GTS_VIRTUAL_RANKS), each
+    scattering only its own pages into its own WA range and packing every other
+    update into per-owner (dst, value) buffers; the in-memory exchange then
+    applies them.  Exercises owner lookup, capacity counting, warp-aggregated
+    packing, hot-partial routing and apply; only the NCCL send/recv is skipped."""
+    monkeypatch.setenv("GTS_VIRTUAL_RANKS", str(vranks))
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
+    want = oracle.pagerank(g.row_ptr, g.col, 10, 0.85)
+    for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3)):
+        got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, strategy=G.GTS_STRATEGY_S, **kw)
+        _pr_check(got, want, g, (name, vranks, order, kw))
