@@ -78,16 +78,18 @@ struct SsspOp {
     uint32_t* next;
     unsigned long long nedges;
     bool ovf;
+    uint32_t T;                // near-far threshold: only pending vertices with dist <= T are expanded
     __device__ const uint32_t* frontier() const { return cur; }
-    __device__ bool select(uint32_t v) { return test_bit(cur, v); }
+    __device__ bool select(uint32_t v) { return test_bit(cur, v) && __ldcg(dist + v) <= T; }
     __device__ uint32_t payload(uint32_t v, uint32_t deg) {
         nedges += deg;
         return *((volatile uint32_t*)dist + v);
     }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t len, uint32_t& pl) {
         if (!test_bit(cur, vid)) return false;
-        if (threadIdx.x == 0) nedges += len;
         pl = *((volatile uint32_t*)dist + vid);
+        if (pl > T) return false;
+        if (threadIdx.x == 0) nedges += len;
         return true;
     }
     // relax (u,v,w): candidates >= 2^32-1 are dropped and flagged (checked
@@ -152,9 +154,9 @@ bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visite
 
 __global__ void __launch_bounds__(kThreads, 2)
 sssp_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* dist, uint32_t* next,
-                   uint32_t* work_ctr, unsigned long long* edges_out, uint32_t* ovf_flag) {
+                   uint32_t* work_ctr, unsigned long long* edges_out, uint32_t* ovf_flag, uint32_t T) {
     __shared__ TileSmem sm;
-    SsspOp<true> op{cur, dist, next, 0ull, false};
+    SsspOp<true> op{cur, dist, next, 0ull, false, T};
     expand_pages(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
     if (__syncthreads_or(op.ovf) && threadIdx.x == 0) *ovf_flag = 1u;
@@ -195,6 +197,43 @@ __global__ void frontier_finish_kernel(const uint32_t* __restrict__ gathered, in
     block_add_u64(c, count);
 }
 
+// SSSP near-far pending set: new pending = improved this round (next, merged over
+// ranks) + pending vertices that were not expanded (dist > T).  Counts the
+// pending vertices, those already within T, and the minimum pending distance.
+__global__ void sssp_finish_kernel(const uint32_t* __restrict__ gathered, int world, uint64_t words,
+                                   const uint32_t* __restrict__ cur, uint32_t* next, const uint32_t* __restrict__ dist,
+                                   uint32_t T, unsigned long long* count, unsigned long long* near,
+                                   unsigned int* minpend) {
+    unsigned long long c = 0, nr = 0;
+    uint32_t mn = 0xFFFFFFFFu;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
+        uint32_t bits = gathered[w];
+        for (int r = 1; r < world; ++r) bits |= gathered[(uint64_t)r * words + w];
+        uint32_t keep = cur[w] & ~bits;
+        while (keep) {
+            const int b = __ffs(keep) - 1;
+            if (dist[w * 32 + b] > T) bits |= 1u << b;
+            keep &= keep - 1;
+        }
+        next[w] = bits;
+        c += __popc(bits);
+        uint32_t t = bits;
+        while (t) {
+            const int b = __ffs(t) - 1;
+            const uint32_t dv = dist[w * 32 + b];
+            mn = min(mn, dv);
+            nr += dv <= T;
+            t &= t - 1;
+        }
+    }
+    block_add_u64(c, count);
+    block_add_u64(nr, near);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mn = min(mn, __shfl_down_sync(0xFFFFFFFFu, mn, o));
+    if ((threadIdx.x & 31) == 0 && mn != 0xFFFFFFFFu) atomicMin(minpend, mn);
+}
+
 // Next page set (nextPIDSet, Alg 1 lines 29-30): the pages among
 // `pages` (this rank's) whose VID range [START_VID, START_VID + nslots) has a
 // bit set in `bits`.  One warp per page.
@@ -233,6 +272,9 @@ struct Counters {               // device scratch, slot kCtr
     unsigned long long edges;
     uint32_t flag;
     uint32_t flag2;
+    unsigned long long near;       // SSSP: pending vertices within the threshold
+    unsigned int minpend;          // SSSP: minimum pending distance
+    unsigned int pad;
 };
 
 enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather };
@@ -319,6 +361,13 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     SweepStats ss;
     std::vector<uint32_t> h_list = l0;             // streamed mode: this level's pages on the host (ascending)
     const bool cached = streamed && rc.cache_mib > 0;
+    // SSSP near-far bucketing: expand only pending vertices with dist <= T; T
+    // advances by delta past the nearest pending distance when no pending vertex
+    // is within it (GTS_SSSP_DELTA, default 64; a label-correcting method, so any
+    // delta gives the exact distances)
+    const char* de = getenv("GTS_SSSP_DELTA");
+    const uint64_t delta = de ? std::max<long>(1, atol(de)) : 64;
+    uint32_t T = algo == kSSSP ? (uint32_t)std::min<uint64_t>(delta, 0xFFFFFFFEull) : 0xFFFFFFFEu;
     for (uint32_t L = 0;; ++L) {
         auto launch = [&](const PageSet& ps, int cap) -> int {
                                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
@@ -332,7 +381,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                         ps, cur, visited, next, &ctr->work, &ctr->edges);
                                 else
                                     sssp_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(
-                                        ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag);
+                                        ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T);
                                 if (timing) cudaEventRecord(ev.second, s);
                                 GTS_CUDA(cudaGetLastError());
                                 ++main_launches;
@@ -353,9 +402,15 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         if (timing) { cudaEventRecord(ev.second, s); ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
         GTS_CUDA(cudaMemsetAsync(&ctr->count, 0, 8, s));
         GTS_CUDA(cudaMemsetAsync(&ctr->list_count, 0, 4, s));
-        frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, next,
-                                                        visited, algo == kBFS ? value : nullptr, L + 1,
-                                                        &ctr->count);
+        if (algo == kBFS) {
+            frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, next,
+                                                            visited, value, L + 1, &ctr->count);
+        } else {
+            GTS_CUDA(cudaMemsetAsync(&ctr->near, 0, 8, s));
+            GTS_CUDA(cudaMemsetAsync(&ctr->minpend, 0xFF, 4, s));
+            sssp_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, cur, next,
+                                                        value, T, &ctr->count, &ctr->near, &ctr->minpend);
+        }
         frontier_pages_kernel<<<fin_grid, 256, 0, s>>>(next, c->dg.rvt_start, c->dg.nslots,
                                                        c->dg.all_local ? nullptr : c->dg.local_list,
                                                        c->dg.all_local ? (uint32_t)g->num_pages : c->dg.n_local,
@@ -367,6 +422,10 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         GTS_CUDA(cudaStreamSynchronize(s));
         ++levels;
         if (h.count == 0) break;
+        if (algo == kSSSP && h.near == 0) {      // nothing pending within T: open the next bucket
+            const uint64_t nt = (uint64_t)h.minpend + delta;
+            T = (uint32_t)std::min<uint64_t>(nt, 0xFFFFFFFEull);
+        }
         pages_processed += h.list_count;
         if (streamed) {                          // the host drives the copies: fetch and sort the page set
             h_list.resize(h.list_count);

@@ -342,3 +342,16 @@ def test_pagerank_strategy_s_routed(G, ctx, name, vranks, order, monkeypatch):
     for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3)):
         got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, strategy=G.GTS_STRATEGY_S, **kw)
         _pr_check(got, want, g, (name, vranks, order, kw))
+
+
+@pytest.mark.parametrize("delta", ["1", "16", "256", "4294967294"])
+@pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "path", "bintree"])
+def test_sssp_near_far_deltas(G, ctx, name, delta, monkeypatch):
+    """Near-far SSSP bucket widths, from 1 (Dijkstra-like) to unbounded (plain
+    frontier Bellman-Ford): distances are exact for every width."""
+    monkeypatch.setenv("GTS_SSSP_DELTA", delta)
+    g, pb = graph(name)
+    w = inputs.edge_weights(g)
+    gr = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb)
+    got, _ = G.gts_sssp(ctx, gr, 0)
+    assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, 0))
