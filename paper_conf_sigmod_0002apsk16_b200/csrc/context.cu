@@ -464,6 +464,7 @@ extern "C" void gts_context_free(gts_context* c) {
             cudaEventDestroy(c->ring_ready[i]);
             cudaEventDestroy(c->ring_free[i]);
         }
+    if (c->persist_limit) cudaCtxResetPersistingL2Cache();
     if (c->comm) ncclCommDestroy(c->comm);
     cudaFreeHost(c->h_small);
     if (c->h_stage) cudaFreeHost(c->h_stage);

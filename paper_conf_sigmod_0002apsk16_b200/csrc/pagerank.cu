@@ -769,8 +769,11 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         std::memset(&at, 0, sizeof(at));
         at.accessPolicyWindow.num_bytes = 0;
         GTS_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &at));
+        // The lines marked persisting stay so until the next PageRank call reuses
+        // them or the context is freed: an explicit cudaCtxResetPersistingL2Cache
+        // here measured +20 ms on the following call (GTS_L2_RESET=1 forces it).
         const char* rs = getenv("GTS_L2_RESET");
-        if (!rs || atoi(rs) != 0) GTS_CUDA(cudaCtxResetPersistingL2Cache());   // release the lines for other work
+        if (rs && atoi(rs) != 0) GTS_CUDA(cudaCtxResetPersistingL2Cache());
     }
     GTS_CUDA(cudaGetLastError());
     GTS_TRY(deliver(c, g, reinterpret_cast<const uint32_t*>(x), rank_out, rc.out_location, false));
