@@ -1,7 +1,7 @@
 """The GTS oracle -- TEST INFRASTRUCTURE ONLY.
 
 Plain single-threaded CPU implementations (oracle/oracle.c, fp64 for
-PageRank) of BFS, PageRank, SSSP and WCC over CSR, plus an independent reader
+PageRank and BC) of BFS, PageRank, SSSP, WCC and betweenness centrality over CSR, plus an independent reader
 of the slotted-page format.  Only tests/, __graft_entry__.smoke() and
 bench.py (cpu_baseline leg and --impl reference) may import this package.
 The product path (paper_conf_sigmod_0002apsk16_b200) never imports it and
@@ -48,6 +48,8 @@ def lib():
         L.oracle_sssp.restype = ctypes.c_int
         L.oracle_wcc.argtypes = [u64, vp, vp, vp]
         L.oracle_wcc.restype = ctypes.c_int
+        L.oracle_bc.argtypes = [u64, vp, vp, vp, u64, vp]
+        L.oracle_bc.restype = ctypes.c_int
         L.oracle_decode_pages.argtypes = [vp, u64, u64, ctypes.c_int, ctypes.c_int, u64, vp, vp, vp, u64]
         L.oracle_decode_pages.restype = ctypes.c_int64
         _lib = L
@@ -105,6 +107,17 @@ def wcc(row_ptr, col):
     rc = lib().oracle_wcc(n, _ptr(row_ptr), _ptr(col), _ptr(out))
     if rc:
         raise ValueError(f"oracle_wcc rc={rc}")
+    return out
+
+
+def bc(row_ptr, col, sources):
+    """Brandes betweenness (fp64, unnormalised) accumulated over `sources`."""
+    row_ptr, col, n = _csr(row_ptr, col)
+    src = np.ascontiguousarray(sources, dtype=np.uint32)
+    out = np.empty(n, dtype=np.float64)
+    rc = lib().oracle_bc(n, _ptr(row_ptr), _ptr(col), _ptr(src), len(src), _ptr(out))
+    if rc:
+        raise ValueError(f"oracle_bc rc={rc}")
     return out
 
 

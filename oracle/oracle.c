@@ -266,3 +266,49 @@ int64_t oracle_decode_pages(const uint8_t* pages, uint64_t num_pages, uint64_t p
     free(start_vid); free(deg);
     return m;
 }
+
+/* ------------------------------------------------------------------- BC ---
+ * Betweenness centrality restricted to a set of sources (the paper runs BC as
+ * a BFS-like algorithm on GTS, Fig 13c; no kernel is given).  Textbook
+ * Brandes (2001) for unweighted directed multigraphs over out-edges, fp64:
+ *   for each source s: BFS levels d and path counts sigma (sigma[s] = 1,
+ *   sigma[w] += sigma[v] over every edge v->w with d[w] = d[v] + 1, parallel
+ *   edges counted with multiplicity); then in non-increasing d order
+ *   delta[v] = sum over edges v->w with d[w] = d[v] + 1 of
+ *              sigma[v] / sigma[w] * (1 + delta[w]);
+ *   bc[v] += delta[v] for v != s.
+ * bc_out[n] is accumulated over the k sources (not normalised). */
+int oracle_bc(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, const uint32_t* sources, uint64_t k,
+              double* bc_out) {
+    uint32_t* d = (uint32_t*)malloc(n * sizeof(uint32_t));
+    double* sigma = (double*)malloc(n * sizeof(double));
+    double* delta = (double*)malloc(n * sizeof(double));
+    uint32_t* order = (uint32_t*)malloc((n ? n : 1) * sizeof(uint32_t));
+    if (!d || !sigma || !delta || !order) return -2;
+    for (uint64_t v = 0; v < n; ++v) bc_out[v] = 0.0;
+    for (uint64_t si = 0; si < k; ++si) {
+        uint32_t s = sources[si];
+        if (s >= n) { free(d); free(sigma); free(delta); free(order); return -1; }
+        for (uint64_t v = 0; v < n; ++v) { d[v] = UNREACHED; sigma[v] = 0.0; delta[v] = 0.0; }
+        uint64_t head = 0, tail = 0;
+        d[s] = 0; sigma[s] = 1.0; order[tail++] = s;
+        while (head < tail) {                       /* BFS: order = vertices by non-decreasing d */
+            uint32_t v = order[head++];
+            for (uint64_t e = row_ptr[v]; e < row_ptr[v + 1]; ++e) {
+                uint32_t w = col[e];
+                if (d[w] == UNREACHED) { d[w] = d[v] + 1; order[tail++] = w; }
+                if (d[w] == d[v] + 1) sigma[w] += sigma[v];
+            }
+        }
+        for (uint64_t i = tail; i-- > 0;) {         /* dependencies in non-increasing d */
+            uint32_t v = order[i];
+            for (uint64_t e = row_ptr[v]; e < row_ptr[v + 1]; ++e) {
+                uint32_t w = col[e];
+                if (d[w] == d[v] + 1) delta[v] += sigma[v] / sigma[w] * (1.0 + delta[w]);
+            }
+            if (v != s) bc_out[v] += delta[v];
+        }
+    }
+    free(d); free(sigma); free(delta); free(order);
+    return 0;
+}
