@@ -221,6 +221,15 @@ int gts_sssp(gts_context* ctx, const gts_graph* g, uint64_t src, const gts_run_c
 int gts_wcc(gts_context* ctx, const gts_graph* g, const gts_run_config* cfg, uint32_t* label_out,
             gts_run_stats* stats);
 
+/* Betweenness centrality (BC is run on GTS in the
+ * paper, Fig 13c, no kernel given): Brandes' dependency accumulation
+ * from each of the k sources over out-edges, unweighted, path counts with
+ * edge multiplicity, summed over the sources: bc_out[n] fp64 (not
+ * normalised).  Pages may be resident or streamed.  One GPU (EUNSUPPORTED for
+ * world_size > 1).  EINVAL if a source >= n. */
+int gts_bc(gts_context* ctx, const gts_graph* g, const uint64_t* sources, uint32_t num_sources,
+           const gts_run_config* cfg, double* bc_out, gts_run_stats* stats);
+
 /* ---------------------------------------------------- multi-GPU helpers --- */
 
 /* Page -> rank assignment used by a strategy (pure host logic, exposed for

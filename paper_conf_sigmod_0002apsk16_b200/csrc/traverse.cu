@@ -495,6 +495,313 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     return GTS_OK;
 }
 
+// ------------------------------------------------------------------- BC ---
+// Betweenness centrality (Brandes) over the same page engine; the paper runs
+// BC as a BFS-like algorithm on GTS (Fig 13c) without giving kernels.
+// Per source: level by level, pass A is the BFS expansion (bfs_expand_kernel)
+// and pass B adds sigma[u] into sigma[w] for every edge u->w from the level's
+// frontier into the vertices discovered by pass A; then, over the stored level
+// bitmaps in reverse, delta[v] += sigma[v]/sigma[w] * (1 + delta[w]) for every
+// edge v->w with LV[w] = LV[v] + 1, each thread folding runs of the same source
+// v before one fp64 atomic; finally bc[v] += delta[v] (v != source).
+
+template <bool W>
+struct BcSigmaOp {
+    static constexpr bool kReadWeights = false;
+    static constexpr bool kWeighted = W;
+    const uint32_t* cur;
+    const uint32_t* next;
+    double* sigma;
+    __device__ const uint32_t* frontier() const { return cur; }
+    __device__ bool select(uint32_t v) { return test_bit(cur, v); }
+    __device__ uint32_t payload(uint32_t, uint32_t) { return 0u; }
+    __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t&) { return test_bit(cur, vid); }
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*, const uint32_t* src,
+                                          const bool* ok) {
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q)
+            if (ok[q] && test_bit(next, dst[q])) atomicAdd(sigma + dst[q], __ldcg(sigma + src[q]));
+    }
+    __device__ void end_page() {}
+};
+
+template <bool W>
+struct BcDeltaOp {
+    static constexpr bool kReadWeights = false;
+    static constexpr bool kWeighted = W;
+    const uint32_t* lvbits;    // vertices at level L
+    const uint32_t* lv;
+    uint32_t L;
+    const double* sigma;
+    double* delta;
+    uint32_t run_src;
+    double run_sum;
+    bool has;
+    __device__ const uint32_t* frontier() const { return lvbits; }
+    __device__ bool select(uint32_t v) { return test_bit(lvbits, v); }
+    __device__ uint32_t payload(uint32_t, uint32_t) { return 0u; }
+    __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t&) { return test_bit(lvbits, vid); }
+    __device__ __forceinline__ void flush() {
+        if (has && run_sum != 0.0) atomicAdd(delta + run_src, run_sum);
+        has = false;
+        run_sum = 0.0;
+    }
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*, const uint32_t* src,
+                                          const bool* ok) {
+        uint32_t l[kEdgesPerThread];
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) l[q] = ok[q] ? __ldg(lv + dst[q]) : 0u;
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            if (!ok[q] || l[q] != L + 1) continue;
+            const double cw = __ldg(sigma + src[q]) / __ldg(sigma + dst[q]) * (1.0 + __ldcg(delta + dst[q]));
+            if (!has || run_src != src[q]) {
+                flush();
+                run_src = src[q];
+                has = true;
+            }
+            run_sum += cw;
+        }
+    }
+    __device__ void end_page() { flush(); }
+};
+
+template <bool W>
+__global__ void __launch_bounds__(kThreads, 2)
+bc_sigma_kernel(PageSet ps, const uint32_t* __restrict__ cur, const uint32_t* __restrict__ next, double* sigma,
+                uint32_t* work_ctr) {
+    __shared__ TileSmem sm;
+    BcSigmaOp<W> op{cur, next, sigma};
+    expand_pages(ps, op, sm, work_ctr);
+}
+
+template <bool W>
+__global__ void __launch_bounds__(kThreads, 2)
+bc_delta_kernel(PageSet ps, const uint32_t* __restrict__ lvbits, const uint32_t* __restrict__ lv, uint32_t L,
+                const double* __restrict__ sigma, double* delta, uint32_t* work_ctr) {
+    __shared__ TileSmem sm;
+    BcDeltaOp<W> op{lvbits, lv, L, sigma, delta, 0u, 0.0, false};
+    expand_pages(ps, op, sm, work_ctr);
+    op.flush();
+}
+
+__global__ void bc_source_kernel(uint32_t* lv, uint32_t* visited, uint32_t* cur, double* sigma, uint64_t s) {
+    lv[s] = 0;
+    visited[s >> 5] |= 1u << (s & 31);
+    cur[s >> 5] |= 1u << (s & 31);
+    sigma[s] = 1.0;
+}
+
+__global__ void bc_accumulate_kernel(double* bc, const double* __restrict__ delta, uint64_t n, uint64_t s) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+        if (v != s) bc[v] += delta[v];
+}
+
+__global__ void gather_f64_kernel(double* out, const double* __restrict__ vals, const uint32_t* __restrict__ idx,
+                                  uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) out[v] = vals[idx[v]];
+}
+
+enum { kBufBcSigma = 40, kBufBcDelta, kBufBcOut, kBufBcList2, kBufBcTmp };
+
+static int betweenness(gts_context* c, const gts_graph* g, const uint64_t* sources, uint32_t k,
+                       const gts_run_config* cfg, double* out, gts_run_stats* st) {
+    clear_error();
+    const double t_start = now_s();
+    gts_run_config rc;
+    GTS_TRY(validate_common(c, g, cfg, &rc));
+    if (!out || (k > 0 && !sources)) return fail(GTS_EINVAL, "NULL argument");
+    for (uint32_t i = 0; i < k; ++i)
+        if (sources[i] >= g->n) return fail(GTS_EINVAL, "source %llu >= n", (unsigned long long)sources[i]);
+    if (c->world > 1) return fail(GTS_EUNSUPPORTED, "gts_bc runs on one GPU in this version");
+    const uint64_t n = g->n, words = (n + 31) / 32;
+    const bool streamed = choose_streamed(c, g, rc, 28 * n + 16 * words);
+    double upload_s = 0;
+    GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
+    const bool timing = rc.flags & GTS_RUN_TIMING;
+    uint32_t *lv, *visited, *cur, *next, *list, *list2;
+    double *sigma, *delta, *bc;
+    Counters* ctr;
+    GTS_TRY(c->buf(kBufValue, n * 4, (void**)&lv));
+    GTS_TRY(c->buf(kBufVisited, words * 4, (void**)&visited));
+    GTS_TRY(c->buf(kBufCur, words * 4, (void**)&cur));
+    GTS_TRY(c->buf(kBufNext, words * 4, (void**)&next));
+    GTS_TRY(c->buf(kBufList, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&list));
+    GTS_TRY(c->buf(kBufBcList2, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&list2));
+    GTS_TRY(c->buf(kBufCtr, sizeof(Counters), (void**)&ctr));
+    GTS_TRY(c->buf(kBufBcSigma, n * 8, (void**)&sigma));
+    GTS_TRY(c->buf(kBufBcDelta, n * 8, (void**)&delta));
+    GTS_TRY(c->buf(kBufBcOut, n * 8, (void**)&bc));
+    cudaStream_t s = c->stream;
+    const int eg = c->num_sms * 4;
+    GTS_CUDA(cudaMemsetAsync(bc, 0, n * 8, s));
+    const bool wgt = g->weighted;
+    const void* kA = wgt ? (const void*)bfs_expand_kernel<true> : (const void*)bfs_expand_kernel<false>;
+    int grid = 0;
+    GTS_TRY(sms_grid(c, kA, kThreads, 0, &grid));
+    uint64_t launches = 1, main_launches = 0, pages_processed = 0, edges = 0;
+    uint32_t levels_total = 0;
+    SweepStats ss;
+    uint32_t* lv_store = nullptr;             // per-level frontier bitmaps [lv_cap][words]
+    uint32_t lv_cap = 0;
+    struct Free { uint32_t*& p; ~Free() { cudaFree(p); } } free_store{lv_store};
+    Counters h;
+    for (uint32_t si = 0; si < k; ++si) {
+        const uint64_t src = map_src(g, sources[si]);
+        GTS_CUDA(cudaMemsetAsync(lv, 0xFF, n * 4, s));
+        GTS_CUDA(cudaMemsetAsync(visited, 0, words * 4, s));
+        GTS_CUDA(cudaMemsetAsync(cur, 0, words * 4, s));
+        GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
+        GTS_CUDA(cudaMemsetAsync(sigma, 0, n * 8, s));
+        GTS_CUDA(cudaMemsetAsync(delta, 0, n * 8, s));
+        GTS_CUDA(cudaMemsetAsync(ctr, 0, sizeof(Counters), s));
+        bc_source_kernel<<<1, 1, 0, s>>>(lv, visited, cur, sigma, src);
+        std::vector<uint32_t> l0 = pages_of_vertex(g, c->dg, c->rank, src);
+        uint32_t* hs = (uint32_t*)c->h_small;
+        hs[0] = (uint32_t)l0.size();
+        if (!l0.empty()) GTS_CUDA(cudaMemcpyAsync(list, l0.data(), l0.size() * 4, cudaMemcpyHostToDevice, s));
+        GTS_CUDA(cudaMemcpyAsync(&ctr->list_count, hs, 4, cudaMemcpyHostToDevice, s));
+        std::vector<uint32_t> h_list = l0;
+        uint32_t cur_count = (uint32_t)l0.size();
+        std::vector<std::vector<uint32_t>> lvl_pages;  // streamed: page sets per level
+        uint32_t L = 0;
+        for (;; ++L) {
+            // keep this level's frontier bitmap for the backward pass (the store grows
+            // by doubling; earlier levels are copied over)
+            if (L >= lv_cap) {
+                const uint32_t ncap = std::max<uint32_t>(16, 2 * lv_cap);
+                uint32_t* nb = nullptr;
+                cudaError_t e = cudaMalloc(&nb, (size_t)ncap * words * 4);
+                if (e != cudaSuccess) {
+                    cudaGetLastError();
+                    return fail(GTS_ENOMEM, "bc level bitmaps: cudaMalloc failed");
+                }
+                if (lv_store) {
+                    GTS_CUDA(cudaMemcpyAsync(nb, lv_store, (size_t)lv_cap * words * 4, cudaMemcpyDeviceToDevice, s));
+                    GTS_CUDA(cudaStreamSynchronize(s));
+                    cudaFree(lv_store);
+                }
+                lv_store = nb;
+                lv_cap = ncap;
+            }
+            GTS_CUDA(cudaMemcpyAsync(lv_store + (size_t)L * words, cur, words * 4, cudaMemcpyDeviceToDevice, s));
+            if (streamed) lvl_pages.push_back(h_list);
+            // pass A: discover level L+1 (BFS expansion)
+            auto launchA = [&](const PageSet& ps, int cap) -> int {
+                GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+                std::pair<cudaEvent_t, cudaEvent_t> ev;
+                if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges);
+                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges);
+                if (timing) cudaEventRecord(ev.second, s);
+                GTS_CUDA(cudaGetLastError());
+                ++main_launches;
+                return GTS_OK;
+            };
+            GTS_TRY(sweep_pages(c, g, rc, streamed, &h_list, list, cur_count, &ctr->list_count, launchA, &ss));
+            GTS_CUDA(cudaMemsetAsync(&ctr->count, 0, 8, s));
+            frontier_finish_kernel<<<eg, 256, 0, s>>>(next, 1, words, next, visited, lv, L + 1, &ctr->count);
+            // pass B: sigma of the newly discovered vertices
+            auto launchB = [&](const PageSet& ps, int cap) -> int {
+                GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+                std::pair<cudaEvent_t, cudaEvent_t> ev;
+                if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+                if (wgt) bc_sigma_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, next, sigma, &ctr->work);
+                else bc_sigma_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, next, sigma, &ctr->work);
+                if (timing) cudaEventRecord(ev.second, s);
+                GTS_CUDA(cudaGetLastError());
+                ++main_launches;
+                return GTS_OK;
+            };
+            GTS_TRY(sweep_pages(c, g, rc, streamed, &h_list, list, cur_count, &ctr->list_count, launchB, &ss));
+            // next page set
+            GTS_CUDA(cudaMemsetAsync(&ctr->list_count, 0, 4, s));
+            frontier_pages_kernel<<<eg, 256, 0, s>>>(next, c->dg.rvt_start, c->dg.nslots, nullptr,
+                                                     (uint32_t)g->num_pages, list, &ctr->list_count);
+            launches += 3;
+            GTS_CUDA(cudaMemcpyAsync(&h, ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
+            GTS_CUDA(cudaStreamSynchronize(s));
+            pages_processed += 2ull * cur_count;
+            if (h.count == 0) break;
+            cur_count = h.list_count;
+            if (streamed) {
+                h_list.resize(h.list_count);
+                GTS_CUDA(cudaMemcpyAsync(h_list.data(), list, h.list_count * 4ull, cudaMemcpyDeviceToHost, s));
+                GTS_CUDA(cudaStreamSynchronize(s));
+                std::sort(h_list.begin(), h_list.end());
+                GTS_CUDA(cudaMemcpyAsync(list, h_list.data(), h.list_count * 4ull, cudaMemcpyHostToDevice, s));
+            }
+            std::swap(cur, next);
+            GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
+        }
+        edges += h.edges;
+        levels_total += L + 1;
+        // backward: levels L-1 .. 0 (level L has no successors)
+        for (int64_t q = (int64_t)L - 1; q >= 0; --q) {
+            uint32_t* bits = lv_store + (size_t)q * words;
+            GTS_CUDA(cudaMemsetAsync(&ctr->list_count, 0, 4, s));
+            frontier_pages_kernel<<<eg, 256, 0, s>>>(bits, c->dg.rvt_start, c->dg.nslots, nullptr,
+                                                     (uint32_t)g->num_pages, list2, &ctr->list_count);
+            std::vector<uint32_t> hl;
+            uint32_t cnt = 0;
+            if (streamed) {
+                hl = lvl_pages[q];
+                cnt = (uint32_t)hl.size();
+                GTS_CUDA(cudaMemcpyAsync(list2, hl.data(), hl.size() * 4, cudaMemcpyHostToDevice, s));
+            }
+            const uint32_t Lq = (uint32_t)q;
+            auto launchD = [&](const PageSet& ps, int cap) -> int {
+                GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
+                std::pair<cudaEvent_t, cudaEvent_t> ev;
+                if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+                if (wgt) bc_delta_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, bits, lv, Lq, sigma, delta, &ctr->work);
+                else bc_delta_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, bits, lv, Lq, sigma, delta, &ctr->work);
+                if (timing) cudaEventRecord(ev.second, s);
+                GTS_CUDA(cudaGetLastError());
+                ++main_launches;
+                return GTS_OK;
+            };
+            GTS_TRY(sweep_pages(c, g, rc, streamed, &hl, list2, cnt, &ctr->list_count, launchD, &ss));
+            ++launches;
+        }
+        bc_accumulate_kernel<<<eg, 256, 0, s>>>(bc, delta, n, src);
+        ++launches;
+    }
+    // result in caller VIDs (fp64)
+    if (g->ordered) {
+        double* tmp;
+        GTS_TRY(c->buf(kBufBcTmp, n * 8, (void**)&tmp));
+        gather_f64_kernel<<<eg, 256, 0, s>>>(tmp, bc, c->dg.new_of_old, n);
+        bc = tmp;
+    }
+    GTS_TRY(copy_out(c, bc, out, n * 8, rc.out_location));
+    if (st) {
+        std::memset(st, 0, sizeof(*st));
+        st->wall_s = now_s() - t_start;
+        st->upload_s = upload_s;
+        if (timing) {
+            st->main_kernel_s = c->t_main.sum_s();
+            st->merge_s = c->t_merge.sum_s();
+            st->finish_s = c->t_finish.sum_s();
+            st->h2d_s = c->t_h2d.sum_s();
+        }
+        st->pages_processed = pages_processed;
+        st->edges_traversed = edges;
+        st->h2d_bytes = ss.h2d_bytes;
+        st->launches = launches + main_launches;
+        st->main_kernel_launches = main_launches;
+        st->levels_or_iters = levels_total;
+    } else if (timing) {
+        c->t_main.sum_s();
+        c->t_merge.sum_s();
+        c->t_finish.sum_s();
+        c->t_h2d.sum_s();
+    }
+    return GTS_OK;
+}
+
 }  // namespace gts
 
 using namespace gts;
@@ -507,4 +814,9 @@ extern "C" int gts_bfs(gts_context* ctx, const gts_graph* g, uint64_t src, const
 extern "C" int gts_sssp(gts_context* ctx, const gts_graph* g, uint64_t src, const gts_run_config* cfg,
                         uint32_t* dist_out, gts_run_stats* stats) {
     return traverse(ctx, g, src, cfg, dist_out, stats, kSSSP);
+}
+
+extern "C" int gts_bc(gts_context* ctx, const gts_graph* g, const uint64_t* sources, uint32_t num_sources,
+                      const gts_run_config* cfg, double* bc_out, gts_run_stats* stats) {
+    return betweenness(ctx, g, sources, num_sources, cfg, bc_out, stats);
 }

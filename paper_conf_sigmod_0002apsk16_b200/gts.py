@@ -35,7 +35,7 @@ GTS_UNREACHED = 0xFFFFFFFF
 EXPORTED = ["gts_last_error", "gts_version", "gts_build_pages", "gts_plan_pages", "gts_graph_get_stats",
             "gts_graph_pages", "gts_graph_directory", "gts_graph_order", "gts_graph_free", "gts_get_unique_id",
             "gts_context_create", "gts_context_free", "gts_context_evict", "gts_context_set_stream",
-            "gts_bfs", "gts_pagerank", "gts_sssp", "gts_wcc", "gts_partition_pages"]
+            "gts_bfs", "gts_pagerank", "gts_sssp", "gts_wcc", "gts_bc", "gts_partition_pages"]
 
 
 class GtsError(RuntimeError):
@@ -97,6 +97,7 @@ _sig = {
                             ctypes.POINTER(RunStats)]),
     "gts_sssp": (_i32, [_vp, _vp, _u64, ctypes.POINTER(RunConfig), _vp, ctypes.POINTER(RunStats)]),
     "gts_wcc": (_i32, [_vp, _vp, ctypes.POINTER(RunConfig), _vp, ctypes.POINTER(RunStats)]),
+    "gts_bc": (_i32, [_vp, _vp, _vp, _u32, ctypes.POINTER(RunConfig), _vp, ctypes.POINTER(RunStats)]),
     "gts_partition_pages": (_i32, [_vp, _u32, _i32, _vp, _vp]),
 }
 for _name, (_res, _args) in _sig.items():
@@ -312,4 +313,14 @@ def gts_wcc(ctx, graph, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDEN
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing)
     st = RunStats()
     _check(_lib.gts_wcc(ctx.handle, graph.handle, ctypes.byref(cfg), ptr, ctypes.byref(st)))
+    return out, st.as_dict()
+
+
+def gts_bc(ctx, graph, sources, out=None, residency=GTS_RESIDENCY_AUTO, ring_slots=0, batch_pages=0, timing=False):
+    """Betweenness centrality summed over `sources` (fp64, unnormalised).  Returns (bc, stats)."""
+    src = np.ascontiguousarray(sources, dtype=np.uint64)
+    out, ptr, loc = _out(out, graph.n, np.float64)
+    cfg = _run_config(GTS_STRATEGY_P, residency, ring_slots, batch_pages, loc, timing)
+    st = RunStats()
+    _check(_lib.gts_bc(ctx.handle, graph.handle, _np_ptr(src), len(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()

@@ -355,3 +355,34 @@ def test_sssp_near_far_deltas(G, ctx, name, delta, monkeypatch):
     gr = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb)
     got, _ = G.gts_sssp(ctx, gr, 0)
     assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, 0))
+
+
+# --------------------------------------------------- betweenness (NEXT #4) ---
+
+def _bc_check(got, want):
+    err = np.abs(got - want)
+    assert np.all(err <= 1e-9 * np.maximum(1.0, np.abs(want))), (float(err.max()), int(np.argmax(err)))
+
+
+@pytest.mark.parametrize("name", ["fig1", "multi", "path", "bintree", "outstar", "rand", "rmat16_4k", "rmat16_1m",
+                                  "twitter20"])
+@pytest.mark.parametrize("order", [False, True])
+def test_bc_vs_oracle(G, ctx, name, order):
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
+    deg = np.diff(g.row_ptr)
+    srcs = sorted({0, int(np.argmax(deg)), g.n // 3})
+    got, st = G.gts_bc(ctx, gr, srcs)
+    _bc_check(got, oracle.bc(g.row_ptr, g.col, srcs))
+
+
+def test_bc_streamed_and_device_output(G, ctx):
+    import torch
+    g, pb = graph("rmat16_4k")
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
+    want = oracle.bc(g.row_ptr, g.col, [0, 7])
+    got, _ = G.gts_bc(ctx, gr, [0, 7], residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3)
+    _bc_check(got, want)
+    d = torch.empty(g.n, dtype=torch.float64, device="cuda")
+    G.gts_bc(ctx, gr, [0, 7], out=d)
+    _bc_check(d.cpu().numpy(), want)
