@@ -72,7 +72,14 @@ typedef enum {
 
 enum { GTS_PAGE_SP = 0, GTS_PAGE_LP = 1 };
 enum { GTS_ENTRY_VID32 = 0, GTS_ENTRY_PID16_SLOT16 = 1 };
-enum { GTS_STRATEGY_P = 0, GTS_STRATEGY_S = 1 };
+/* Strategy-P: pages partitioned h(j) = j mod N, WA replicated.
+ * Strategy-S: WA range-partitioned, each rank holds the pages of its range and
+ *             routes updates to their owners (north_star "routes updates").
+ * Strategy-S_BCAST: the paper-literal Strategy-S: every rank
+ *             processes every page and keeps only the updates of its own WA
+ *             range; no exchange until the final gather (PageRank; the other
+ *             algorithms run replicated). */
+enum { GTS_STRATEGY_P = 0, GTS_STRATEGY_S = 1, GTS_STRATEGY_S_BCAST = 2 };
 enum { GTS_RESIDENCY_AUTO = 0, GTS_RESIDENT = 1, GTS_STREAMED = 2 };
 enum { GTS_DANGLING_UNIFORM = 0, GTS_DANGLING_DROP = 1 };
 enum { GTS_OUT_HOST = 0, GTS_OUT_DEVICE = 1 };
@@ -168,7 +175,7 @@ int gts_context_set_stream(gts_context* ctx, void* cuda_stream);
 
 typedef struct {
     uint32_t struct_size;     /* sizeof(gts_run_config) */
-    uint32_t strategy;        /* GTS_STRATEGY_P (replicated WA) | GTS_STRATEGY_S (partitioned WA) */
+    uint32_t strategy;        /* GTS_STRATEGY_P | GTS_STRATEGY_S | GTS_STRATEGY_S_BCAST (see above) */
     uint32_t residency;       /* GTS_RESIDENCY_AUTO | GTS_RESIDENT | GTS_STREAMED */
     uint32_t ring_slots;      /* streamed: device ring depth (0 -> 4) */
     uint32_t batch_pages;     /* streamed: pages per H2D batch (0 -> 8) */

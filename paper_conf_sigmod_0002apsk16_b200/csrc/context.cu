@@ -66,6 +66,8 @@ void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t
         for (uint64_t j = 0; j < P; ++j) owner[j] = (int32_t)(j % (uint64_t)world);   // h(j) = j mod N
         return;
     }
+    // Strategy-S and S_BCAST share the WA ranges; under S_BCAST owner[j] is the
+    // WA owner of the page's sources, but every rank processes every page.
     // Strategy-S: contiguous VID ranges cut at page boundaries (never inside an
     // LP run) with ~equal page counts; rank r owns WA[vrange[r], vrange[r+1]).
     uint64_t p = 0;
@@ -153,8 +155,9 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
         const uint64_t P = g->num_pages;
         std::vector<uint32_t> loc(P, UINT32_MAX);
         d.h_local_list.clear();
+        const bool every_page = strategy == GTS_STRATEGY_S_BCAST;   // each rank streams all pages
         for (uint64_t j = 0; j < P; ++j)
-            if (d.h_owner[j] == c->rank) {
+            if (every_page || d.h_owner[j] == c->rank) {
                 loc[j] = (uint32_t)d.h_local_list.size();
                 d.h_local_list.push_back((uint32_t)j);
             }
@@ -253,7 +256,7 @@ int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* 
             return fail(GTS_EINVAL, "gts_run_config.struct_size too small");
         d = *cfg;
     }
-    if (d.strategy > GTS_STRATEGY_S) return fail(GTS_EINVAL, "unknown strategy %u", d.strategy);
+    if (d.strategy > GTS_STRATEGY_S_BCAST) return fail(GTS_EINVAL, "unknown strategy %u", d.strategy);
     if (d.residency > GTS_STREAMED) return fail(GTS_EINVAL, "unknown residency %u", d.residency);
     if (d.out_location > GTS_OUT_DEVICE) return fail(GTS_EINVAL, "unknown out_location %u", d.out_location);
     if (d.ring_slots == 0) d.ring_slots = 4;
@@ -512,7 +515,7 @@ extern "C" int gts_partition_pages(const gts_graph* g, uint32_t strategy, int wo
                                    uint64_t* vrange) {
     clear_error();
     if (!g || !owner || world_size < 1) return fail(GTS_EINVAL, "bad argument");
-    if (strategy > GTS_STRATEGY_S) return fail(GTS_EINVAL, "unknown strategy");
+    if (strategy > GTS_STRATEGY_S_BCAST) return fail(GTS_EINVAL, "unknown strategy");
     std::vector<int32_t> o;
     std::vector<uint64_t> vr;
     partition(g, strategy, world_size, o, vr);

@@ -60,6 +60,7 @@ struct RouteParams {
     uint32_t send_cap[kMaxRanks];
     uint64_t lo, hi;
     int nranks;
+    int drop_remote;                   // paper-literal Strategy-S (broadcast pages): ignore remote updates
 };
 
 __device__ __forceinline__ int route_owner(const RouteParams& rp, uint32_t v) {
@@ -101,7 +102,7 @@ struct PrEmitter {
         if (kMode == kRoute) {
             if (dst < H) atomicAdd(hacc + dst, c);
             else if ((uint64_t)dst >= rp->lo && (uint64_t)dst < rp->hi) atomicAdd(rp->acc_loc + (dst - rp->lo), c);
-            else route_push(*rp, dst, c);
+            else if (!rp->drop_remote) route_push(*rp, dst, c);
             return;
         }
         if (kMode == kDense) {
@@ -245,7 +246,10 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                     const uint32_t deg = (sm.off[tid + 1] - sm.off[tid] - 1) >> wshift;
                     const float xv = ld_stream_f32(x + start + t0 + tid, pol);
                     float c = 0.f;
-                    if (deg == 0) dang += (double)xv;
+                    // dangling mass (R3); a routed rank counts only its own WA range (under
+                    // S_BCAST every rank sees every page)
+                    if (deg == 0 && (kMode != kRoute || (uint64_t)(start + t0 + tid) - rp.lo < rp.hi - rp.lo))
+                        dang += (double)xv;
                     else c = d * xv / (float)deg;
                     sm.c[tid] = c;
                 }
@@ -302,7 +306,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             const float v = hacc[i];
             if (v == 0.f) continue;
             if ((uint64_t)i >= rp.lo && (uint64_t)i < rp.hi) atomicAdd(rp.acc_loc + (i - rp.lo), v);
-            else atomicAdd(rp.hot_out + i, v);
+            else if (!rp.drop_remote) atomicAdd(rp.hot_out + i, v);
         }
     } else {
         for (uint32_t i = tid; i < n_hot; i += T) {
@@ -444,9 +448,10 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     // Strategy-S with routed updates: N > 1 ranks, or (tests, one GPU) GTS_VIRTUAL_RANKS=V
     // virtual ranks run one after another on this GPU with an in-memory exchange
     const char* vre = getenv("GTS_VIRTUAL_RANKS");
-    const int vranks = (rc.strategy == GTS_STRATEGY_S && c->world == 1 && vre) ? std::max(1, atoi(vre)) : 1;
+    const int vranks = (rc.strategy != GTS_STRATEGY_P && c->world == 1 && vre) ? std::max(1, atoi(vre)) : 1;
     const bool virt = vranks > 1;
-    const bool route = rc.strategy == GTS_STRATEGY_S && (c->world > 1 || virt);
+    const bool bcast = rc.strategy == GTS_STRATEGY_S_BCAST;
+    const bool route = (rc.strategy == GTS_STRATEGY_S || bcast) && (c->world > 1 || virt);
     const int R = virt ? vranks : c->world;
     if (route && R > kMaxRanks) return fail(GTS_EUNSUPPORTED, "Strategy-S routing supports at most %d ranks", kMaxRanks);
     double upload_s = 0;
@@ -578,7 +583,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         std::vector<uint64_t> vr;
         partition(g, GTS_STRATEGY_S, R, owner, vr);
         std::vector<std::vector<uint32_t>> plist(R);          // pages of each (virtual) rank
-        for (uint64_t j = 0; j < g->num_pages; ++j) plist[owner[j]].push_back((uint32_t)j);
+        for (uint64_t j = 0; j < g->num_pages; ++j)
+            for (int r = 0; r < R; ++r)
+                if (bcast || owner[j] == r) plist[r].push_back((uint32_t)j);   // S_BCAST: every rank, every page
         const int me = virt ? -1 : c->rank;
         const int r0 = virt ? 0 : me, r1 = virt ? R : me + 1;  // ranks simulated by this process
         uint32_t* d_plist = nullptr;
@@ -599,6 +606,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
             rp.hi = vr[r + 1];
             rp.nranks = R;
             rp.acc_loc = acc + vr[r];
+            rp.drop_remote = bcast ? 1 : 0;
             return rp;
         };
         auto pages_of = [&](int r, const uint32_t*& d, uint32_t& cnt) {
@@ -614,7 +622,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         const void* kcount = g->weighted ? (const void*)route_count_kernel<true> : (const void*)route_count_kernel<false>;
         int cgrid = 0;
         GTS_TRY(sms_grid(c, kcount, kThreads, 0, &cgrid));
-        for (int r = r0; r < r1; ++r) {
+        for (int r = r0; r < r1 && !bcast; ++r) {
             RouteParams rp = make_rp(r);
             const uint32_t* dl;
             uint32_t cnt;
@@ -635,7 +643,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         uint32_t* d_flags = reinterpret_cast<uint32_t*>(d_cnt64 + (size_t)kMaxRanks * kMaxRanks);  // [0] overflow
         uint32_t* d_scnt = d_flags + 8;            // send counts [R] per simulated rank (R x R in virtual mode)
         uint32_t* d_rcnt = d_flags + 8 + kMaxRanks * kMaxRanks;
-        if (!virt) {   // everyone learns what it will receive: all-gather the capacity rows
+        if (!virt && !bcast) {   // everyone learns what it will receive: all-gather the capacity rows
             uint32_t* d_caprow;
             uint32_t* d_capall;
             GTS_TRY(c->buf(kBufRouteHotIn + 10, (size_t)(R + R * R) * 4, (void**)&d_caprow));
@@ -706,6 +714,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                     dense_add_kernel<<<eg, 256, 0, s>>>(acc, d_hot + (size_t)r * n_hot, 0, n_hot);
                     launches += 2;
                 }
+            } else if (bcast) {        // paper-literal S: no exchange, only the dangling mass
+                GTS_NCCL(ncclAllReduce(D, D, 1, ncclFloat64, ncclSum, c->comm, s));
+                nccl_bytes += 8;
             } else {
                 const uint32_t* scnt_me = d_scnt + (size_t)me * kMaxRanks;
                 GTS_NCCL(ncclGroupStart());
@@ -749,6 +760,14 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                                                  dangling == GTS_DANGLING_UNIFORM ? 1 : 0, 0);
             if (timing) cudaEventRecord(ev.second, s);
             ++launches;
+            if (bcast && !virt && it + 1 < iters) {   // every rank reads every source's RA next iteration
+                GTS_NCCL(ncclGroupStart());
+                for (int r = 0; r < R; ++r)
+                    if (vr[r + 1] > vr[r])
+                        GTS_NCCL(ncclBroadcast(x + vr[r], x + vr[r], vr[r + 1] - vr[r], ncclFloat32, r, c->comm, s));
+                GTS_NCCL(ncclGroupEnd());
+                nccl_bytes += n * 4;
+            }
         }
         uint32_t ovf = 0;
         GTS_CUDA(cudaMemcpyAsync(&ovf, d_flags, 4, cudaMemcpyDeviceToHost, s));

@@ -38,6 +38,7 @@ struct BfsOp {
     uint32_t* visited;
     uint32_t* next;
     unsigned long long nedges;
+    uint32_t vprefix;          // every vertex below this ID is already visited (no test needed)
     __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
@@ -57,7 +58,8 @@ struct BfsOp {
                                           const bool* valid) {
         uint32_t vis[kEdgesPerThread];
 #pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q) vis[q] = valid[q] ? __ldca(visited + (dst[q] >> 5)) : ~0u;
+        for (int q = 0; q < kEdgesPerThread; ++q)
+            vis[q] = (valid[q] && dst[q] >= vprefix) ? __ldca(visited + (dst[q] >> 5)) : ~0u;
 #pragma unroll
         for (int q = 0; q < kEdgesPerThread; ++q) {
             const uint32_t wi = dst[q] >> 5, b = 1u << (dst[q] & 31);
@@ -145,9 +147,9 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 template <bool W>
 __global__ void __launch_bounds__(kThreads, 2)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
-                  uint32_t* work_ctr, unsigned long long* edges_out) {
+                  uint32_t* work_ctr, unsigned long long* edges_out, uint32_t vprefix) {
     __shared__ TileSmem sm;
-    BfsOp<W> op{cur, visited, next, 0ull};
+    BfsOp<W> op{cur, visited, next, 0ull, vprefix};
     expand_pages(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
@@ -234,6 +236,20 @@ __global__ void sssp_finish_kernel(const uint32_t* __restrict__ gathered, int wo
     if ((threadIdx.x & 31) == 0 && mn != 0xFFFFFFFFu) atomicMin(minpend, mn);
 }
 
+// Length of the all-visited prefix of the bitmap, in words: the first word that
+// is not all ones.  On a degree-ordered graph the low IDs are the hubs and are
+// reached in the first levels, so later levels skip the visited test of every
+// edge into that prefix.
+__global__ void visited_prefix_kernel(const uint32_t* __restrict__ visited, uint64_t words, unsigned int* first) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
+        const bool hole = visited[w] != 0xFFFFFFFFu;
+        const uint32_t m = __ballot_sync(__activemask(), hole);
+        if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicMin(first, (unsigned int)w);
+        if (__any_sync(__activemask(), hole)) break;   // later words of this thread cannot be smaller
+    }
+}
+
 // Next page set (nextPIDSet, Alg 1 lines 29-30): the pages among
 // `pages` (this rank's) whose VID range [START_VID, START_VID + nslots) has a
 // bit set in `bits`.  One warp per page.
@@ -274,7 +290,7 @@ struct Counters {               // device scratch, slot kCtr
     uint32_t flag2;
     unsigned long long near;       // SSSP: pending vertices within the threshold
     unsigned int minpend;          // SSSP: minimum pending distance
-    unsigned int pad;
+    unsigned int vprefix_words;    // BFS: all-visited prefix of the bitmap (words)
 };
 
 enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather };
@@ -361,6 +377,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     SweepStats ss;
     std::vector<uint32_t> h_list = l0;             // streamed mode: this level's pages on the host (ascending)
     const bool cached = streamed && rc.cache_mib > 0;
+    uint32_t vprefix = 0;
     // SSSP near-far bucketing: expand only pending vertices with dist <= T; T
     // advances by delta past the nearest pending distance when no pending vertex
     // is within it.  Label-correcting, so any delta gives the exact distances.
@@ -377,10 +394,10 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
                                 if (algo == kBFS && g->weighted)
                                     bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(
-                                        ps, cur, visited, next, &ctr->work, &ctr->edges);
+                                        ps, cur, visited, next, &ctr->work, &ctr->edges, vprefix);
                                 else if (algo == kBFS)
                                     bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(
-                                        ps, cur, visited, next, &ctr->work, &ctr->edges);
+                                        ps, cur, visited, next, &ctr->work, &ctr->edges, vprefix);
                                 else
                                     sssp_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(
                                         ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T);
@@ -407,6 +424,9 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         if (algo == kBFS) {
             frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, next,
                                                             visited, value, L + 1, &ctr->count);
+            GTS_CUDA(cudaMemsetAsync(&ctr->vprefix_words, 0xFF, 4, s));
+            visited_prefix_kernel<<<fin_grid, 256, 0, s>>>(visited, words, &ctr->vprefix_words);
+            ++launches;
         } else {
             GTS_CUDA(cudaMemsetAsync(&ctr->near, 0, 8, s));
             GTS_CUDA(cudaMemsetAsync(&ctr->minpend, 0xFF, 4, s));
@@ -423,6 +443,8 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         GTS_CUDA(cudaMemcpyAsync(&h, ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
         GTS_CUDA(cudaStreamSynchronize(s));
         ++levels;
+        if (algo == kBFS)
+            vprefix = (uint32_t)std::min<uint64_t>((uint64_t)std::min<uint64_t>(h.vprefix_words, words) * 32, n);
         if (h.count == 0) break;
         if (algo == kSSSP && h.near == 0) {      // nothing pending within T: open the next bucket
             const uint64_t nt = (uint64_t)h.minpend + delta;
@@ -695,8 +717,8 @@ static int betweenness(gts_context* c, const gts_graph* g, const uint64_t* sourc
                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges);
-                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges);
+                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, 0u);
+                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, 0u);
                 if (timing) cudaEventRecord(ev.second, s);
                 GTS_CUDA(cudaGetLastError());
                 ++main_launches;

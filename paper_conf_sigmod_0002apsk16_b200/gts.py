@@ -24,7 +24,7 @@ GTS_OK = 0
 GTS_EINVAL, GTS_ENOMEM, GTS_ECUDA, GTS_ENCCL, GTS_EUNSUPPORTED, GTS_EOVERFLOW = -1, -2, -3, -4, -5, -6
 GTS_PAGE_SP, GTS_PAGE_LP = 0, 1
 GTS_ENTRY_VID32, GTS_ENTRY_PID16_SLOT16 = 0, 1
-GTS_STRATEGY_P, GTS_STRATEGY_S = 0, 1
+GTS_STRATEGY_P, GTS_STRATEGY_S, GTS_STRATEGY_S_BCAST = 0, 1, 2
 GTS_RESIDENCY_AUTO, GTS_RESIDENT, GTS_STREAMED = 0, 1, 2
 GTS_DANGLING_UNIFORM, GTS_DANGLING_DROP = 0, 1
 GTS_OUT_HOST, GTS_OUT_DEVICE = 0, 1

@@ -386,3 +386,17 @@ def test_bc_streamed_and_device_output(G, ctx):
     d = torch.empty(g.n, dtype=torch.float64, device="cuda")
     G.gts_bc(ctx, gr, [0, 7], out=d)
     _bc_check(d.cpu().numpy(), want)
+
+
+@pytest.mark.parametrize("name", ["rmat16_4k", "twitter20", "instar"])
+@pytest.mark.parametrize("vranks", [2, 5])
+def test_pagerank_strategy_s_bcast(G, ctx, name, vranks, monkeypatch):
+    """Paper-literal Strategy-S: every (virtual) rank sweeps every
+    page and keeps only the updates of its own WA range; no exchange."""
+    monkeypatch.setenv("GTS_VIRTUAL_RANKS", str(vranks))
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+    got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, strategy=G.GTS_STRATEGY_S_BCAST)
+    _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, vranks, "bcast"))
+    lv, _ = G.gts_bfs(ctx, gr, 0, strategy=G.GTS_STRATEGY_S_BCAST)
+    assert np.array_equal(lv, oracle.bfs(g.row_ptr, g.col, 0))
