@@ -588,10 +588,10 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                 if (bcast || owner[j] == r) plist[r].push_back((uint32_t)j);   // S_BCAST: every rank, every page
         const int me = virt ? -1 : c->rank;
         const int r0 = virt ? 0 : me, r1 = virt ? R : me + 1;  // ranks simulated by this process
-        uint32_t* d_plist = nullptr;
-        GTS_TRY(c->buf(kBufRouteList, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&d_plist));
         std::vector<uint32_t> pl_off(R + 1, 0);
         for (int r = 0; r < R; ++r) pl_off[r + 1] = pl_off[r] + (uint32_t)plist[r].size();
+        uint32_t* d_plist = nullptr;              // (S_BCAST: every rank lists every page)
+        GTS_TRY(c->buf(kBufRouteList, std::max<uint64_t>(pl_off[R], 1) * 4, (void**)&d_plist));
         {
             std::vector<uint32_t> flat;
             for (int r = 0; r < R; ++r) flat.insert(flat.end(), plist[r].begin(), plist[r].end());
