@@ -84,6 +84,18 @@ enum { GTS_RESIDENCY_AUTO = 0, GTS_RESIDENT = 1, GTS_STREAMED = 2 };
 enum { GTS_DANGLING_UNIFORM = 0, GTS_DANGLING_DROP = 1 };
 enum { GTS_OUT_HOST = 0, GTS_OUT_DEVICE = 1 };
 enum { GTS_RUN_TIMING = 1u };   /* gts_run_config.flags: time the main kernels with CUDA events */
+/* gts_run_config.flags bits 8-10: the micro-level technique applied inside each
+ * slotted page (App E, Fig 14), for gts_bfs and
+ * gts_pagerank (other calls reject a non-default value with EUNSUPPORTED).
+ *   DEFAULT: the B200 tile engine (BFS) / the hot-set scatter (PageRank);
+ *   EDGE:    edge-centric = VWC, a warp per vertex (the paper's default, Alg 2/4);
+ *   VERTEX:  vertex-centric, a thread per vertex and all of its edges;
+ *   HYBRID:  per page, vertex-centric if the page has < 8 edges per vertex, else
+ *            edge-centric (env GTS_HYBRID_DEG overrides the 8);
+ *   TILE:    PageRank only: the tile engine with one plain red.add per edge (no hot set).
+ * Results are identical for every technique (PageRank: within the fp32 gates). */
+enum { GTS_MICRO_DEFAULT = 0u, GTS_MICRO_EDGE = 1u << 8, GTS_MICRO_VERTEX = 2u << 8,
+       GTS_MICRO_HYBRID = 3u << 8, GTS_MICRO_TILE = 4u << 8, GTS_MICRO_MASK = 7u << 8 };
 /* gts_page_config.flags: store vertices in descending in-degree order (ties by
  * VID) inside the pages.  A builder policy, not a different graph: every call
  * maps its source vertex in and its result out, so callers always see their
@@ -178,9 +190,9 @@ typedef struct {
     uint32_t strategy;        /* GTS_STRATEGY_P | GTS_STRATEGY_S | GTS_STRATEGY_S_BCAST (see above) */
     uint32_t residency;       /* GTS_RESIDENCY_AUTO | GTS_RESIDENT | GTS_STREAMED */
     uint32_t ring_slots;      /* streamed: device ring depth (0 -> 4) */
-    uint32_t batch_pages;     /* streamed: pages per H2D batch (0 -> 8) */
+    uint32_t batch_pages;     /* streamed: pages per H2D batch (0 -> 64 MiB worth of pages) */
     uint32_t out_location;    /* GTS_OUT_HOST (default) | GTS_OUT_DEVICE (out pointer is device memory on this rank's GPU) */
-    uint32_t flags;           /* GTS_RUN_TIMING */
+    uint32_t flags;           /* GTS_RUN_TIMING | one GTS_MICRO_* value */
     uint32_t cache_mib;       /* streamed BFS/SSSP: device LRU cache of topology pages across levels,
                                  in MiB (cachedPIDMap, Alg 1 lines 8/16/29); 0 = none */
 } gts_run_config;

@@ -205,7 +205,74 @@ __device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, cons
     }
 }
 
+// ---- the paper's micro-level techniques (App E / Fig 14) ----
+// Kept beside the tile engine for the Fig 14 comparison (GTS_MICRO_* run flags):
+//   edge-centric   = VWC with W_SZ = 32 (Alg 2 l.9-11, R8): a warp per vertex of
+//                    the SP, its lanes strided over the ADJLIST;
+//   vertex-centric = a thread per vertex and its entire ADJLIST;
+//   hybrid         = per page by density: vertex-centric if the page's edges per
+//                    vertex are below ps.hybrid_deg, else edge-centric (R24).
+// Every vertex of the page is tested (Alg 2 l.12 tests LV of each vertex).
+enum { kMicroTile = 0, kMicroEdge = 1, kMicroVertex = 2, kMicroHybrid = 3 };
+
 template <class Op>
+__device__ __forceinline__ void micro_edges(const PageSet& ps, Op& op, const uint32_t* adj, uint32_t deg,
+                                            uint32_t k0, uint32_t stride, uint32_t pay, uint32_t v, uint64_t pol) {
+    uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
+    bool valid[kEdgesPerThread];
+#pragma unroll
+    for (int q = 0; q < kEdgesPerThread; ++q) {
+        const uint32_t k = k0 + q * stride;
+        valid[q] = k < deg;
+        dst[q] = valid[q] ? ld_stream_u32(adj + k, pol) : 0u;
+        w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_u32(adj + deg + k, pol) : 0u;
+        pl[q] = pay;
+        src[q] = v;
+    }
+#pragma unroll
+    for (int q = 0; q < kEdgesPerThread; ++q) dst[q] = decode_entry(ps, dst[q]);
+    op.edges(dst, w, pl, src, valid);
+}
+
+template <class Op, int kMicro>
+__device__ void expand_sp_micro(const PageSet& ps, Op& op, const uint8_t* data, const uint8_t* end,
+                                uint32_t nslots, uint64_t pol) {
+    const uint32_t* words = reinterpret_cast<const uint32_t*>(data);
+    const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
+    constexpr uint32_t wsh = Op::kWeighted ? 1 : 0;
+    bool vertex = kMicro == kMicroVertex;
+    if (kMicro == kMicroHybrid) {              // page density from its last record's end
+        const uint32_t lo = ld32(end - kSpFooter - kSlotBytes * (uint64_t)nslots + 4);
+        const uint32_t used = lo / 4 + 1 + (ld32(data + lo) << wsh);     // record words
+        const uint32_t nedges = (used - nslots) >> wsh;
+        vertex = nedges < ps.hybrid_deg * nslots;
+    }
+    if (vertex) {
+        for (uint32_t u = threadIdx.x; u < nslots; u += kThreads) {
+            const uint32_t v = start + u;
+            if (!op.select(v)) continue;
+            const uint32_t off = ld_stream_u32(end - kSpFooter - kSlotBytes * (uint64_t)(u + 1) + 4, pol);
+            const uint32_t deg = ld_stream_u32(data + off, pol);
+            const uint32_t pay = op.payload(v, deg);
+            const uint32_t* adj = words + off / 4 + 1;
+            for (uint32_t k0 = 0; k0 < deg; k0 += kEdgesPerThread) micro_edges(ps, op, adj, deg, k0, 1, pay, v, pol);
+        }
+    } else {
+        const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+        for (uint32_t u = warp; u < nslots; u += kWarps) {       // warp-uniform loop
+            const uint32_t v = start + u;
+            if (!op.select(v)) continue;
+            const uint32_t off = ld_stream_u32(end - kSpFooter - kSlotBytes * (uint64_t)(u + 1) + 4, pol);
+            const uint32_t deg = ld_stream_u32(data + off, pol);
+            uint32_t pay = lane == 0 ? op.payload(v, deg) : 0u;
+            pay = __shfl_sync(0xFFFFFFFFu, pay, 0);
+            const uint32_t* adj = words + off / 4 + 1;
+            for (uint32_t k0 = lane; k0 < deg; k0 += 32 * kEdgesPerThread) micro_edges(ps, op, adj, deg, k0, 32, pay, v, pol);
+        }
+    }
+}
+
+template <class Op, int kMicro = kMicroTile>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
     const uint32_t count = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
     const int tid = threadIdx.x;
@@ -247,6 +314,8 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     op.edges(dst, w, pl, src, valid);
                 }
             }
+        } else if (kMicro != kMicroTile) {
+            expand_sp_micro<Op, kMicro>(ps, op, data, end, nslots, pol);
         } else {
             const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
             const uint4* q4 = reinterpret_cast<const uint4*>(data);

@@ -319,6 +319,53 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
     if ((tid & 31) == 0 && dang != 0.0) atomicAdd(dang_out, dang);
 }
 
+// Plain push PageRank (Alg 4/5: c = d x[u] / deg(u), one red.add per edge, no
+// hot set) on the generic page engine, for the micro-level comparison of App E
+// (GTS_MICRO_EDGE / VERTEX / HYBRID / TILE).  Same arguments as pr_scatter_kernel.
+template <bool W>
+struct PrMicroOp {
+    static constexpr bool kReadWeights = false;
+    static constexpr bool kWeighted = W;
+    const float* x;
+    float* acc;
+    float d;
+    double dang;
+    __device__ const uint32_t* frontier() const { return nullptr; }
+    __device__ bool select(uint32_t) { return true; }
+    __device__ uint32_t payload(uint32_t v, uint32_t deg) {
+        const float xv = __ldg(x + v);
+        if (deg == 0) {
+            dang += xv;
+            return 0u;
+        }
+        return __float_as_uint(d * xv / (float)deg);
+    }
+    __device__ bool select_lp(uint32_t vid, uint32_t total, uint32_t, uint32_t& pl) {
+        pl = __float_as_uint(d * __ldg(x + vid) / (float)total);   // R4: total out-degree
+        return true;
+    }
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t* pl, const uint32_t*,
+                                          const bool* valid) {
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q)
+            if (valid[q]) atomicAdd(acc + dst[q], __uint_as_float(pl[q]));
+    }
+    __device__ void end_page() {}
+};
+
+template <bool W, int M>
+__global__ void __launch_bounds__(kThreads, 2)
+pr_micro_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__, float d,
+                double* dang_out, uint32_t* work_ctr, uint32_t, const RouteParams) {
+    __shared__ TileSmem sm;
+    PrMicroOp<W> op{x, acc, d, 0.0};
+    expand_pages<PrMicroOp<W>, M>(ps, op, sm, work_ctr);
+    double v = op.dang;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
+    if ((threadIdx.x & 31) == 0 && v != 0.0) atomicAdd(dang_out, v);
+}
+
 __global__ void pr_init_kernel(float* x, float* acc, uint64_t n, float v0) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
@@ -468,6 +515,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     // scatter variant: degree-ordered graphs use the dense hot set held by one 1024-thread CTA per
     // SM (53,248 floats; GTS_PR_BIG=0 selects two 512-thread CTAs with 24,576 each, 3% slower
     // on RMAT-27); natural-order graphs the hash table; routed Strategy-S always the dense set
+    const uint32_t micro = (rc.flags & GTS_MICRO_MASK) >> 8;
+    if (micro > (GTS_MICRO_TILE >> 8)) return fail(GTS_EINVAL, "unknown GTS_MICRO value");
+    if (micro && route) return fail(GTS_EUNSUPPORTED, "GTS_MICRO_* techniques run without Strategy-S routing");
     const char* pbig = getenv("GTS_PR_BIG");
     const bool big = (g->ordered || route) && (!pbig || atoi(pbig) > 0);
     const int mode = route ? kRoute : (g->ordered ? kDense : kHash);
@@ -475,7 +525,18 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     size_t dyn;
     int threads;
     uint32_t n_hot;
-    if (mode == kHash) {
+    if (micro) {
+        // App E comparison: the generic engine with plain REDs (TILE = 4 -> engine mode kMicroTile)
+        static const void* mk[2][4] = {
+            {(const void*)pr_micro_kernel<false, kMicroTile>, (const void*)pr_micro_kernel<false, kMicroEdge>,
+             (const void*)pr_micro_kernel<false, kMicroVertex>, (const void*)pr_micro_kernel<false, kMicroHybrid>},
+            {(const void*)pr_micro_kernel<true, kMicroTile>, (const void*)pr_micro_kernel<true, kMicroEdge>,
+             (const void*)pr_micro_kernel<true, kMicroVertex>, (const void*)pr_micro_kernel<true, kMicroHybrid>}};
+        kern = mk[g->weighted ? 1 : 0][micro & 3];
+        dyn = 0;
+        threads = kThreads;
+        n_hot = 0;
+    } else if (mode == kHash) {
         kern = g->weighted ? (const void*)pr_scatter_kernel<true, kHash, kThreads, 2, 0>
                            : (const void*)pr_scatter_kernel<false, kHash, kThreads, 2, 0>;
         dyn = pr_dyn_smem<kHash, 0>();
@@ -535,11 +596,15 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     SweepStats ss;
     float dmp = (float)damping;
     const uint32_t* hk = c->dg.hot_keys;
+    const char* hde = getenv("GTS_HYBRID_DEG");
+    const uint32_t hybrid_deg = hde ? (uint32_t)std::max(1L, atol(hde)) : 8u;
     auto scatter = [&](const PageSet& ps, int cap, double* D, const RouteParams& rp) -> int {
         GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
         std::pair<cudaEvent_t, cudaEvent_t> e2;
         if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
-        void* args[] = {(void*)&ps, (void*)&x, (void*)&acc, (void*)&hk, (void*)&dmp, (void*)&D,
+        PageSet p2 = ps;
+        p2.hybrid_deg = hybrid_deg;
+        void* args[] = {(void*)&p2, (void*)&x, (void*)&acc, (void*)&hk, (void*)&dmp, (void*)&D,
                         (void*)&ctr, (void*)&n_hot, (void*)&rp};
         cudaLaunchConfig_t lc;
         std::memset(&lc, 0, sizeof(lc));

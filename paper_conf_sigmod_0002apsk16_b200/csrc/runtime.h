@@ -51,6 +51,7 @@ struct PageSet {
     uint32_t mode;
     uint32_t entry_encoding;
     const uint32_t* rvt_start; // START_VID per page (PID16 decode)
+    uint32_t hybrid_deg = 8;   // GTS_MICRO_HYBRID: vertex-centric below this many edges per vertex (R24)
 };
 
 // Device copy of a graph for one rank.

@@ -144,13 +144,13 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 
 // -------------------------------------------------------------- kernels ---
 
-template <bool W>
+template <bool W, int M = kMicroTile>
 __global__ void __launch_bounds__(kThreads, 2)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
                   uint32_t* work_ctr, unsigned long long* edges_out, uint32_t vprefix) {
     __shared__ TileSmem sm;
     BfsOp<W> op{cur, visited, next, 0ull, vprefix};
-    expand_pages(ps, op, sm, work_ctr);
+    expand_pages<BfsOp<W>, M>(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
 
@@ -365,9 +365,21 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     if (!l0.empty()) GTS_CUDA(cudaMemcpyAsync(list, l0.data(), l0.size() * 4, cudaMemcpyHostToDevice, s));
     GTS_CUDA(cudaMemcpyAsync(&ctr->list_count, hs, 4, cudaMemcpyHostToDevice, s));
 
-    const void* kexp = algo == kBFS ? (g->weighted ? (const void*)bfs_expand_kernel<true>
-                                                   : (const void*)bfs_expand_kernel<false>)
-                                    : (const void*)sssp_expand_kernel;
+    // micro-level technique inside each page (GTS_MICRO_*, App E): BFS only
+    uint32_t micro = (rc.flags & GTS_MICRO_MASK) >> 8;
+    if (micro == (GTS_MICRO_TILE >> 8)) micro = kMicroTile;
+    if (micro > kMicroHybrid) return fail(GTS_EINVAL, "unknown GTS_MICRO value");
+    if (algo == kSSSP && micro) return fail(GTS_EUNSUPPORTED, "GTS_MICRO_* techniques apply to gts_bfs and gts_pagerank");
+    using BfsKern = decltype(&bfs_expand_kernel<false, kMicroTile>);
+    static const BfsKern bfs_k[2][4] = {
+        {bfs_expand_kernel<false, kMicroTile>, bfs_expand_kernel<false, kMicroEdge>,
+         bfs_expand_kernel<false, kMicroVertex>, bfs_expand_kernel<false, kMicroHybrid>},
+        {bfs_expand_kernel<true, kMicroTile>, bfs_expand_kernel<true, kMicroEdge>,
+         bfs_expand_kernel<true, kMicroVertex>, bfs_expand_kernel<true, kMicroHybrid>}};
+    const BfsKern bfs_kern = bfs_k[g->weighted ? 1 : 0][micro];
+    const char* hde = getenv("GTS_HYBRID_DEG");
+    const uint32_t hybrid_deg = hde ? (uint32_t)std::max(1L, atol(hde)) : 8u;
+    const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_expand_kernel;
     int grid = 0;
     GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
     const int fin_grid = c->num_sms * 4;
@@ -392,13 +404,12 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-                                if (algo == kBFS && g->weighted)
-                                    bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(
-                                        ps, cur, visited, next, &ctr->work, &ctr->edges, vprefix);
-                                else if (algo == kBFS)
-                                    bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(
-                                        ps, cur, visited, next, &ctr->work, &ctr->edges, vprefix);
-                                else
+                                if (algo == kBFS) {
+                                    PageSet p2 = ps;
+                                    p2.hybrid_deg = hybrid_deg;
+                                    bfs_kern<<<std::min(grid, cap), kThreads, 0, s>>>(
+                                        p2, cur, visited, next, &ctr->work, &ctr->edges, vprefix);
+                                } else
                                     sssp_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(
                                         ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T);
                                 if (timing) cudaEventRecord(ev.second, s);
@@ -640,6 +651,7 @@ static int betweenness(gts_context* c, const gts_graph* g, const uint64_t* sourc
     for (uint32_t i = 0; i < k; ++i)
         if (sources[i] >= g->n) return fail(GTS_EINVAL, "source %llu >= n", (unsigned long long)sources[i]);
     if (c->world > 1) return fail(GTS_EUNSUPPORTED, "gts_bc runs on one GPU in this version");
+    if (rc.flags & GTS_MICRO_MASK) return fail(GTS_EUNSUPPORTED, "GTS_MICRO_* techniques apply to gts_bfs and gts_pagerank");
     const uint64_t n = g->n, words = (n + 31) / 32;
     const bool streamed = choose_streamed(c, g, rc, 28 * n + 16 * words);
     double upload_s = 0;

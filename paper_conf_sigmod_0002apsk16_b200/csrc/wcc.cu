@@ -113,6 +113,7 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     const double t_start = now_s();
     gts_run_config rc;
     GTS_TRY(validate_common(c, g, cfg, &rc));
+    if (rc.flags & GTS_MICRO_MASK) return fail(GTS_EUNSUPPORTED, "GTS_MICRO_* techniques apply to gts_bfs and gts_pagerank");
     if (!label_out) return fail(GTS_EINVAL, "NULL output");
     const uint64_t n = g->n;
     const bool streamed = choose_streamed(c, g, rc, 4 * n);

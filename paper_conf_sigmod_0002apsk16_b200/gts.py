@@ -29,6 +29,10 @@ GTS_RESIDENCY_AUTO, GTS_RESIDENT, GTS_STREAMED = 0, 1, 2
 GTS_DANGLING_UNIFORM, GTS_DANGLING_DROP = 0, 1
 GTS_OUT_HOST, GTS_OUT_DEVICE = 0, 1
 GTS_RUN_TIMING = 1
+# micro-level technique inside each page (gts_run_config.flags bits 8-10; App E, Fig 14)
+GTS_MICRO_DEFAULT, GTS_MICRO_EDGE, GTS_MICRO_VERTEX, GTS_MICRO_HYBRID, GTS_MICRO_TILE = 0, 1 << 8, 2 << 8, 3 << 8, 4 << 8
+MICRO = {"default": GTS_MICRO_DEFAULT, "edge": GTS_MICRO_EDGE, "vertex": GTS_MICRO_VERTEX,
+         "hybrid": GTS_MICRO_HYBRID, "tile": GTS_MICRO_TILE}
 GTS_BUILD_DEGREE_ORDER = 1
 GTS_UNREACHED = 0xFFFFFFFF
 
@@ -256,9 +260,10 @@ def gts_context_create(device=0, rank=0, world_size=1, unique_id: bytes | None =
     return Context(h, device, rank, world_size)
 
 
-def _run_config(strategy, residency, ring_slots, batch_pages, out_location, timing, cache_mib=0):
+def _run_config(strategy, residency, ring_slots, batch_pages, out_location, timing, cache_mib=0, micro=0):
+    micro = MICRO[micro] if isinstance(micro, str) else int(micro)
     return RunConfig(ctypes.sizeof(RunConfig), strategy, residency, ring_slots, batch_pages, out_location,
-                     GTS_RUN_TIMING if timing else 0, int(cache_mib))
+                     (GTS_RUN_TIMING if timing else 0) | micro, int(cache_mib))
 
 
 def _out(out, n, dtype):
@@ -279,19 +284,20 @@ def _out(out, n, dtype):
 
 
 def gts_bfs(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-            batch_pages=0, timing=False, cache_mib=0):
-    """Returns (levels, stats dict)."""
+            batch_pages=0, timing=False, cache_mib=0, micro=GTS_MICRO_DEFAULT):
+    """Returns (levels, stats dict).  micro: GTS_MICRO_* or "default"/"edge"/"vertex"/"hybrid"."""
     out, ptr, loc = _out(out, graph.n, np.uint32)
-    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib)
+    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib, micro)
     st = RunStats()
     _check(_lib.gts_bfs(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()
 
 
 def gts_pagerank(ctx, graph, iters=10, damping=0.85, dangling=GTS_DANGLING_UNIFORM, out=None,
-                 strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0, batch_pages=0, timing=False):
+                 strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0, batch_pages=0, timing=False,
+                 micro=GTS_MICRO_DEFAULT):
     out, ptr, loc = _out(out, graph.n, np.float32)
-    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing)
+    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, 0, micro)
     st = RunStats()
     _check(_lib.gts_pagerank(ctx.handle, graph.handle, int(iters), float(damping), int(dangling),
                              ctypes.byref(cfg), ptr, ctypes.byref(st)))

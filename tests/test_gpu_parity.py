@@ -400,3 +400,80 @@ def test_pagerank_strategy_s_bcast(G, ctx, name, vranks, monkeypatch):
     _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, vranks, "bcast"))
     lv, _ = G.gts_bfs(ctx, gr, 0, strategy=G.GTS_STRATEGY_S_BCAST)
     assert np.array_equal(lv, oracle.bfs(g.row_ptr, g.col, 0))
+
+
+# ---- micro-level techniques inside a page (App E / Fig 14) ----
+
+MICRO_GRAPHS = ["fig1", "path", "outstar", "instar", "multi", "bintree", "rmat16_4k", "rmat16_256", "rmat20",
+                "twitter20"]
+
+
+@pytest.mark.parametrize("name", MICRO_GRAPHS)
+@pytest.mark.parametrize("micro", ["edge", "vertex", "hybrid"])
+def test_bfs_micro_variants(G, ctx, name, micro):
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
+    deg = np.diff(g.row_ptr).astype(np.int64)
+    for src in _sources(g):
+        want = oracle.bfs(g.row_ptr, g.col, src)
+        got, st = G.gts_bfs(ctx, gr, src, micro=micro)
+        assert np.array_equal(got, want), (name, micro, src, int(np.sum(got != want)))
+        assert st["edges_traversed"] == int(deg[want != oracle.UNREACHED].sum())
+
+
+@pytest.mark.parametrize("micro", ["edge", "vertex", "hybrid"])
+def test_bfs_micro_weighted_pid16_streamed(G, ctx, micro):
+    """Weighted records (adj + w words), PID16 entries and streamed pages under each technique."""
+    g, pb = graph("rmat16_4k")
+    w = inputs.edge_weights(g)
+    want = oracle.bfs(g.row_ptr, g.col, 0)
+    gw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=8192)
+    got, _ = G.gts_bfs(ctx, gw, 0, micro=micro)
+    assert np.array_equal(got, want)
+    gp = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, entry_encoding=G.GTS_ENTRY_PID16_SLOT16)
+    got, _ = G.gts_bfs(ctx, gp, 0, micro=micro)
+    assert np.array_equal(got, want)
+    gs = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
+    got, st = G.gts_bfs(ctx, gs, 0, micro=micro, residency=G.GTS_STREAMED, ring_slots=2, batch_pages=5)
+    assert np.array_equal(got, want) and st["h2d_bytes"] > 0
+
+
+@pytest.mark.parametrize("hdeg", ["1", "1000000"])
+def test_hybrid_threshold_extremes(G, ctx, hdeg, monkeypatch):
+    """GTS_HYBRID_DEG=1 sends (almost) every page edge-centric, 10^6 every page vertex-centric."""
+    monkeypatch.setenv("GTS_HYBRID_DEG", hdeg)
+    g, pb = graph("rmat20")
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=65536)
+    got, _ = G.gts_bfs(ctx, gr, 0, micro="hybrid")
+    assert np.array_equal(got, oracle.bfs(g.row_ptr, g.col, 0))
+    pr, _ = G.gts_pagerank(ctx, gr, 10, 0.85, micro="hybrid")
+    _pr_check(pr, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, ("hybrid", hdeg))
+
+
+@pytest.mark.parametrize("name", ["fig1", "outstar", "multi", "bintree", "rmat16_4k", "rmat16_256", "rmat20",
+                                  "twitter20"])
+@pytest.mark.parametrize("micro", ["edge", "vertex", "hybrid", "tile"])
+def test_pagerank_micro_variants(G, ctx, name, micro):
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
+    for mode in (G.GTS_DANGLING_UNIFORM, G.GTS_DANGLING_DROP):
+        got, st = G.gts_pagerank(ctx, gr, 10, 0.85, mode, micro=micro)
+        _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85, dangling=mode), g, (name, micro, mode))
+
+
+def test_micro_rejected_elsewhere(G, ctx):
+    g, pb = graph("rmat16_4k")
+    w = inputs.edge_weights(g)
+    gr = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=8192)
+    import ctypes
+    from paper_conf_sigmod_0002apsk16_b200 import gts as B
+    out = np.empty(g.n, np.uint32)
+    for micro in ("edge", "vertex", "hybrid"):
+        cfg = B._run_config(0, 0, 0, 0, 0, False, 0, micro)
+        rc = B._lib.gts_sssp(ctx.handle, gr.handle, 0, ctypes.byref(cfg), ctypes.c_void_p(out.ctypes.data), None)
+        assert rc == G.GTS_EUNSUPPORTED
+        rc = B._lib.gts_wcc(ctx.handle, gr.handle, ctypes.byref(cfg), ctypes.c_void_p(out.ctypes.data), None)
+        assert rc == G.GTS_EUNSUPPORTED
+    bad = B._run_config(0, 0, 0, 0, 0, False, 0, 7 << 8)
+    rc = B._lib.gts_bfs(ctx.handle, gr.handle, 0, ctypes.byref(bad), ctypes.c_void_p(out.ctypes.data), None)
+    assert rc == G.GTS_EINVAL
