@@ -319,6 +319,187 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
     if ((tid & 31) == 0 && dang != 0.0) atomicAdd(dang_out, dang);
 }
 
+// ---- Warp-window page walk ---------------------------------------------------
+//
+// The record region of a tile of T vertices is cut into 128-word windows (one
+// 16-byte load per lane, 512 contiguous bytes per warp); each warp walks a
+// contiguous run of windows.  The owner of every word comes from a 128-bit
+// record-start mask built with four redux.or per 32 candidate slots and a
+// popcount prefix, instead of a binary search per 16 bytes: the owner of word
+// i is j0 + #(record starts at or before i), j0 = the last vertex starting
+// before the window (carried from window to window).
+struct WinMask {
+    uint32_t m[4];
+};
+
+// record starts in [base, base + 128) among off[j0 + 1 .. nv)
+__device__ __forceinline__ WinMask win_mask(const uint32_t* off, int j0, uint32_t nv, uint32_t base, int& nstarts) {
+    const int lane = threadIdx.x & 31;
+    WinMask wm{{0u, 0u, 0u, 0u}};
+    nstarts = 0;
+    for (int r = j0 + 1;; r += 32) {
+        const int j = r + lane;
+        const uint32_t o = (uint32_t)j < nv ? off[j] : 0xFFFFFFFFu;
+        const bool in = o - base < 128u && o >= base;
+        const uint32_t p = o - base;
+        const uint32_t bit = in ? 1u << (p & 31) : 0u;
+        wm.m[0] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 0) ? bit : 0u);
+        wm.m[1] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 1) ? bit : 0u);
+        wm.m[2] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 2) ? bit : 0u);
+        wm.m[3] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 3) ? bit : 0u);
+        const uint32_t b = __ballot_sync(0xFFFFFFFFu, in);
+        nstarts += __popc(b);
+        if (b != 0xFFFFFFFFu) break;        // offsets ascend: a gap means no later start in the window
+    }
+    return wm;
+}
+
+template <bool kWeighted, int T, int kMinBlocks, uint32_t H>
+__global__ void __launch_bounds__(T, kMinBlocks)
+pr_scatter_ww_kernel(PageSet ps, const float* __restrict__ x, float* acc, float d, double* dang_out,
+                     uint32_t* work_ctr, uint32_t n_hot) {
+    __shared__ PrSmem<T> sm;
+    extern __shared__ uint4 dyn_smem[];
+    float* hacc = reinterpret_cast<float*>(dyn_smem);
+    constexpr int kW = T / 32;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    for (uint32_t i = tid; i < H; i += T) hacc[i] = 0.f;
+    __syncthreads();
+    const uint64_t pol = policy_evict_first();
+    const uint32_t count = ps.count;
+    const uint32_t enc = ps.entry_encoding;
+    constexpr uint32_t wshift = kWeighted ? 1 : 0;
+    PrEmitter<kDense, H> em{acc, nullptr, hacc, nullptr, 0u, 0.f, false};
+    double dang = 0.0;
+    for (;;) {
+        if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
+        __syncthreads();
+        const uint32_t it = sm.item;
+        __syncthreads();
+        if (it >= count) break;
+        uint32_t pid;
+        const uint8_t* data;
+        page_at(ps, it, pid, data);
+        const uint8_t* end = data + ps.page_bytes;
+        const uint32_t kind = ld32(end - 4);
+        const uint32_t nslots = ld32(end - 8);
+        const uint4* q4 = reinterpret_cast<const uint4*>(data);
+        if (kind == GTS_PAGE_LP) {
+            const uint32_t vid = ld32(end - kLpFooter - kSlotBytes);
+            const uint32_t total = ld32(end - 16);
+            const uint32_t len = ld32(data);
+            const float c = d * __ldg(x + vid) / (float)total;
+            const uint32_t wend = 1 + len, qend = (wend + 3) >> 2;
+            for (uint32_t qb = tid; qb < qend; qb += T * kPrUnroll) {
+                uint4 v[kPrUnroll];
+#pragma unroll
+                for (int u = 0; u < kPrUnroll; ++u) {
+                    const uint32_t q = qb + u * T;
+                    if (q < qend) v[u] = ld_stream_v4(q4 + q, pol);
+                }
+#pragma unroll
+                for (int u = 0; u < kPrUnroll; ++u) {
+                    const uint32_t q = qb + u * T;
+                    if (q >= qend) break;
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        const uint32_t w = 4 * q + k;
+                        if (w >= 1 && w < wend) em.edge(pr_decode(word_of(v[u], k), enc, ps.rvt_start), c);
+                    }
+                }
+            }
+        } else {
+            const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
+            for (uint32_t t0 = 0; t0 < nslots; t0 += T) {
+                const uint32_t nv = min((uint32_t)T, nslots - t0);
+                if ((uint32_t)tid < nv) {
+                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
+                    sm.off[tid] = ld_stream_u32(slot + 4, pol) >> 2;
+                    if ((uint32_t)tid == nv - 1) {
+                        if (t0 + nv < nslots) {
+                            sm.off[nv] = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
+                        } else {
+                            const uint32_t o = ld_stream_u32(slot + 4, pol);
+                            sm.off[nv] = (o >> 2) + 1 + (ld32(data + o) << wshift);
+                        }
+                    }
+                }
+                __syncthreads();
+                if ((uint32_t)tid < nv) {
+                    const uint32_t deg = (sm.off[tid + 1] - sm.off[tid] - 1) >> wshift;
+                    const float xv = ld_stream_f32(x + start + t0 + tid, pol);
+                    float c = 0.f;
+                    if (deg == 0) dang += (double)xv;      // dangling mass (R3)
+                    else c = d * xv / (float)deg;
+                    sm.c[tid] = c;
+                }
+                __syncthreads();
+                const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
+                const uint32_t wbase = W0 & ~3u;
+                const uint32_t nwin = (W1 - wbase + 127) >> 7;
+                // contiguous run of windows per warp
+                const uint32_t per = (nwin + kW - 1) / kW;
+                const uint32_t wa = min(nwin, warp * per), wb = min(nwin, wa + per);
+                if (wa < wb) {
+                    const uint32_t base = wbase + (wa << 7);
+                    // j0 = last vertex whose record starts before base (-1: none)
+                    int lo = -1, hi = (int)nv;               // off[lo] < base <= off[hi]
+                    while (hi - lo > 1) {
+                        const int mid = (lo + hi) >> 1;
+                        if (sm.off[mid] < base) lo = mid; else hi = mid;
+                    }
+                    int j0 = lo;
+                    for (uint32_t wi = wa; wi < wb; wi += kPrUnroll) {
+                        uint4 v[kPrUnroll];                  // kPrUnroll windows' loads in flight
+#pragma unroll
+                        for (int u = 0; u < kPrUnroll; ++u) {
+                            const uint32_t q = ((wbase + ((wi + u) << 7)) >> 2) + lane;
+                            v[u] = make_uint4(0u, 0u, 0u, 0u);
+                            if (wi + u < wb && 4 * q < W1) v[u] = ld_stream_v4(q4 + q, pol);
+                        }
+#pragma unroll
+                        for (int u = 0; u < kPrUnroll; ++u) {
+                            if (wi + u >= wb) break;
+                            const uint32_t bw = wbase + ((wi + u) << 7);
+                            const uint32_t q = (bw >> 2) + lane;
+                            int ns;
+                            const WinMask wm = win_mask(sm.off, j0, nv, bw, ns);
+                            const uint32_t mw = lane >> 3;
+                            uint32_t before = 0;
+#pragma unroll
+                            for (int k = 0; k < 4; ++k) before += (uint32_t)k < mw ? __popc(wm.m[k]) : 0u;
+                            const uint32_t mword = mw == 0 ? wm.m[0] : mw == 1 ? wm.m[1] : mw == 2 ? wm.m[2] : wm.m[3];
+#pragma unroll
+                            for (int k = 0; k < 4; ++k) {
+                                const uint32_t w = 4 * q + k;
+                                const uint32_t bpos = (4 * lane + k) & 31;
+                                if (w < W0 || w >= W1 || ((mword >> bpos) & 1u)) continue;
+                                const int j = j0 + (int)(before + __popc(mword & ((2u << bpos) - 1u)));
+                                if (kWeighted) {
+                                    const uint32_t o = sm.off[j];
+                                    if (w - o > ((sm.off[j + 1] - o - 1) >> 1)) continue;   // weight words
+                                }
+                                em.edge(pr_decode(word_of(v[u], k), enc, ps.rvt_start), sm.c[j]);
+                            }
+                            j0 += ns;
+                        }
+                    }
+                }
+                __syncthreads();
+            }
+        }
+        em.flush();
+    }
+    __syncthreads();
+    for (uint32_t i = tid; i < n_hot; i += T) {
+        const float v = hacc[i];
+        if (v != 0.f) atomicAdd(acc + i, v);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) dang += __shfl_down_sync(0xFFFFFFFFu, dang, o);
+    if ((tid & 31) == 0 && dang != 0.0) atomicAdd(dang_out, dang);
+}
+
 // Plain push PageRank (Alg 4/5: c = d x[u] / deg(u), one red.add per edge, no
 // hot set) on the generic page engine, for the micro-level comparison of App E
 // (GTS_MICRO_EDGE / VERTEX / HYBRID / TILE).  Same arguments as pr_scatter_kernel.
@@ -474,8 +655,492 @@ __global__ void dense_add_kernel(float* acc, float* hot, uint64_t a, uint64_t b)
     }
 }
 
+// ---- Binned scatter (propagation blocking) for degree-ordered pages ---------
+//
+// The plain scatter issues one L2 reduction per cold edge (~1.7 G per RMAT-27
+// iteration), and L2 reduction throughput (~188 G/s measured) is what bounds
+// it.  The binned scatter keeps Alg 4/5's push order but defers the WA update
+// (DESIGN.md section 6b):
+//   phase 1 (pr_bin_kernel): the page sweep; hot destinations [0, hot) are
+//     summed per CTA in shared memory as before; every other (dst, c) pair is
+//     appended to the bin of dst's range: a CTA stages up to kPbStage pairs of
+//     a round in shared memory, counting-sorts them by bin and writes each
+//     bin's run with one global cursor bump (coalesced 8-byte pairs);
+//   phase 2 (pr_apply_kernel): per (bin, chunk) work item, fine bins (ranges
+//     of 2^fine_shift vertices) are summed in a shared-memory slice of WA and
+//     flushed with 16-byte reductions; coarse bins (the cold tail, whose WA
+//     slice stays L2-resident while its items run) take one L2 red per pair.
+// Same additions per destination as Alg 4 l.16, grouped by destination range.
+constexpr int kPbThreads = 512;
+constexpr int kPbBlocks = 2;                                   // CTAs per SM (phase 1)
+constexpr uint32_t kPbUnroll = 2;                              // 16-byte words per thread per round
+constexpr uint32_t kPbStage = kPbThreads * kPbUnroll * 4;      // pairs staged per round (4096)
+constexpr uint32_t kPbMaxBins = 1024;                          // two bins per thread in the scan
+constexpr uint32_t kPbHot = 8192;                              // shared-memory hot set (32 KB)
+constexpr uint32_t kPbFineShiftMax = 15;                       // phase-2 slice: 2^15 floats (128 KB)
+constexpr int kPbWarps = kPbThreads / 32;
+
+struct PbGeom {
+    uint32_t hot;          // destinations [0, hot) use the shared-memory hot set (multiple of 4, <= kPbHot)
+    uint32_t fine_shift;   // fine bins: 2^fine_shift vertices each, starting at `hot`
+    uint32_t nfine;
+    uint32_t coarse_shift; // coarse bins: 2^coarse_shift vertices each, starting at fine_end
+    uint32_t nbins;
+    uint64_t fine_end;     // hot + nfine << fine_shift
+    uint64_t n;
+};
+
+__device__ __forceinline__ uint32_t pb_bin(const PbGeom& g, uint32_t v) {
+    return (uint64_t)v < g.fine_end ? (v - g.hot) >> g.fine_shift
+                                    : g.nfine + (uint32_t)(((uint64_t)v - g.fine_end) >> g.coarse_shift);
+}
+
+struct PbParams {
+    PbGeom geo;
+    uint2* pairs;                 // bin b occupies pairs[boff[b], boff[b] + cap[b])
+    const uint32_t* boff;         // [nbins]
+    uint32_t* cur;                // [nbins] pairs appended (phase 1), zeroed before the sweep
+    unsigned long long* count;    // count mode: [nbins] pairs per bin
+};
+
+struct PbSmem {                   // dynamic shared memory after the hot set
+    uint2 stage[kPbStage];
+    uint16_t sbin[kPbStage];
+    uint32_t hist[kPbMaxBins];
+    uint32_t start[kPbMaxBins];
+    uint32_t gpos[kPbMaxBins];
+    uint32_t wsum[kPbWarps];
+};
+
+__device__ __forceinline__ void st_stream_v2(uint2* p, uint2 v) {
+    asm volatile("st.global.cs.v2.u32 [%0], {%1,%2};" ::"l"(p), "r"(v.x), "r"(v.y) : "memory");
+}
+
+// Per-thread run combiner for hot destinations (rows are sorted, so a thread's
+// consecutive edges often share a hub): one shared-memory add per run, which
+// keeps a hub's fp32 sum two-level (SURVEY section 7 hard parts).
+struct HotRun {
+    uint32_t last;
+    float sum;
+    __device__ __forceinline__ void add(float* hacc, uint32_t v, float c) {
+        if (v == last) {
+            sum += c;
+            return;
+        }
+        if (last != 0xFFFFFFFFu) atomicAdd(hacc + last, sum);
+        last = v;
+        sum = c;
+    }
+    __device__ __forceinline__ void flush(float* hacc) {
+        if (last != 0xFFFFFFFFu) atomicAdd(hacc + last, sum);
+        last = 0xFFFFFFFFu;
+    }
+};
+
+constexpr uint32_t kNoEdge = 0xFFFFFFFFu;   // VIDs are < 2^32 - 1 (n <= 2^32 - 1)
+
+// One staging round of the CTA: every thread hands in up to kPbUnroll*4 edges
+// (dst[k], c[k]; dst[k] = kNoEdge: no edge).  Hot destinations go to the thread's
+// run combiner; the rest are ranked per bin (shared-memory counters),
+// counting-sorted into stage[] and written out bin run by bin run, one global
+// cursor bump per non-empty bin.  Four barriers; all threads call.
+template <bool kCount>
+__device__ __forceinline__ void pb_round(const PbParams& pb, float* hacc, HotRun& hr, PbSmem& s, const uint32_t* dst,
+                                         const float* c) {
+    constexpr int E = kPbUnroll * 4;
+    uint32_t rk[E / 2];                                // per-bin ranks, two 16-bit halves; 0xFFFF = none
+#pragma unroll
+    for (int k = 0; k < E; ++k) {
+        uint32_t r = 0xFFFFu;
+        if (dst[k] != kNoEdge) {
+            if (dst[k] < pb.geo.hot) {
+                if (!kCount) hr.add(hacc, dst[k], c[k]);
+            } else {
+                r = atomicAdd(s.hist + pb_bin(pb.geo, dst[k]), 1u);
+            }
+        }
+        if (k & 1) rk[k >> 1] |= r << 16;
+        else rk[k >> 1] = r;
+    }
+    if (kCount) return;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    __syncthreads();
+    // exclusive scan of hist[0, nbins): thread t owns bins 2t, 2t+1
+    const uint32_t b0 = 2 * tid;
+    const uint32_t h0 = b0 < pb.geo.nbins ? s.hist[b0] : 0u;
+    const uint32_t h1 = b0 + 1 < pb.geo.nbins ? s.hist[b0 + 1] : 0u;
+    uint32_t x = h0 + h1;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) s.wsum[warp] = x;
+    __syncthreads();
+    uint32_t before = 0, total = 0;
+#pragma unroll
+    for (int w = 0; w < kPbWarps; ++w) {
+        const uint32_t v = s.wsum[w];
+        before += w < warp ? v : 0u;
+        total += v;
+    }
+    const uint32_t e0 = before + x - h0 - h1;
+    if (b0 < pb.geo.nbins) {
+        s.start[b0] = e0;
+        s.gpos[b0] = h0 ? __ldg(pb.boff + b0) + atomicAdd(pb.cur + b0, h0) : 0u;
+        s.hist[b0] = 0u;
+    }
+    if (b0 + 1 < pb.geo.nbins) {
+        s.start[b0 + 1] = e0 + h0;
+        s.gpos[b0 + 1] = h1 ? __ldg(pb.boff + b0 + 1) + atomicAdd(pb.cur + b0 + 1, h1) : 0u;
+        s.hist[b0 + 1] = 0u;
+    }
+    __syncthreads();                                   // start / gpos of every bin written
+#pragma unroll
+    for (int k = 0; k < E; ++k) {
+        const uint32_t r = (rk[k >> 1] >> ((k & 1) * 16)) & 0xFFFFu;
+        if (r == 0xFFFFu) continue;
+        const uint32_t b = pb_bin(pb.geo, dst[k]), pos = s.start[b] + r;
+        s.stage[pos] = make_uint2(dst[k], __float_as_uint(c[k]));
+        s.sbin[pos] = (uint16_t)b;
+    }
+    __syncthreads();
+    for (uint32_t i = tid; i < total; i += kPbThreads) {
+        const uint32_t b = s.sbin[i];
+        st_stream_v2(pb.pairs + (s.gpos[b] + (i - s.start[b])), s.stage[i]);
+    }
+}
+
+// Phase 1.  Same page walk as pr_scatter_kernel (tiles of T slots, 16-byte
+// evict_first record loads, owner search per 16 bytes), but rounds are
+// CTA-uniform so the staging barriers line up.  kCount: only count pairs per
+// bin (sizes the bins once per graph).
+template <bool kWeighted, bool kCount>
+__global__ void __launch_bounds__(kPbThreads, kPbBlocks)
+pr_bin_kernel(PageSet ps, const float* __restrict__ x, float* acc, float d, double* dang_out, uint32_t* work_ctr,
+              const PbParams pb) {
+    constexpr int T = kPbThreads;
+    constexpr int E = kPbUnroll * 4;
+    __shared__ PrSmem<T> sm;
+    extern __shared__ uint4 dyn_smem[];
+    float* hacc = reinterpret_cast<float*>(dyn_smem);
+    PbSmem& s = *reinterpret_cast<PbSmem*>(hacc + kPbHot);
+    const int tid = threadIdx.x;
+    if (!kCount)
+        for (uint32_t i = tid; i < pb.geo.hot; i += T) hacc[i] = 0.f;
+    for (uint32_t i = tid; i < kPbMaxBins; i += T) s.hist[i] = 0u;
+    __syncthreads();
+    const uint64_t pol = policy_evict_first();
+    const uint32_t count = ps.count;
+    const uint32_t enc = ps.entry_encoding;
+    constexpr uint32_t wshift = kWeighted ? 1 : 0;
+    double dang = 0.0;
+    HotRun hr{0xFFFFFFFFu, 0.f};
+    uint32_t dst[E];
+    float cv[E];
+    for (;;) {
+        if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
+        __syncthreads();
+        const uint32_t it = sm.item;
+        __syncthreads();
+        if (it >= count) break;
+        uint32_t pid;
+        const uint8_t* data;
+        page_at(ps, it, pid, data);
+        const uint8_t* end = data + ps.page_bytes;
+        const uint32_t kind = ld32(end - 4);
+        const uint32_t nslots = ld32(end - 8);
+        const uint4* q4 = reinterpret_cast<const uint4*>(data);
+        if (kind == GTS_PAGE_LP) {
+            const uint32_t vid = ld32(end - kLpFooter - kSlotBytes);
+            const uint32_t total = ld32(end - 16);
+            const uint32_t len = ld32(data);
+            const float c = kCount ? 0.f : d * __ldg(x + vid) / (float)total;
+            const uint32_t wend = 1 + len, qend = (wend + 3) >> 2;
+            for (uint32_t qb0 = 0; qb0 < qend; qb0 += T * kPbUnroll) {
+                uint4 v[kPbUnroll];
+#pragma unroll
+                for (int u = 0; u < (int)kPbUnroll; ++u) {
+                    const uint32_t q = qb0 + tid + u * T;
+                    if (q < qend) v[u] = ld_stream_v4(q4 + q, pol);
+                }
+#pragma unroll
+                for (int u = 0; u < (int)kPbUnroll; ++u) {
+                    const uint32_t q = qb0 + tid + u * T;
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        const uint32_t w = 4 * q + k;
+                        const bool e = q < qend && w >= 1 && w < wend;
+                        dst[u * 4 + k] = e ? pr_decode(word_of(v[u], k), enc, ps.rvt_start) : kNoEdge;
+                        cv[u * 4 + k] = c;
+                    }
+                }
+                pb_round<kCount>(pb, hacc, hr, s, dst, cv);
+            }
+        } else {
+            const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
+            for (uint32_t t0 = 0; t0 < nslots; t0 += T) {
+                const uint32_t nv = min((uint32_t)T, nslots - t0);
+                if ((uint32_t)tid < nv) {
+                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
+                    sm.off[tid] = ld_stream_u32(slot + 4, pol) >> 2;
+                    if ((uint32_t)tid == nv - 1) {
+                        if (t0 + nv < nslots) {
+                            sm.off[nv] = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
+                        } else {
+                            const uint32_t o = ld_stream_u32(slot + 4, pol);
+                            sm.off[nv] = (o >> 2) + 1 + (ld32(data + o) << wshift);
+                        }
+                    }
+                }
+                __syncthreads();
+                if (!kCount && (uint32_t)tid < nv) {
+                    const uint32_t deg = (sm.off[tid + 1] - sm.off[tid] - 1) >> wshift;
+                    const float xv = ld_stream_f32(x + start + t0 + tid, pol);
+                    float c = 0.f;
+                    if (deg == 0) dang += (double)xv;     // dangling mass (R3)
+                    else c = d * xv / (float)deg;
+                    sm.c[tid] = c;
+                }
+                __syncthreads();
+                const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
+                const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
+                for (uint32_t qb0 = qbeg; qb0 < qend; qb0 += T * kPbUnroll) {
+                    uint4 v[kPbUnroll];
+#pragma unroll
+                    for (int u = 0; u < (int)kPbUnroll; ++u) {
+                        const uint32_t q = qb0 + tid + u * T;
+                        if (q < qend) v[u] = ld_stream_v4(q4 + q, pol);
+                    }
+#pragma unroll
+                    for (int u = 0; u < (int)kPbUnroll; ++u) {
+                        const uint32_t q = qb0 + tid + u * T;
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) dst[u * 4 + k] = kNoEdge;
+                        if (q >= qend) continue;
+                        const uint32_t w0 = 4 * q;
+                        uint32_t lo = 0, hi = nv;               // off[lo] <= max(w0, W0) < off[hi]
+                        while (hi - lo > 1) {
+                            const uint32_t mid = (lo + hi) >> 1;
+                            if (sm.off[mid] <= w0) lo = mid; else hi = mid;
+                        }
+                        uint32_t j = lo, cur = sm.off[j], nxt = sm.off[j + 1];
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            const uint32_t w = w0 + k;
+                            if (w < W0 || w >= W1) continue;
+                            while (w >= nxt) {
+                                ++j;
+                                cur = nxt;
+                                nxt = sm.off[j + 1];
+                            }
+                            const uint32_t rel = w - cur;     // 0 = ADJLIST_SZ word; > deg = weight words
+                            if (rel == 0 || rel > ((nxt - cur - 1) >> wshift)) continue;
+                            dst[u * 4 + k] = pr_decode(word_of(v[u], k), enc, ps.rvt_start);
+                            cv[u * 4 + k] = kCount ? 0.f : sm.c[j];
+                        }
+                    }
+                    pb_round<kCount>(pb, hacc, hr, s, dst, cv);
+                }
+                __syncthreads();
+            }
+        }
+    }
+    __syncthreads();
+    if (kCount) {
+        for (uint32_t b = tid; b < pb.geo.nbins; b += T)
+            if (s.hist[b]) atomicAdd(pb.count + b, (unsigned long long)s.hist[b]);
+        return;
+    }
+    hr.flush(hacc);
+    __syncthreads();
+    for (uint32_t i = tid; i < pb.geo.hot; i += T) {
+        const float v = hacc[i];
+        if (v != 0.f) atomicAdd(acc + i, v);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) dang += __shfl_down_sync(0xFFFFFFFFu, dang, o);
+    if ((tid & 31) == 0 && dang != 0.0) atomicAdd(dang_out, dang);
+}
+
+__device__ __forceinline__ uint2 ld_stream_pair(const uint2* p, uint64_t pol) { return ld_stream_v2(p, pol); }
+
+__device__ __forceinline__ void red_v4(float* p, float4 v) {
+    asm volatile("red.global.add.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+                 : "memory");
+}
+
+// Phase 2.  items[i] = (bin, first pair, end pair) relative to the bin start;
+// the bin's filled length cur[b] clips the end.
+template <int T>
+__global__ void __launch_bounds__(T, 1)
+pr_apply_kernel(const PbParams pb, const uint4* __restrict__ items, uint32_t n_items, uint32_t* work_ctr, float* acc) {
+    extern __shared__ uint4 dyn_smem[];
+    float* sacc = reinterpret_cast<float*>(dyn_smem);
+    __shared__ uint32_t s_item;
+    const int tid = threadIdx.x;
+    const uint64_t pol = policy_evict_first();
+    const uint32_t bw = 1u << pb.geo.fine_shift;
+    constexpr int U = 4;
+    for (;;) {
+        if (tid == 0) s_item = atomicAdd(work_ctr, 1u);
+        __syncthreads();
+        const uint32_t it = s_item;
+        __syncthreads();
+        if (it >= n_items) break;
+        const uint4 item = __ldg(items + it);
+        const uint32_t b = item.x;
+        const uint32_t filled = __ldg(pb.cur + b);
+        const uint32_t lo = item.y, hi = min(item.z, filled);
+        if (lo >= hi) continue;                                // CTA-uniform
+        const uint2* pr = pb.pairs + __ldg(pb.boff + b);
+        if (b < pb.geo.nfine) {
+            const uint32_t base = pb.geo.hot + (b << pb.geo.fine_shift);
+            for (uint32_t i = tid; i < bw; i += T) sacc[i] = 0.f;
+            __syncthreads();
+            for (uint32_t i0 = lo + tid; i0 < hi; i0 += T * U) {
+                uint2 e[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (i0 + u * T < hi) e[u] = ld_stream_pair(pr + i0 + u * T, pol);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (i0 + u * T < hi) atomicAdd(sacc + (e[u].x - base), __uint_as_float(e[u].y));
+            }
+            __syncthreads();
+            const float4* s4 = reinterpret_cast<const float4*>(sacc);
+            for (uint32_t j = tid; j < bw / 4; j += T) {
+                const float4 v = s4[j];
+                if (v.x == 0.f && v.y == 0.f && v.z == 0.f && v.w == 0.f) continue;
+                const uint64_t g = (uint64_t)base + 4 * j;
+                if (g + 4 <= pb.geo.n) {
+                    red_v4(acc + g, v);
+                } else {
+                    const float a[4] = {v.x, v.y, v.z, v.w};
+                    for (int k = 0; k < 4; ++k)
+                        if (g + k < pb.geo.n && a[k] != 0.f) atomicAdd(acc + g + k, a[k]);
+                }
+            }
+            __syncthreads();                                   // sacc is zeroed by the next item
+        } else {
+            for (uint32_t i0 = lo + tid; i0 < hi; i0 += T * U) {
+                uint2 e[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (i0 + u * T < hi) e[u] = ld_stream_pair(pr + i0 + u * T, pol);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (i0 + u * T < hi) atomicAdd(acc + e[u].x, __uint_as_float(e[u].y));
+            }
+        }
+    }
+}
+
 enum { kBufX = 20, kBufAcc, kBufDang, kBufPrCtr, kBufRouteSend, kBufRouteRecv, kBufRouteHot, kBufRouteHotIn,
-       kBufRouteCnt, kBufRouteList };
+       kBufRouteCnt, kBufRouteList, kBufPbPairs = 90, kBufPbMeta, kBufPbItems, kBufPbCount };
+
+inline size_t pb_bin_smem() { return (size_t)kPbHot * 4 + sizeof(PbSmem); }
+
+inline uint32_t env_u32(const char* name, uint32_t dflt) {
+    const char* v = getenv(name);
+    return v ? (uint32_t)atol(v) : dflt;
+}
+
+// Bin geometry, pair counts (once per graph and geometry, one counting sweep
+// over this rank's resident pages), bin offsets and phase-2 work items.
+// *ok = false when the pairs do not fit the u32 offsets (caller keeps the
+// plain scatter).
+int pb_plan(Context* c, const Graph* g, cudaStream_t s, PbParams& pb, uint4** d_items, uint32_t* n_items, bool* ok) {
+    const uint64_t n = g->n;
+    PbGeom& geo = pb.geo;
+    uint32_t hot = std::min<uint32_t>(env_u32("GTS_PB_HOT", kPbHot), kPbHot) & ~3u;
+    if ((uint64_t)hot > n) hot = (uint32_t)((n + 3) & ~3ull);
+    geo.hot = hot;
+    geo.fine_shift = std::max<uint32_t>(2, std::min<uint32_t>(env_u32("GTS_PB_FINE_SHIFT", kPbFineShiftMax), kPbFineShiftMax));
+    const uint64_t rest = n > hot ? n - hot : 0;
+    const uint64_t bw = 1ull << geo.fine_shift;
+    geo.nfine = (uint32_t)std::min<uint64_t>((rest + bw - 1) / bw, std::min<uint32_t>(env_u32("GTS_PB_NFINE", 512), kPbMaxBins / 2));
+    geo.fine_end = hot + ((uint64_t)geo.nfine << geo.fine_shift);
+    const uint64_t rest2 = n > geo.fine_end ? n - geo.fine_end : 0;
+    uint32_t cs = env_u32("GTS_PB_COARSE_SHIFT", 21);
+    while (cs < 40 && (rest2 >> cs) + 1 > kPbMaxBins - geo.nfine) ++cs;
+    geo.coarse_shift = cs;
+    const uint32_t ncoarse = (uint32_t)((rest2 + (1ull << cs) - 1) >> cs);
+    geo.nbins = geo.nfine + ncoarse;
+    geo.n = n;
+    DevGraph& dg = c->dg;
+    const uint64_t key = (g->uid << 24) ^ ((uint64_t)hot << 8) ^ ((uint64_t)geo.fine_shift << 40) ^
+                         ((uint64_t)geo.nfine << 44) ^ ((uint64_t)cs << 56) ^ 1;
+    uint32_t* meta;   // boff[kPbMaxBins] | cur[kPbMaxBins]
+    GTS_TRY(c->buf(kBufPbMeta, 2 * kPbMaxBins * 4, (void**)&meta));
+    pb.boff = meta;
+    pb.cur = meta + kPbMaxBins;
+    PageSet ps;
+    ps.base = dg.pages;
+    ps.list = dg.all_local ? nullptr : dg.local_list;
+    ps.loc = dg.loc;
+    ps.d_count = nullptr;
+    ps.count = dg.n_local;
+    ps.page_bytes = g->page_bytes;
+    ps.mode = dg.all_local ? kAddrByPid : kAddrByLoc;
+    ps.entry_encoding = g->entry_encoding;
+    ps.rvt_start = dg.rvt_start;
+    const size_t smem = pb_bin_smem();
+    static bool attr = false;
+    if (!attr) {
+        for (const void* k : {(const void*)pr_bin_kernel<false, false>, (const void*)pr_bin_kernel<true, false>,
+                              (const void*)pr_bin_kernel<false, true>, (const void*)pr_bin_kernel<true, true>})
+            GTS_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        GTS_CUDA(cudaFuncSetAttribute((const void*)pr_apply_kernel<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      4 << kPbFineShiftMax));
+        attr = true;
+    }
+    if (dg.pb_key != key) {
+        unsigned long long* cnt;
+        uint32_t* ctr;
+        GTS_TRY(c->buf(kBufPbCount, kPbMaxBins * 8 + 8, (void**)&cnt));
+        ctr = reinterpret_cast<uint32_t*>(cnt + kPbMaxBins);
+        GTS_CUDA(cudaMemsetAsync(cnt, 0, kPbMaxBins * 8 + 8, s));
+        PbParams pc = pb;
+        pc.count = cnt;
+        const float dz = 0.f;
+        const float* xz = nullptr;
+        float* az = nullptr;
+        double* dd = nullptr;
+        const void* kc = g->weighted ? (const void*)pr_bin_kernel<true, true> : (const void*)pr_bin_kernel<false, true>;
+        void* a[] = {(void*)&ps, (void*)&xz, (void*)&az, (void*)&dz, (void*)&dd, (void*)&ctr, (void*)&pc};
+        GTS_CUDA(cudaLaunchKernel(kc, dim3(c->num_sms * kPbBlocks), dim3(kPbThreads), a, smem, s));
+        GTS_CUDA(cudaGetLastError());
+        dg.pb_count.assign(kPbMaxBins, 0);
+        GTS_CUDA(cudaMemcpyAsync(dg.pb_count.data(), cnt, kPbMaxBins * 8, cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+        dg.pb_key = key;
+    }
+    std::vector<uint32_t> boff(kPbMaxBins, 0);
+    uint64_t tot = 0;
+    for (uint32_t b = 0; b < geo.nbins; ++b) {
+        boff[b] = (uint32_t)tot;
+        tot += dg.pb_count[b];
+        if (tot >= (1ull << 32)) {
+            *ok = false;
+            return GTS_OK;
+        }
+    }
+    const uint32_t chunk = std::max<uint32_t>(1024, env_u32("GTS_PB_CHUNK", 1u << 17));
+    std::vector<uint4> items;
+    for (uint32_t b = 0; b < geo.nbins; ++b)
+        for (uint64_t lo = 0; lo < dg.pb_count[b]; lo += chunk)
+            items.push_back(make_uint4(b, (uint32_t)lo, (uint32_t)std::min<uint64_t>(lo + chunk, dg.pb_count[b]), 0));
+    GTS_TRY(c->buf(kBufPbPairs, std::max<uint64_t>(tot, 1) * 8, (void**)&pb.pairs));
+    GTS_TRY(c->buf(kBufPbItems, std::max<size_t>(items.size(), 1) * sizeof(uint4), (void**)d_items));
+    GTS_CUDA(cudaMemcpyAsync(meta, boff.data(), kPbMaxBins * 4, cudaMemcpyHostToDevice, s));
+    if (!items.empty())
+        GTS_CUDA(cudaMemcpyAsync(*d_items, items.data(), items.size() * sizeof(uint4), cudaMemcpyHostToDevice, s));
+    GTS_CUDA(cudaStreamSynchronize(s));        // host vectors go out of scope
+    *n_items = (uint32_t)items.size();
+    *ok = true;
+    return GTS_OK;
+}
 
 }  // namespace gts
 
@@ -521,6 +1186,10 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     const char* pbig = getenv("GTS_PR_BIG");
     const bool big = (g->ordered || route) && (!pbig || atoi(pbig) > 0);
     const int mode = route ? kRoute : (g->ordered ? kDense : kHash);
+    // warp-window page walk (record-start masks instead of a binary search per 16 bytes)
+    // (measured on RMAT-27: 12.48 vs 12.24 ms for the tile walk, so opt-in: GTS_PR_WW=1)
+    const char* wwe = getenv("GTS_PR_WW");
+    const bool ww = mode == kDense && big && wwe && atoi(wwe) > 0;
     const void* kern;
     size_t dyn;
     int threads;
@@ -554,6 +1223,12 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         dyn = pr_dyn_smem<kDense, kHotDense>();
         threads = kThreads;
         n_hot = (uint32_t)std::min<uint64_t>(n, kHotDense);
+    } else if (ww) {
+        kern = g->weighted ? (const void*)pr_scatter_ww_kernel<true, 1024, 1, kHotDenseBig>
+                           : (const void*)pr_scatter_ww_kernel<false, 1024, 1, kHotDenseBig>;
+        dyn = pr_dyn_smem<kDense, kHotDenseBig>();
+        threads = 1024;
+        n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
     } else {
         kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, 1024, 1, kHotDenseBig>
                            : (const void*)pr_scatter_kernel<false, kDense, 1024, 1, kHotDenseBig>;
@@ -569,7 +1244,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     // device's persisting-L2 limit); GTS_L2_PERSIST=<MiB> overrides, 0 disables.
     bool persist = false;
     const char* pe = getenv("GTS_L2_PERSIST");
-    if (g->ordered && !route && (!pe || atol(pe) > 0)) {
+    const char* pbe = getenv("GTS_PR_BINNED");
+    bool binned = g->ordered && !streamed && !route && !micro && pbe && atoi(pbe) > 0;
+    if (g->ordered && !route && !binned && (!pe || atol(pe) > 0)) {
         size_t want = (size_t)(pe ? atol(pe) : 96) << 20;
         want = std::min<size_t>(want, c->persist_max);
         want = std::min<size_t>(want, n * 4);
@@ -604,8 +1281,10 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
         PageSet p2 = ps;
         p2.hybrid_deg = hybrid_deg;
-        void* args[] = {(void*)&p2, (void*)&x, (void*)&acc, (void*)&hk, (void*)&dmp, (void*)&D,
-                        (void*)&ctr, (void*)&n_hot, (void*)&rp};
+        void* args_full[] = {(void*)&p2, (void*)&x, (void*)&acc, (void*)&hk, (void*)&dmp, (void*)&D,
+                             (void*)&ctr, (void*)&n_hot, (void*)&rp};
+        void* args_ww[] = {(void*)&p2, (void*)&x, (void*)&acc, (void*)&dmp, (void*)&D, (void*)&ctr, (void*)&n_hot};
+        void** args = ww && !micro ? args_ww : args_full;
         cudaLaunchConfig_t lc;
         std::memset(&lc, 0, sizeof(lc));
         lc.gridDim = dim3(std::min(grid, cap));
@@ -620,13 +1299,42 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     };
     RouteParams rp0;
     std::memset(&rp0, 0, sizeof(rp0));
+    // binned scatter (section 6b of DESIGN.md): degree-ordered, resident, not routed
+    PbParams pb;
+    std::memset(&pb, 0, sizeof(pb));
+    uint4* d_items = nullptr;
+    uint32_t n_items = 0;
+    if (binned) {
+        GTS_TRY(pb_plan(c, g, s, pb, &d_items, &n_items, &binned));
+        if (binned) GTS_TRY(c->buf(kBufPrCtr, 8, (void**)&ctr));
+    }
+    auto binned_scatter = [&](const PageSet& ps, double* D) -> int {
+        GTS_CUDA(cudaMemsetAsync(ctr, 0, 8, s));
+        GTS_CUDA(cudaMemsetAsync(pb.cur, 0, (size_t)pb.geo.nbins * 4, s));
+        std::pair<cudaEvent_t, cudaEvent_t> e2;
+        if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
+        const void* k1 = g->weighted ? (const void*)pr_bin_kernel<true, false> : (const void*)pr_bin_kernel<false, false>;
+        void* a1[] = {(void*)&ps, (void*)&x, (void*)&acc, (void*)&dmp, (void*)&D, (void*)&ctr, (void*)&pb};
+        GTS_CUDA(cudaLaunchKernel(k1, dim3(c->num_sms * kPbBlocks), dim3(kPbThreads), a1, pb_bin_smem(), s));
+        uint32_t* ctr2 = ctr + 1;
+        void* a2[] = {(void*)&pb, (void*)&d_items, (void*)&n_items, (void*)&ctr2, (void*)&acc};
+        GTS_CUDA(cudaLaunchKernel((const void*)pr_apply_kernel<1024>, dim3(c->num_sms), dim3(1024), a2,
+                                  (size_t)4 << pb.geo.fine_shift, s));
+        if (timing) cudaEventRecord(e2.second, s);
+        GTS_CUDA(cudaGetLastError());
+        ++main_launches;
+        ++launches;
+        return GTS_OK;
+    };
     if (!route) {
         const uint32_t* d_list = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
         for (uint32_t it = 0; it < iters; ++it) {
             double* D = dang + (it & 1);
             std::pair<cudaEvent_t, cudaEvent_t> ev;
             GTS_TRY(sweep_pages(c, g, rc, streamed, &c->dg.h_local_list, d_list, c->dg.n_local, nullptr,
-                                [&](const PageSet& ps, int cap) -> int { return scatter(ps, cap, D, rp0); }, &ss));
+                                [&](const PageSet& ps, int cap) -> int {
+                                    return binned ? binned_scatter(ps, D) : scatter(ps, cap, D, rp0);
+                                }, &ss));
             if (c->world > 1) {         // Strategy-P: every replica receives the full sum
                 if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
                 GTS_NCCL(ncclGroupStart());

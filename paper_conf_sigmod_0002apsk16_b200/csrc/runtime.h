@@ -74,6 +74,9 @@ struct DevGraph {
     std::vector<uint32_t> h_local_list;
     std::vector<int32_t> h_owner;
     uint64_t vlo = 0, vhi = 0;         // Strategy-S WA range of this rank
+    // binned PageRank scatter: pairs per bin of this rank's pages, for the geometry pb_key
+    std::vector<unsigned long long> pb_count;
+    uint64_t pb_key = 0;
     std::vector<uint64_t> h_vrange;    // all ranks' WA ranges (world + 1)
 };
 

@@ -167,12 +167,14 @@ def test_pagerank_tolerance(G, ctx, name):
 
 
 @pytest.mark.parametrize("k", [1_300_000, 4_600_000])
-def test_pagerank_in_star_hub(G, ctx, k):
-    """Hub stress pin: k leaves -> dangling hub; closed-form recurrence in fp64."""
+@pytest.mark.parametrize("order", [False, True])
+def test_pagerank_in_star_hub(G, ctx, k, order):
+    """Hub stress pin: k leaves -> dangling hub; closed-form recurrence in fp64.
+    order=True runs the degree-ordered binned scatter (hub in the shared-memory hot set)."""
     n = k + 1
     row_ptr = np.concatenate([[0, 0], np.arange(1, k + 1)]).astype(np.uint64)
     col = np.zeros(k, np.uint32)
-    gr = G.gts_build_pages(row_ptr, col)
+    gr = G.gts_build_pages(row_ptr, col, order=order)
     got, _ = G.gts_pagerank(ctx, gr, 10, 0.85)
     d = 0.85
     leaf = eta = 1.0 / n
@@ -281,16 +283,51 @@ def test_degree_ordered_device_outputs(G, ctx):
 
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "instar", "multi"])
-@pytest.mark.parametrize("mode", ["persist", "nopersist"])
+@pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow"])
 def test_pagerank_ordered_variants(G, ctx, name, mode, monkeypatch):
-    """Degree-ordered PageRank with and without the L2 persistence window (GTS_L2_PERSIST=0)."""
+    """Degree-ordered PageRank with and without the L2 persistence window (GTS_L2_PERSIST=0),
+    and with the warp-window walk (record-start masks) instead of the tile walk."""
     if mode == "nopersist":
         monkeypatch.setenv("GTS_L2_PERSIST", "0")
+    if mode == "warpwindow":
+        monkeypatch.setenv("GTS_PR_WW", "1")
     g, pb = graph(name)
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
     for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3)):
         got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, **kw)
         _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, mode, kw))
+
+
+# Binned (propagation-blocking) scatter geometries (DESIGN.md 6b): hot set,
+# fine-bin width, fine-bin count, coarse-bin width, phase-2 chunk.  The small
+# geometries push RMAT-16 / in-star edges through hundreds of fine and coarse
+# bins and multi-chunk items; "off" is the plain red.add scatter.
+PB_GEOMS = {
+    "default": dict(GTS_PR_BINNED="1"),
+    "small": dict(GTS_PR_BINNED="1", GTS_PB_HOT="64", GTS_PB_FINE_SHIFT="6", GTS_PB_NFINE="100", GTS_PB_COARSE_SHIFT="9",
+                  GTS_PB_CHUNK="1024"),
+    "hubonly": dict(GTS_PR_BINNED="1", GTS_PB_HOT="4", GTS_PB_FINE_SHIFT="8", GTS_PB_CHUNK="1024"),
+    "coarse_only": dict(GTS_PR_BINNED="1", GTS_PB_HOT="128", GTS_PB_NFINE="0", GTS_PB_COARSE_SHIFT="4"),
+    "fine_max": dict(GTS_PR_BINNED="1", GTS_PB_HOT="4", GTS_PB_FINE_SHIFT="2", GTS_PB_NFINE="512", GTS_PB_COARSE_SHIFT="2"),
+    "off": dict(GTS_PR_BINNED="0"),
+    "warpwindow": dict(GTS_PR_BINNED="0", GTS_PR_WW="1"),
+}
+
+
+@pytest.mark.parametrize("name", ["rmat16_4k", "rmat16_1m", "rmat20", "twitter20", "instar", "multi", "fig1", "path"])
+@pytest.mark.parametrize("geom", list(PB_GEOMS))
+def test_pagerank_binned_geometries(G, ctx, name, geom, monkeypatch):
+    for k, v in PB_GEOMS[geom].items():
+        monkeypatch.setenv(k, v)
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+    for mode in (G.GTS_DANGLING_UNIFORM, G.GTS_DANGLING_DROP):
+        got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, mode)
+        _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85, dangling=mode), g, (name, geom, mode))
+    if name == "rmat16_4k":               # weighted pages skip the weight words
+        grw = G.gts_build_pages(g.row_ptr, g.col, inputs.edge_weights(g), page_bytes=2 * pb, order=True)
+        got, _ = G.gts_pagerank(ctx, grw, 10, 0.85)
+        _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, geom, "weighted"))
 
 
 # ------------------------------------------------- streamed + LRU page cache ---
