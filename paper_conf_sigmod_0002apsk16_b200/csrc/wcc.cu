@@ -12,6 +12,7 @@
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <cstdlib>
 #include <cstring>
 
 #include "expand.cuh"
@@ -55,33 +56,105 @@ __device__ __forceinline__ bool uf_hook(uint32_t* parent, uint32_t a, uint32_t b
     return hooked;
 }
 
+// Per edge u -> v: the payload is parent[u] read once per vertex per tile; if
+// parent[v] equals it the endpoints already share a tree (trees only ever
+// merge, so equal pointers, even stale ones, mean one component) and the edge
+// costs a single gather; otherwise a full hook.  After the sampling pass below
+// most vertices point straight at their component's root, so most edges of
+// the giant component end here.
+//
+// Giant filter: after the sampling pass, gbm marks the vertices whose parent
+// was the root r* of vertex 0's tree (on degree-ordered pages the giant
+// component); an edge whose source points at r* and whose destination bit is
+// set is skipped on a bitmap test (n/8 bytes, L1/L2-resident like BFS's
+// visited bitmap) without touching parent[].
 template <bool W>
 struct WccOp {
     static constexpr bool kReadWeights = false;
     static constexpr bool kWeighted = W;
     uint32_t* parent;
     bool changed;
+    const uint32_t* gbm;      // nullptr: no giant filter
+    uint32_t rstar;
     __device__ const uint32_t* frontier() const { return nullptr; }
     __device__ bool select(uint32_t) { return true; }
-    __device__ uint32_t payload(uint32_t v, uint32_t) { return v; }
+    __device__ uint32_t payload(uint32_t v, uint32_t) { return __ldcg(parent + v); }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t, uint32_t& pl) {
-        pl = vid;
+        pl = __ldcg(parent + vid);
         return true;
     }
-    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*,
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t* pl,
                                           const uint32_t* src, const bool* valid) {
+        bool live[kEdgesPerThread];
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            live[q] = valid[q];
+            if (gbm && valid[q] && pl[q] == rstar) live[q] = !((__ldg(gbm + (dst[q] >> 5)) >> (dst[q] & 31)) & 1u);
+        }
+        uint32_t pv[kEdgesPerThread];
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) pv[q] = live[q] ? __ldcg(parent + dst[q]) : 0u;
 #pragma unroll
         for (int q = 0; q < kEdgesPerThread; ++q)
-            if (valid[q] && src[q] != dst[q] && uf_hook(parent, src[q], dst[q])) changed = true;
+            if (live[q] && pv[q] != pl[q] && src[q] != dst[q] && uf_hook(parent, src[q], dst[q])) changed = true;
     }
     __device__ void end_page() {}
 };
 
+// Sampling pass (Afforest-style, Sutton et al. 2018, adapted to out-edge
+// pages): every vertex hooks only its first `ks` out-neighbours (an LP vertex:
+// from its first chunk).  Rows are sorted by destination, so on degree-ordered
+// pages these are the vertex's highest in-degree neighbours and the giant
+// component's trees form almost at once.  The full sweep that follows still
+// visits every edge (the result is exact); the sample only makes its edges
+// cheap (one gather instead of two finds).
+__global__ void __launch_bounds__(kThreads, 2)
+wcc_sample_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t ks) {
+    __shared__ uint32_t s_item;
+    const int tid = threadIdx.x;
+    const uint64_t pol = policy_evict_first();
+    for (;;) {
+        if (tid == 0) s_item = atomicAdd(work_ctr, 1u);
+        __syncthreads();
+        const uint32_t it = s_item;
+        __syncthreads();
+        if (it >= ps.count) break;
+        uint32_t pid;
+        const uint8_t* data;
+        page_at(ps, it, pid, data);
+        const uint8_t* end = data + ps.page_bytes;
+        const uint32_t kind = ld32(end - 4);
+        const uint32_t* words = reinterpret_cast<const uint32_t*>(data);
+        if (kind == GTS_PAGE_LP) {
+            const uint32_t vid = ld32(end - kLpFooter - kSlotBytes);
+            const uint32_t chunk = ld32(end - 12);
+            const uint32_t len = ld32(data);
+            if (chunk == 0 && (uint32_t)tid < min(ks, len)) {
+                const uint32_t v = decode_entry(ps, ld_stream_u32(words + 1 + tid, pol));
+                if (v != vid) uf_hook(parent, vid, v);
+            }
+        } else {
+            const uint32_t nslots = ld32(end - 8);
+            const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
+            for (uint32_t u = tid; u < nslots; u += kThreads) {
+                const uint32_t off = ld_stream_u32(end - kSpFooter - kSlotBytes * (uint64_t)(u + 1) + 4, pol) >> 2;
+                const uint32_t deg = ld_stream_u32(words + off, pol);
+                const uint32_t kk = min(ks, deg);
+                for (uint32_t k = 0; k < kk; ++k) {
+                    const uint32_t v = decode_entry(ps, ld_stream_u32(words + off + 1 + k, pol));
+                    if (v != start + u) uf_hook(parent, start + u, v);
+                }
+            }
+        }
+    }
+}
+
 template <bool W>
 __global__ void __launch_bounds__(kThreads, 2)
-wcc_sweep_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t* changed) {
+wcc_sweep_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t* changed, const uint32_t* gbm,
+                 const uint32_t* rstar) {
     __shared__ TileSmem sm;
-    WccOp<W> op{parent, false};
+    WccOp<W> op{parent, false, gbm, gbm ? __ldg(rstar) : 0u};
     expand_pages(ps, op, sm, work_ctr);
     if (__syncthreads_or(op.changed) && threadIdx.x == 0) *changed = 1u;
 }
@@ -89,6 +162,19 @@ wcc_sweep_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t* cha
 __global__ void wcc_init_kernel(uint32_t* label, uint64_t n) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) label[i] = (uint32_t)i;
+}
+
+// gbm bit v = (parent[v] == parent[0]); *rstar = parent[0] (run after a finalize pass)
+__global__ void wcc_giant_kernel(const uint32_t* parent, uint64_t n, uint32_t* gbm, uint32_t* rstar) {
+    const uint32_t r = __ldcg(parent);
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t nw = (n + 31) / 32 * 32;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += stride) {
+        const bool in = i < n && __ldcg(parent + i) == r;
+        const uint32_t b = __ballot_sync(0xFFFFFFFFu, in);
+        if ((threadIdx.x & 31) == 0) gbm[i >> 5] = b;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) *rstar = r;
 }
 
 // every vertex points at its root (the component's minimum VID)
@@ -101,7 +187,7 @@ __global__ void wcc_finalize_kernel(uint32_t* parent, uint64_t n) {
     }
 }
 
-enum { kBufLabel = 30, kBufWccCtr };
+enum { kBufLabel = 30, kBufWccCtr, kBufWccGiant };
 
 }  // namespace gts
 
@@ -134,6 +220,35 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     uint32_t* hs = (uint32_t*)c->h_small;
     SweepStats ss;
     const uint32_t* d_list = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
+    // sampling pass + compression (resident pages only: streamed, it would cost a
+    // whole extra transfer of the topology); GTS_WCC_SAMPLE=k neighbours, 0 = off
+    const char* se = getenv("GTS_WCC_SAMPLE");
+    const uint32_t ks = se ? (uint32_t)atol(se) : 1u;
+    uint32_t* gbm = nullptr;   // giant filter bitmap (+ r* after it)
+    if (!streamed && ks > 0) {
+        std::pair<cudaEvent_t, cudaEvent_t> ev;
+        if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+        GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
+        PageSet ps;
+        ps.base = c->dg.pages;
+        ps.list = d_list;
+        ps.loc = c->dg.loc;
+        ps.d_count = nullptr;
+        ps.count = c->dg.n_local;
+        ps.page_bytes = g->page_bytes;
+        ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
+        ps.entry_encoding = g->entry_encoding;
+        ps.rvt_start = c->dg.rvt_start;
+        int sg = 0;
+        GTS_TRY(sms_grid(c, (const void*)wcc_sample_kernel, kThreads, 0, &sg));
+        wcc_sample_kernel<<<sg, kThreads, 0, s>>>(ps, label, ctr, ks);
+        wcc_finalize_kernel<<<eg, 256, 0, s>>>(label, n);
+        GTS_TRY(c->buf(kBufWccGiant, (n + 31) / 32 * 4 + 16, (void**)&gbm));
+        wcc_giant_kernel<<<eg, 256, 0, s>>>(label, n, gbm, gbm + (n + 31) / 32);
+        if (timing) cudaEventRecord(ev.second, s);
+        GTS_CUDA(cudaGetLastError());
+        launches += 2;
+    }
     for (;;) {
         GTS_CUDA(cudaMemsetAsync(ctr + 1, 0, 4, s));
         std::pair<cudaEvent_t, cudaEvent_t> ev;
@@ -142,7 +257,8 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
                                 GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
                                 std::pair<cudaEvent_t, cudaEvent_t> e2;
                                 if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
-                                sweep_k<<<std::min(grid, cap), kThreads, 0, s>>>(ps, label, ctr, ctr + 1);
+                                sweep_k<<<std::min(grid, cap), kThreads, 0, s>>>(ps, label, ctr, ctr + 1, gbm,
+                                                                                  gbm ? gbm + (n + 31) / 32 : nullptr);
                                 if (timing) cudaEventRecord(e2.second, s);
                                 GTS_CUDA(cudaGetLastError());
                                 ++main_launches;

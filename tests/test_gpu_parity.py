@@ -330,6 +330,23 @@ def test_pagerank_binned_geometries(G, ctx, name, geom, monkeypatch):
         _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, geom, "weighted"))
 
 
+@pytest.mark.parametrize("name", ["fig1", "multi", "path", "cycle", "outstar", "instar", "rand", "rmat16_4k",
+                                  "rmat16_256", "rmat20", "twitter20"])
+@pytest.mark.parametrize("ks", ["0", "1", "2", "8"])
+@pytest.mark.parametrize("order", [False, True])
+def test_wcc_sampling(G, ctx, name, ks, order, monkeypatch):
+    """WCC with the sampling pre-pass hooking the first ks out-neighbours (0 = off)."""
+    monkeypatch.setenv("GTS_WCC_SAMPLE", ks)
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
+    got, _ = G.gts_wcc(ctx, gr)
+    assert np.array_equal(got, oracle.wcc(g.row_ptr, g.col)), (name, ks, order)
+    if name == "rmat16_4k":
+        grw = G.gts_build_pages(g.row_ptr, g.col, inputs.edge_weights(g), page_bytes=2 * pb, order=order)
+        got, _ = G.gts_wcc(ctx, grw)
+        assert np.array_equal(got, oracle.wcc(g.row_ptr, g.col)), (name, ks, order, "weighted")
+
+
 # ------------------------------------------------- streamed + LRU page cache ---
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "path", "bintree"])
