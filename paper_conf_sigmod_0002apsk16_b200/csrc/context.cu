@@ -384,6 +384,26 @@ int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_
     return copy_out(c, dst, out, n * 4, out_location);
 }
 
+int persist_window(Context* c, cudaStream_t s, void* p, size_t bytes) {
+    cudaStreamAttrValue at;
+    std::memset(&at, 0, sizeof(at));
+    if (p && bytes) {
+        const size_t want = std::min(bytes, c->persist_max);
+        if (want == 0) return GTS_OK;
+        if (c->persist_limit != c->persist_max) {   // device-wide set-aside: the maximum, set once
+            GTS_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, c->persist_max));
+            c->persist_limit = c->persist_max;
+        }
+        at.accessPolicyWindow.base_ptr = p;
+        at.accessPolicyWindow.num_bytes = std::min(want, c->window_max);
+        at.accessPolicyWindow.hitRatio = 1.0f;
+        at.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        at.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    }
+    GTS_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &at));
+    return GTS_OK;
+}
+
 int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid) {
     int per_sm = 0;
     GTS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem));

@@ -100,6 +100,35 @@ __device__ __forceinline__ void tile_scan(bool sel, uint32_t deg, uint32_t& pos,
     nf = sm.wcnt[kWarps - 1];
 }
 
+// ---- warp-window walk helpers ----
+// A 128-word window of a tile's record region is one 16-byte load per lane;
+// the owner of word i is j0 + #(record starts at or before i).
+struct WinMask {
+    uint32_t m[4];
+};
+
+// record starts in [base, base + 128) among off[j0 + 1 .. nv)
+__device__ __forceinline__ WinMask win_mask(const uint32_t* off, int j0, uint32_t nv, uint32_t base, int& nstarts) {
+    const int lane = threadIdx.x & 31;
+    WinMask wm{{0u, 0u, 0u, 0u}};
+    nstarts = 0;
+    for (int r = j0 + 1;; r += 32) {
+        const int j = r + lane;
+        const uint32_t o = (uint32_t)j < nv ? off[j] : 0xFFFFFFFFu;
+        const bool in = o - base < 128u && o >= base;
+        const uint32_t p = o - base;
+        const uint32_t bit = in ? 1u << (p & 31) : 0u;
+        wm.m[0] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 0) ? bit : 0u);
+        wm.m[1] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 1) ? bit : 0u);
+        wm.m[2] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 2) ? bit : 0u);
+        wm.m[3] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 3) ? bit : 0u);
+        const uint32_t b = __ballot_sync(0xFFFFFFFFu, in);
+        nstarts += __popc(b);
+        if (b != 0xFFFFFFFFu) break;        // offsets ascend: a gap means no later start in the window
+    }
+    return wm;
+}
+
 // Op interface:
 //   static constexpr bool kReadWeights;  -- the op needs edge weights
 //   static constexpr bool kWeighted;     -- the pages carry weights (record = sz, adj[sz], w[sz])
@@ -272,6 +301,73 @@ __device__ void expand_sp_micro(const PageSet& ps, Op& op, const uint8_t* data, 
     }
 }
 
+// Dense tile by warp windows (sm.soff / sm.sel / sm.paytile of the tile are
+// published).  Same per-edge contract as the tile walk: op.edges gets the 4
+// words of one 16-byte load per call.
+template <class Op>
+__device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSmem& sm, const uint4* q4,
+                                              const uint32_t* words, uint32_t v0, uint32_t nv, uint32_t W0,
+                                              uint32_t W1, uint64_t pol) {
+    constexpr uint32_t wsh = Op::kWeighted ? 1 : 0;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t wbase = W0 & ~3u;
+    const uint32_t nwin = (W1 - wbase + 127) >> 7;
+    const uint32_t per = (nwin + kWarps - 1) / kWarps;
+    const uint32_t wa = min(nwin, warp * per), wb = min(nwin, wa + per);
+    if (wa >= wb) return;
+    const uint32_t base0 = wbase + (wa << 7);
+    int lo = -1, hi = (int)nv;                      // soff[lo] < base0 <= soff[hi]
+    while (hi - lo > 1) {
+        const int mid = (lo + hi) >> 1;
+        if (sm.soff[mid] < base0) lo = mid; else hi = mid;
+    }
+    int j0 = lo;
+    for (uint32_t wi = wa; wi < wb; wi += kDenseUnroll) {
+        uint4 vv[kDenseUnroll];
+#pragma unroll
+        for (int u = 0; u < kDenseUnroll; ++u) {
+            const uint32_t q = ((wbase + ((wi + u) << 7)) >> 2) + lane;
+            vv[u] = make_uint4(0u, 0u, 0u, 0u);
+            if (wi + u < wb && 4 * q < W1) vv[u] = ld_stream_v4(q4 + q, pol);
+        }
+#pragma unroll
+        for (int u = 0; u < kDenseUnroll; ++u) {
+            if (wi + u >= wb) break;
+            const uint32_t bw = wbase + ((wi + u) << 7);
+            const uint32_t q = (bw >> 2) + lane;
+            int ns;
+            const WinMask wm = win_mask(sm.soff, j0, nv, bw, ns);
+            const uint32_t mw = lane >> 3;
+            uint32_t before = 0;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) before += (uint32_t)k < mw ? __popc(wm.m[k]) : 0u;
+            const uint32_t mword = mw == 0 ? wm.m[0] : mw == 1 ? wm.m[1] : mw == 2 ? wm.m[2] : wm.m[3];
+            uint32_t dst[kEdgesPerThread], wt[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
+            bool valid[kEdgesPerThread];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const uint32_t w = 4 * q + k;
+                const uint32_t bpos = (4 * lane + k) & 31;
+                const int j = j0 + (int)(before + __popc(mword & ((2u << bpos) - 1u)));
+                bool ok = w >= W0 && w < W1 && !((mword >> bpos) & 1u);
+                uint32_t dj = 0;
+                if (ok) {
+                    const uint32_t o = sm.soff[j];
+                    dj = (sm.soff[j + 1] - o - 1) >> wsh;
+                    ok = w - o <= dj && sm.sel[j];
+                }
+                wt[k] = (Op::kReadWeights && ok) ? ld_stream_l1_u32(words + w + dj, pol) : 0u;
+                valid[k] = ok;
+                dst[k] = decode_entry(ps, word_of(vv[u], k));
+                pl[k] = ok ? sm.paytile[j] : 0u;
+                src[k] = v0 + (uint32_t)j;
+            }
+            op.edges(dst, wt, pl, src, valid);
+            j0 += ns;
+        }
+    }
+}
+
 template <class Op, int kMicro = kMicroTile>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
     const uint32_t count = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
@@ -376,6 +472,13 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 uint32_t pos, nf, excl, total;
                 tile_scan(sel, sel ? deg : 0u, pos, nf, excl, total, sm);
                 const uint32_t W0 = sm.soff[0], W1 = sm.soff[nv];
+                if (2 * total >= W1 - W0 && ps.ww) {
+                    // dense tile, warp-window walk: each warp streams a contiguous run of
+                    // 128-word windows; owners from record-start masks (no binary search)
+                    dense_tile_ww(ps, op, sm, q4, words, start + t0, nv, W0, W1, pol);
+                    __syncthreads();
+                    continue;
+                }
                 if (2 * total >= W1 - W0) {
                     // dense tile: stream the whole record region with 16-byte loads and
                     // act on the words of selected owners (hybrid micro-level, App E)

@@ -328,32 +328,6 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
 // popcount prefix, instead of a binary search per 16 bytes: the owner of word
 // i is j0 + #(record starts at or before i), j0 = the last vertex starting
 // before the window (carried from window to window).
-struct WinMask {
-    uint32_t m[4];
-};
-
-// record starts in [base, base + 128) among off[j0 + 1 .. nv)
-__device__ __forceinline__ WinMask win_mask(const uint32_t* off, int j0, uint32_t nv, uint32_t base, int& nstarts) {
-    const int lane = threadIdx.x & 31;
-    WinMask wm{{0u, 0u, 0u, 0u}};
-    nstarts = 0;
-    for (int r = j0 + 1;; r += 32) {
-        const int j = r + lane;
-        const uint32_t o = (uint32_t)j < nv ? off[j] : 0xFFFFFFFFu;
-        const bool in = o - base < 128u && o >= base;
-        const uint32_t p = o - base;
-        const uint32_t bit = in ? 1u << (p & 31) : 0u;
-        wm.m[0] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 0) ? bit : 0u);
-        wm.m[1] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 1) ? bit : 0u);
-        wm.m[2] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 2) ? bit : 0u);
-        wm.m[3] |= __reduce_or_sync(0xFFFFFFFFu, (in && (p >> 5) == 3) ? bit : 0u);
-        const uint32_t b = __ballot_sync(0xFFFFFFFFu, in);
-        nstarts += __popc(b);
-        if (b != 0xFFFFFFFFu) break;        // offsets ascend: a gap means no later start in the window
-    }
-    return wm;
-}
-
 template <bool kWeighted, int T, int kMinBlocks, uint32_t H>
 __global__ void __launch_bounds__(T, kMinBlocks)
 pr_scatter_ww_kernel(PageSet ps, const float* __restrict__ x, float* acc, float d, double* dang_out,
@@ -1247,22 +1221,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     const char* pbe = getenv("GTS_PR_BINNED");
     bool binned = g->ordered && !streamed && !route && !micro && pbe && atoi(pbe) > 0;
     if (g->ordered && !route && !binned && (!pe || atol(pe) > 0)) {
-        size_t want = (size_t)(pe ? atol(pe) : 96) << 20;
-        want = std::min<size_t>(want, c->persist_max);
-        want = std::min<size_t>(want, n * 4);
+        const size_t want = std::min<size_t>((size_t)(pe ? atol(pe) : 96) << 20, n * 4);
         if (want > 0) {
-            if (c->persist_limit != want) {           // set once per context (a device-wide limit)
-                GTS_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
-                c->persist_limit = want;
-            }
-            cudaStreamAttrValue at;
-            std::memset(&at, 0, sizeof(at));
-            at.accessPolicyWindow.base_ptr = acc;
-            at.accessPolicyWindow.num_bytes = std::min<size_t>(want, c->window_max);
-            at.accessPolicyWindow.hitRatio = 1.0f;
-            at.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-            at.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-            GTS_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &at));
+            GTS_TRY(persist_window(c, s, acc, want));
             persist = true;
         }
     }
@@ -1557,13 +1518,11 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     }
     launches += main_launches;
     if (persist) {
-        cudaStreamAttrValue at;
-        std::memset(&at, 0, sizeof(at));
-        at.accessPolicyWindow.num_bytes = 0;
-        GTS_CUDA(cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &at));
-        // The lines marked persisting stay so until the next PageRank call reuses
-        // them or the context is freed: an explicit cudaCtxResetPersistingL2Cache
-        // here measured +20 ms on the following call (GTS_L2_RESET=1 forces it).
+        GTS_TRY(persist_window(c, s, nullptr, 0));
+        // The lines marked persisting stay so until a later call's window (BFS
+        // visited, SSSP dist, WCC parents, PageRank acc) replaces them or the
+        // context is freed: an explicit cudaCtxResetPersistingL2Cache here
+        // measured +20 ms on the following call (GTS_L2_RESET=1 forces it).
         const char* rs = getenv("GTS_L2_RESET");
         if (rs && atoi(rs) != 0) GTS_CUDA(cudaCtxResetPersistingL2Cache());
     }

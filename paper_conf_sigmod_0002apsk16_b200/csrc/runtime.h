@@ -5,6 +5,7 @@
 #include <nccl.h>
 
 #include <chrono>
+#include <cstdlib>
 #include <utility>
 #include <vector>
 
@@ -52,6 +53,7 @@ struct PageSet {
     uint32_t entry_encoding;
     const uint32_t* rvt_start; // START_VID per page (PID16 decode)
     uint32_t hybrid_deg = 8;   // GTS_MICRO_HYBRID: vertex-centric below this many edges per vertex (R24)
+    uint32_t ww = 0;           // dense tiles by warp windows (expand.cuh dense_tile_ww)
 };
 
 // Device copy of a graph for one rank.
@@ -134,6 +136,9 @@ int copy_out(Context* c, const void* dsrc, void* dst, size_t bytes, uint32_t out
 int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_t out_location, bool labels);
 inline uint64_t map_src(const Graph* g, uint64_t src) { return g->ordered ? g->new_of_old[src] : src; }
 int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid);
+// access-policy window on stream s: [p, p + bytes) persisting in L2 (bytes clipped to the
+// device limits); p = nullptr clears the window
+int persist_window(Context* c, cudaStream_t s, void* p, size_t bytes);
 int pinned_register(Graph* g);
 void free_cache(PageCache& pc);
 // residency decision (GTS_RESIDENCY_AUTO: resident iff this rank's pages + attributes fit in free HBM)
@@ -142,6 +147,13 @@ bool choose_streamed(Context* c, const Graph* g, const gts_run_config& rc, uint6
 // P-strategy page ownership (h(j) = j mod N) and S ranges.
 void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t>& owner,
                std::vector<uint64_t>& vrange);
+
+// dense tiles by warp windows unless GTS_WW=0 (read per call so tests can switch it);
+// RMAT-27: SSSP 33.8 vs 36.2 ms, WCC 13.7 vs 14.2, BFS equal (profiles/r01_ww_dense.txt)
+inline uint32_t env_ww() {
+    const char* e = getenv("GTS_WW");
+    return e && atoi(e) == 0 ? 0u : 1u;
+}
 
 inline double now_s() {
     return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();

@@ -48,6 +48,7 @@ int sweep_pages(Context* c, const Graph* g, const gts_run_config& rc, bool strea
         ps.mode = d.all_local ? kAddrByPid : kAddrByLoc;
         ps.entry_encoding = g->entry_encoding;
         ps.rvt_start = d.rvt_start;
+        ps.ww = env_ww();
         GTS_TRY(launch(ps, 1 << 30));
         ss->launches++;
         return GTS_OK;
@@ -89,6 +90,7 @@ int sweep_pages(Context* c, const Graph* g, const gts_run_config& rc, bool strea
         ps.mode = kAddrByPos;
         ps.entry_encoding = g->entry_encoding;
         ps.rvt_start = d.rvt_start;
+        ps.ww = env_ww();
         GTS_TRY(launch(ps, (int)nb));
         GTS_CUDA(cudaEventRecord(c->ring_free[slot], c->stream));
         ss->h2d_bytes += (uint64_t)nb * pb;
@@ -178,6 +180,7 @@ int sweep_pages_cached(Context* c, const Graph* g, const gts_run_config& rc, con
         ps.mode = kAddrByLoc;
         ps.entry_encoding = g->entry_encoding;
         ps.rvt_start = c->dg.rvt_start;
+        ps.ww = env_ww();
         return ps;
     };
     if (!hits.empty()) {                          // overlaps the miss copies below

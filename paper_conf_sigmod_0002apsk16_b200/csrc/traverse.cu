@@ -322,6 +322,7 @@ static PageSet resident_set(Context* c, const Graph* g, const uint32_t* list, co
     ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
     ps.entry_encoding = g->entry_encoding;
     ps.rvt_start = c->dg.rvt_start;
+    ps.ww = env_ww();
     return ps;
 }
 
@@ -399,6 +400,19 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     const char* de = getenv("GTS_SSSP_DELTA");
     const uint64_t delta = de ? std::max<long>(1, atol(de)) : 0xFFFFFFFEull;
     uint32_t T = algo == kSSSP ? (uint32_t)std::min<uint64_t>(delta, 0xFFFFFFFEull) : 0xFFFFFFFEu;
+    // Persisting-L2 window on the structure every edge probes: SSSP on degree-ordered
+    // pages the dense head [0, W) of dist (the most relaxed entries), BFS the visited
+    // bitmap.  It also replaces lines an earlier PageRank call left persisting.
+    // GTS_L2_PERSIST_SSSP / GTS_L2_PERSIST_BFS = <MiB>, 0 = off.
+    bool persist = false;
+    if (!streamed && (algo == kBFS || g->ordered)) {
+        const char* pe = getenv(algo == kBFS ? "GTS_L2_PERSIST_BFS" : "GTS_L2_PERSIST_SSSP");
+        const size_t want = std::min<size_t>((size_t)(pe ? atol(pe) : 96) << 20, algo == kBFS ? words * 4 : n * 4);
+        if (want > 0) {
+            GTS_TRY(persist_window(c, s, algo == kBFS ? (void*)visited : (void*)value, want));
+            persist = true;
+        }
+    }
     for (uint32_t L = 0;; ++L) {
         auto launch = [&](const PageSet& ps, int cap) -> int {
                                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
@@ -475,6 +489,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         std::swap(cur, next);
         GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
     }
+    if (persist) GTS_TRY(persist_window(c, s, nullptr, 0));
     if (algo == kSSSP && c->world > 1) {   // every rank must agree before the collective check
         GTS_NCCL(ncclAllReduce(&ctr->flag, &ctr->flag, 1, ncclUint32, ncclMax, c->comm, s));
         GTS_CUDA(cudaMemcpyAsync(&h.flag, &ctr->flag, 4, cudaMemcpyDeviceToHost, s));

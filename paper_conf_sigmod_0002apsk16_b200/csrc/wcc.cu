@@ -224,6 +224,17 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     // whole extra transfer of the topology); GTS_WCC_SAMPLE=k neighbours, 0 = off
     const char* se = getenv("GTS_WCC_SAMPLE");
     const uint32_t ks = se ? (uint32_t)atol(se) : 1u;
+    // persisting-L2 window on the head of the union-find forest (degree-ordered
+    // pages: the most probed parents); GTS_L2_PERSIST_WCC=<MiB>, 0 = off
+    bool persist = false;
+    if (!streamed && g->ordered) {
+        const char* pe = getenv("GTS_L2_PERSIST_WCC");
+        const size_t want = std::min<size_t>((size_t)(pe ? atol(pe) : 96) << 20, n * 4);
+        if (want > 0) {
+            GTS_TRY(persist_window(c, s, label, want));
+            persist = true;
+        }
+    }
     uint32_t* gbm = nullptr;   // giant filter bitmap (+ r* after it)
     if (!streamed && ks > 0) {
         std::pair<cudaEvent_t, cudaEvent_t> ev;
@@ -239,6 +250,7 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
         ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
         ps.entry_encoding = g->entry_encoding;
         ps.rvt_start = c->dg.rvt_start;
+        ps.ww = env_ww();
         int sg = 0;
         GTS_TRY(sms_grid(c, (const void*)wcc_sample_kernel, kThreads, 0, &sg));
         wcc_sample_kernel<<<sg, kThreads, 0, s>>>(ps, label, ctr, ks);
@@ -283,6 +295,7 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
         GTS_CUDA(cudaStreamSynchronize(s));
         if (hs[0] == 0) break;
     }
+    if (persist) GTS_TRY(persist_window(c, s, nullptr, 0));
     GTS_TRY(deliver(c, g, label, label_out, rc.out_location, true));
     if (st) {
         std::memset(st, 0, sizeof(*st));

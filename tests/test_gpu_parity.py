@@ -347,6 +347,25 @@ def test_wcc_sampling(G, ctx, name, ks, order, monkeypatch):
         assert np.array_equal(got, oracle.wcc(g.row_ptr, g.col)), (name, ks, order, "weighted")
 
 
+@pytest.mark.parametrize("name", ["fig1", "multi", "path", "bintree", "rand", "rmat16_4k", "rmat16_256", "rmat20",
+                                  "twitter20"])
+@pytest.mark.parametrize("order", [False, True])
+def test_tile_walk_dense_tiles(G, ctx, name, order, monkeypatch):
+    """Dense tiles by the tile walk (binary search per 16 bytes, GTS_WW=0) instead of warp windows."""
+    monkeypatch.setenv("GTS_WW", "0")
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
+    for s in _sources(g):
+        lv, _ = G.gts_bfs(ctx, gr, s)
+        assert np.array_equal(lv, oracle.bfs(g.row_ptr, g.col, s)), (name, s)
+    w = inputs.edge_weights(g)
+    grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=2 * pb, order=order)
+    d, _ = G.gts_sssp(ctx, grw, 0)
+    assert np.array_equal(d, oracle.sssp(g.row_ptr, g.col, w, 0)), name
+    lab, _ = G.gts_wcc(ctx, gr)
+    assert np.array_equal(lab, oracle.wcc(g.row_ptr, g.col)), name
+
+
 # ------------------------------------------------- streamed + LRU page cache ---
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "path", "bintree"])
