@@ -177,10 +177,9 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
         GTS_CUDA(cudaMemcpyAsync(d.hot_keys, g->hot_keys.data(), kHotSlots * 4, cudaMemcpyHostToDevice, c->stream));
         if (g->ordered) {
             GTS_TRY(pinned_register(g));
+            // old_of_new is uploaded on first use (WCC label renaming in deliver)
             GTS_CUDA(cudaMalloc(&d.new_of_old, g->n * 4));
-            GTS_CUDA(cudaMalloc(&d.old_of_new, g->n * 4));
             GTS_CUDA(cudaMemcpyAsync(d.new_of_old, g->new_of_old.data(), g->n * 4, cudaMemcpyHostToDevice, c->stream));
-            GTS_CUDA(cudaMemcpyAsync(d.old_of_new, g->old_of_new.data(), g->n * 4, cudaMemcpyHostToDevice, c->stream));
         }
         GTS_CUDA(cudaStreamSynchronize(c->stream));   // host vectors above are temporaries
     }
@@ -364,6 +363,11 @@ int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_
     const int eg = c->num_sms * 4;
     const uint32_t* src = vals;
     if (labels) {             // internal min-ID label -> min caller VID of the component
+        if (!c->dg.old_of_new) {
+            GTS_CUDA(cudaMalloc(&c->dg.old_of_new, n * 4));
+            GTS_CUDA(cudaMemcpyAsync(c->dg.old_of_new, g->old_of_new.data(), n * 4, cudaMemcpyHostToDevice,
+                                     c->stream));
+        }
         uint32_t *minorig, *tmp;
         GTS_TRY(c->buf(70, n * 4, (void**)&minorig));
         GTS_TRY(c->buf(71, n * 4, (void**)&tmp));
