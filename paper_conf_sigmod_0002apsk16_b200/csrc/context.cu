@@ -357,17 +357,23 @@ __global__ void label_map_kernel(uint32_t* tmp, const uint32_t* __restrict__ lab
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) tmp[i] = minorig[label[i]];
 }
 
+int ensure_old_of_new(Context* c, const Graph* g, const uint32_t** out) {
+    if (!c->dg.old_of_new) {
+        GTS_CUDA(cudaMalloc(&c->dg.old_of_new, g->n * 4));
+        GTS_CUDA(cudaMemcpyAsync(c->dg.old_of_new, g->old_of_new.data(), g->n * 4, cudaMemcpyHostToDevice, c->stream));
+    }
+    *out = c->dg.old_of_new;
+    return GTS_OK;
+}
+
 int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_t out_location, bool labels) {
     const uint64_t n = g->n;
     if (!g->ordered) return copy_out(c, vals, out, n * 4, out_location);
     const int eg = c->num_sms * 4;
     const uint32_t* src = vals;
     if (labels) {             // internal min-ID label -> min caller VID of the component
-        if (!c->dg.old_of_new) {
-            GTS_CUDA(cudaMalloc(&c->dg.old_of_new, n * 4));
-            GTS_CUDA(cudaMemcpyAsync(c->dg.old_of_new, g->old_of_new.data(), n * 4, cudaMemcpyHostToDevice,
-                                     c->stream));
-        }
+        const uint32_t* onew;
+        GTS_TRY(ensure_old_of_new(c, g, &onew));
         uint32_t *minorig, *tmp;
         GTS_TRY(c->buf(70, n * 4, (void**)&minorig));
         GTS_TRY(c->buf(71, n * 4, (void**)&tmp));

@@ -134,6 +134,8 @@ int copy_out(Context* c, const void* dsrc, void* dst, size_t bytes, uint32_t out
 // labels = true: the values are themselves internal VIDs (WCC) and are renamed to
 // the minimum caller VID of their component.
 int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_t out_location, bool labels);
+// device copy of old_of_new (internal ID -> caller VID), uploaded on first use
+int ensure_old_of_new(Context* c, const Graph* g, const uint32_t** out);
 inline uint64_t map_src(const Graph* g, uint64_t src) { return g->ordered ? g->new_of_old[src] : src; }
 int sms_grid(Context* c, const void* kernel, int threads, size_t smem, int* grid);
 // access-policy window on stream s: [p, p + bytes) persisting in L2 (bytes clipped to the
