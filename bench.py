@@ -123,8 +123,9 @@ def run_reference(args, rank):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / len(times),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
-            "config": {"workload": f"rmat{args.scale}_bfs (reference arm: oracle BFS on the RMAT-{scale} sample)",
-                       "sample_scale": scale, "src": 0},
+            "config": {"workload": f"rmat{args.scale}_bfs_pr_sssp_wcc", "scale": args.scale, "src": 0,
+                       "sample": f"reference arm: oracle BFS (the metric's algorithm) on the RMAT-{scale} sample",
+                       "sample_scale": scale},
             "cpu_baseline": {"value": gteps, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                              "sample": f"oracle BFS from vertex 0 on RMAT-{scale} (same generator as RMAT-{args.scale},"
                                        f" 1/{2 ** (args.scale - scale)} of its edges), single thread, per step"},
