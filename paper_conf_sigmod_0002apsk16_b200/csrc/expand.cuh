@@ -38,6 +38,11 @@ __device__ __forceinline__ void page_at(const PageSet& ps, uint32_t i, uint32_t&
 __device__ __forceinline__ uint32_t decode_entry(const PageSet& ps, uint32_t e) {
     return ps.entry_encoding == GTS_ENTRY_VID32 ? e : __ldg(ps.rvt_start + (e >> 16)) + (e & 0xFFFFu);
 }
+// same, with the encoding fixed at compile time (kVid32: entries are VIDs)
+template <bool kVid32>
+__device__ __forceinline__ uint32_t decode_entry_t(const PageSet& ps, uint32_t e) {
+    return kVid32 ? e : __ldg(ps.rvt_start + (e >> 16)) + (e & 0xFFFFu);
+}
 
 __device__ __forceinline__ bool test_bit(const uint32_t* bm, uint32_t v) {
     return (__ldg(bm + (v >> 5)) >> (v & 31)) & 1u;
@@ -48,7 +53,8 @@ constexpr uint32_t kListWords = 128;    // sparse pages: frontier bitmap words c
 
 struct TileSmem {
     uint32_t soff[kTile + 1];  // word index of every record of the tile (all slots); soff[nv] = end
-    uint8_t sel[kTile];        // dense mode: vertex t of the tile is selected
+    uint8_t sel[kTile + 8];    // dense mode: vertex t of the tile is selected (4-byte aligned; +8:
+                               // dense_tile_ww reads 8-byte windows up to sel[nv + 3])
     uint32_t paytile[kTile];   // dense mode: payload of vertex t of the tile
     uint32_t tmask[kMaxTileWords];   // tiles of the current page holding a frontier vertex
     uint32_t off[kTile];       // word index of the first ADJLIST entry of item j
@@ -304,7 +310,7 @@ __device__ void expand_sp_micro(const PageSet& ps, Op& op, const uint8_t* data, 
 // Dense tile by warp windows (sm.soff / sm.sel / sm.paytile of the tile are
 // published).  Same per-edge contract as the tile walk: op.edges gets the 4
 // words of one 16-byte load per call.
-template <class Op>
+template <class Op, bool kVid32>
 __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSmem& sm, const uint4* q4,
                                               const uint32_t* words, uint32_t v0, uint32_t nv, uint32_t W0,
                                               uint32_t W1, uint64_t pol) {
@@ -344,6 +350,35 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
             const uint32_t mword = mw == 0 ? wm.m[0] : mw == 1 ? wm.m[1] : mw == 2 ? wm.m[2] : wm.m[3];
             uint32_t dst[kEdgesPerThread], wt[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
             bool valid[kEdgesPerThread];
+            if (!Op::kWeighted) {
+                // Unweighted records: every non-start word of a record is an entry.  The
+                // lane's 4 words have owners jb + c (c = record starts up to the word), so
+                // sel[jb .. jb+4] comes from one 8-byte window of sm.sel (two aligned LDS)
+                // instead of a dependent LDS.U8 per word.  selw = sm.sel - 4 bytes (jb >= -1).
+                const uint32_t bpos0 = (4 * lane) & 31;
+                const uint32_t nb = (mword >> bpos0) & 0xFu;           // record starts among my words
+                const int jb = j0 + (int)(before + __popc(mword & ((1u << bpos0) - 1u)));
+                const uint32_t t = (uint32_t)(jb + 4);
+                const uint32_t* selw = reinterpret_cast<const uint32_t*>(sm.sel) - 1;
+                const unsigned long long sw =
+                    ((unsigned long long)selw[(t >> 2) + 1] << 32 | selw[t >> 2]) >> (8 * (t & 3));
+                uint32_t c = 0;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const uint32_t w = 4 * q + k;
+                    const uint32_t st = (nb >> k) & 1u;
+                    c += st;
+                    valid[k] = !st && w >= W0 && w < W1 && ((sw >> (8 * c)) & 0xFFu);
+                    wt[k] = 0u;
+                    dst[k] = decode_entry_t<kVid32>(ps, word_of(vv[u], k));
+                    const int j = jb + (int)c;
+                    pl[k] = valid[k] ? sm.paytile[j] : 0u;
+                    src[k] = v0 + (uint32_t)j;
+                }
+                op.edges(dst, wt, pl, src, valid);
+                j0 += ns;
+                continue;
+            }
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
                 const uint32_t w = 4 * q + k;
@@ -351,14 +386,14 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
                 const int j = j0 + (int)(before + __popc(mword & ((2u << bpos) - 1u)));
                 bool ok = w >= W0 && w < W1 && !((mword >> bpos) & 1u);
                 uint32_t dj = 0;
-                if (ok) {
+                if (ok) {                              // adjacency words only, not the weights after them
                     const uint32_t o = sm.soff[j];
                     dj = (sm.soff[j + 1] - o - 1) >> wsh;
                     ok = w - o <= dj && sm.sel[j];
                 }
                 wt[k] = (Op::kReadWeights && ok) ? ld_stream_l1_u32(words + w + dj, pol) : 0u;
                 valid[k] = ok;
-                dst[k] = decode_entry(ps, word_of(vv[u], k));
+                dst[k] = decode_entry_t<kVid32>(ps, word_of(vv[u], k));
                 pl[k] = ok ? sm.paytile[j] : 0u;
                 src[k] = v0 + (uint32_t)j;
             }
@@ -475,7 +510,10 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 if (2 * total >= W1 - W0 && ps.ww) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
                     // 128-word windows; owners from record-start masks (no binary search)
-                    dense_tile_ww(ps, op, sm, q4, words, start + t0, nv, W0, W1, pol);
+                    if (ps.entry_encoding == GTS_ENTRY_VID32)
+                        dense_tile_ww<Op, true>(ps, op, sm, q4, words, start + t0, nv, W0, W1, pol);
+                    else
+                        dense_tile_ww<Op, false>(ps, op, sm, q4, words, start + t0, nv, W0, W1, pol);
                     __syncthreads();
                     continue;
                 }

@@ -144,8 +144,8 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 
 // -------------------------------------------------------------- kernels ---
 
-template <bool W, int M = kMicroTile>
-__global__ void __launch_bounds__(kThreads, 2)
+template <bool W, int M = kMicroTile, int MB = 2>
+__global__ void __launch_bounds__(kThreads, MB)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
                   uint32_t* work_ctr, unsigned long long* edges_out, uint32_t vprefix) {
     __shared__ TileSmem sm;
@@ -236,6 +236,130 @@ __global__ void sssp_finish_kernel(const uint32_t* __restrict__ gathered, int wo
     if ((threadIdx.x & 31) == 0 && mn != 0xFFFFFFFFu) atomicMin(minpend, mn);
 }
 
+// BFS level array from the per-level frontier bitmaps (slot L = the vertices
+// first reached at level L; slots are disjoint): LV[v] = the L whose slot holds
+// v, UNREACHED if none.  One coalesced pass writes every entry, replacing the
+// per-level scattered LV stores and the initial memset (Alg 2 l.18 writes
+// curLevel+1 once per discovered vertex; the result is the same array).
+// A thread takes one bitmap word (32 vertices): it loads the word of every
+// slot (independent loads), folds them into 8 bit planes of the level number,
+// and writes its 32 entries as 16-byte stores.  nlev <= 255.
+struct LevelPlanes {
+    uint32_t reached, p[8];
+};
+
+__device__ __forceinline__ LevelPlanes level_planes(const uint32_t* __restrict__ slots, uint32_t nlev, uint64_t words,
+                                                    uint64_t w) {
+    LevelPlanes lp{0u, {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u}};
+#pragma unroll 8
+    for (uint32_t L = 0; L < nlev; ++L) {
+        const uint32_t x = __ldg(slots + (uint64_t)L * words + w);
+        lp.reached |= x;
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+            if ((L >> k) & 1u) lp.p[k] |= x;
+    }
+    return lp;
+}
+
+__device__ __forceinline__ uint32_t level_of_bit(const LevelPlanes& lp, int b) {
+    uint32_t l = 0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) l |= ((lp.p[k] >> b) & 1u) << k;
+    return l;
+}
+
+__global__ void level_fill_kernel(uint32_t* level, const uint32_t* __restrict__ slots, uint32_t nlev, uint64_t words,
+                                  uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
+        const LevelPlanes lp = level_planes(slots, nlev, words, w);
+        const uint64_t v0 = w * 32;
+        if (v0 + 32 <= n) {
+            uint4* o = reinterpret_cast<uint4*>(level + v0);
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                uint32_t e[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const int b = 4 * q + k;
+                    e[k] = ((lp.reached >> b) & 1u) ? level_of_bit(lp, b) : GTS_UNREACHED;
+                }
+                o[q] = make_uint4(e[0], e[1], e[2], e[3]);
+            }
+        } else {
+            for (int b = 0; v0 + b < n; ++b) level[v0 + b] = ((lp.reached >> b) & 1u) ? level_of_bit(lp, b) : GTS_UNREACHED;
+        }
+    }
+}
+
+// Degree-ordered graphs: the same levels as bytes (0xFF = unreached; fewer than
+// 255 levels; the byte array holds words * 32 entries), then the caller-order
+// output gathered from that n-byte array (mostly L2-resident) instead of from
+// the 4n-byte LV.
+__global__ void level_fill8_kernel(uint8_t* lv8, const uint32_t* __restrict__ slots, uint32_t nlev, uint64_t words) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
+        const LevelPlanes lp = level_planes(slots, nlev, words, w);
+        uint32_t e[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            uint32_t x = 0;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const int b = 4 * q + k;
+                const uint32_t l = ((lp.reached >> b) & 1u) ? level_of_bit(lp, b) : 0xFFu;
+                x |= l << (8 * k);
+            }
+            e[q] = x;
+        }
+        uint4* o = reinterpret_cast<uint4*>(lv8 + w * 32);
+        o[0] = make_uint4(e[0], e[1], e[2], e[3]);
+        o[1] = make_uint4(e[4], e[5], e[6], e[7]);
+    }
+}
+
+// Fewer than 15 levels (every RMAT / power-law traversal): 4-bit levels, 0xF =
+// unreached.  The n/2-byte array (67 MB at RMAT-27) stays in L2 for the gather.
+__global__ void level_fill4_kernel(uint8_t* lv4, const uint32_t* __restrict__ slots, uint32_t nlev, uint64_t words) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
+        const LevelPlanes lp = level_planes(slots, nlev, words, w);
+        uint32_t e[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            uint32_t x = 0;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                const int b = 8 * q + k;
+                const uint32_t l = ((lp.reached >> b) & 1u) ? level_of_bit(lp, b) : 0xFu;
+                x |= l << (4 * k);
+            }
+            e[q] = x;
+        }
+        reinterpret_cast<uint4*>(lv4)[w] = make_uint4(e[0], e[1], e[2], e[3]);
+    }
+}
+
+__global__ void gather4_kernel(uint32_t* out, const uint8_t* __restrict__ lv4, const uint32_t* __restrict__ idx,
+                               uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+        const uint32_t i = idx[v];
+        const uint32_t l = (lv4[i >> 1] >> (4 * (i & 1))) & 0xFu;
+        out[v] = l == 0xFu ? GTS_UNREACHED : l;
+    }
+}
+
+__global__ void gather8_kernel(uint32_t* out, const uint8_t* __restrict__ lv8, const uint32_t* __restrict__ idx,
+                               uint64_t n) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+        const uint32_t l = lv8[idx[v]];
+        out[v] = l == 0xFFu ? GTS_UNREACHED : l;
+    }
+}
+
 // Length of the all-visited prefix of the bitmap, in words: the first word that
 // is not all ones.  On a degree-ordered graph the low IDs are the hubs and are
 // reached in the first levels, so later levels skip the visited test of every
@@ -293,7 +417,24 @@ struct Counters {               // device scratch, slot kCtr
     unsigned int vprefix_words;    // BFS: all-visited prefix of the bitmap (words)
 };
 
-enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather };
+enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather, kBufLvSlots, kBufLv8 };
+
+// deliver() for byte levels of a degree-ordered graph: out[v] = lv8[new_of_old[v]]
+static int deliver_levels8(Context* c, const Graph* g, const uint8_t* lv8, bool nibbles, void* out,
+                           uint32_t out_location) {
+    const uint64_t n = g->n;
+    uint32_t* dst;
+    if (out_location == GTS_OUT_DEVICE) dst = static_cast<uint32_t*>(out);
+    else GTS_TRY(c->buf(72, n * 4, (void**)&dst));     // deliver()'s staging slot
+    if (nibbles) gather4_kernel<<<c->num_sms * 4, 256, 0, c->stream>>>(dst, lv8, c->dg.new_of_old, n);
+    else gather8_kernel<<<c->num_sms * 4, 256, 0, c->stream>>>(dst, lv8, c->dg.new_of_old, n);
+    GTS_CUDA(cudaGetLastError());
+    if (out_location == GTS_OUT_DEVICE) {
+        GTS_CUDA(cudaStreamSynchronize(c->stream));
+        return GTS_OK;
+    }
+    return copy_out(c, dst, out, n * 4, out_location);
+}
 
 // pages holding vertex v among this rank's pages (Alg 1 line 5: "page ID containing start vertex")
 static std::vector<uint32_t> pages_of_vertex(const Graph* g, const DevGraph& d, int rank, uint64_t v) {
@@ -352,7 +493,26 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     GTS_TRY(c->buf(kBufCtr, sizeof(Counters), (void**)&ctr));
     if (c->world > 1) GTS_TRY(c->buf(kBufGather, words * 4 * c->world, (void**)&gathered));
     cudaStream_t s = c->stream;
-    GTS_CUDA(cudaMemsetAsync(value, 0xFF, n * 4, s));
+    // BFS level slots: the frontier of level L lives in slot L of a K-slot bitmap
+    // store, and LV is written once at the end by level_fill_kernel.  A traversal
+    // deeper than K levels fills LV from the slots and continues with the
+    // ping-pong frontiers, writing LV per level in frontier_finish_kernel.
+    // GTS_BFS_SLOTS=<K> (0 = per-level LV writes throughout); default 32, capped at 1 GiB.
+    uint32_t K = 0;
+    uint32_t* lvb = nullptr;
+    if (algo == kBFS) {
+        const char* ke = getenv("GTS_BFS_SLOTS");
+        K = ke ? (uint32_t)std::max(0L, atol(ke)) : 32u;
+        K = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(K, 255), (1ull << 30) / (words * 4));
+        if (K < 3) K = 0;
+        if (K) {
+            GTS_TRY(c->buf(kBufLvSlots, (size_t)K * words * 4, (void**)&lvb));
+            cur = lvb;
+            next = lvb + words;
+        }
+    }
+    bool slots = K > 0;
+    if (!slots) GTS_CUDA(cudaMemsetAsync(value, 0xFF, n * 4, s));
     if (visited) GTS_CUDA(cudaMemsetAsync(visited, 0, words * 4, s));
     GTS_CUDA(cudaMemsetAsync(cur, 0, words * 4, s));
     GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
@@ -377,7 +537,13 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
          bfs_expand_kernel<false, kMicroVertex>, bfs_expand_kernel<false, kMicroHybrid>},
         {bfs_expand_kernel<true, kMicroTile>, bfs_expand_kernel<true, kMicroEdge>,
          bfs_expand_kernel<true, kMicroVertex>, bfs_expand_kernel<true, kMicroHybrid>}};
-    const BfsKern bfs_kern = bfs_k[g->weighted ? 1 : 0][micro];
+    BfsKern bfs_kern = bfs_k[g->weighted ? 1 : 0][micro];
+    // three 512-thread CTAs per SM (40 registers, a few spilled bytes) by default: the
+    // per-tile barriers of one CTA are covered by the other two (RMAT-27 BFS kernels
+    // 10.25 -> 9.26 ms); GTS_BFS_OCC=2 selects two CTAs (64 registers)
+    const char* oce = getenv("GTS_BFS_OCC");
+    if (micro == kMicroTile && (!oce || atoi(oce) != 2))
+        bfs_kern = g->weighted ? bfs_expand_kernel<true, kMicroTile, 3> : bfs_expand_kernel<false, kMicroTile, 3>;
     const char* hde = getenv("GTS_HYBRID_DEG");
     const uint32_t hybrid_deg = hde ? (uint32_t)std::max(1L, atol(hde)) : 8u;
     const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_expand_kernel;
@@ -448,7 +614,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         GTS_CUDA(cudaMemsetAsync(&ctr->list_count, 0, 4, s));
         if (algo == kBFS) {
             frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, next,
-                                                            visited, value, L + 1, &ctr->count);
+                                                            visited, slots ? nullptr : value, L + 1, &ctr->count);
             GTS_CUDA(cudaMemsetAsync(&ctr->vprefix_words, 0xFF, 4, s));
             visited_prefix_kernel<<<fin_grid, 256, 0, s>>>(visited, words, &ctr->vprefix_words);
             ++launches;
@@ -486,8 +652,39 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                 GTS_CUDA(cudaStreamSynchronize(s));
             }
         }
-        std::swap(cur, next);
+        if (slots && L + 2 < K) {                // next level's frontier in the next slot
+            cur = next;
+            next = lvb + (uint64_t)(L + 2) * words;
+        } else {
+            if (slots) {                          // out of slots: LV for levels 0..L+1 now
+                level_fill_kernel<<<fin_grid, 256, 0, s>>>(value, lvb, L + 2, words, n);
+                GTS_CUDA(cudaGetLastError());
+                ++launches;
+                slots = false;
+                GTS_TRY(c->buf(kBufNext, words * 4, (void**)&next));
+                cur = lvb + (uint64_t)(L + 1) * words;
+                std::swap(cur, next);             // (swapped back below)
+            }
+            std::swap(cur, next);
+        }
         GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
+    }
+    uint8_t* lv8 = nullptr;
+    const bool nib = levels < 15;
+    if (slots && g->ordered && nib) {
+        GTS_TRY(c->buf(kBufLv8, words * 32, (void**)&lv8));
+        level_fill4_kernel<<<fin_grid, 256, 0, s>>>(lv8, lvb, levels, words);
+        GTS_CUDA(cudaGetLastError());
+        launches += 2;
+    } else if (slots && g->ordered && levels < 255) {
+        GTS_TRY(c->buf(kBufLv8, words * 32, (void**)&lv8));
+        level_fill8_kernel<<<fin_grid, 256, 0, s>>>(lv8, lvb, levels, words);
+        GTS_CUDA(cudaGetLastError());
+        launches += 2;
+    } else if (slots) {
+        level_fill_kernel<<<fin_grid, 256, 0, s>>>(value, lvb, levels, words, n);
+        GTS_CUDA(cudaGetLastError());
+        ++launches;
     }
     if (persist) GTS_TRY(persist_window(c, s, nullptr, 0));
     if (algo == kSSSP && c->world > 1) {   // every rank must agree before the collective check
@@ -516,7 +713,8 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         GTS_CUDA(cudaStreamSynchronize(s));
         if (bad) return fail(GTS_EOVERFLOW, "an SSSP distance reaches 2^32-1");
     }
-    GTS_TRY(deliver(c, g, value, out, rc.out_location, false));
+    if (lv8) GTS_TRY(deliver_levels8(c, g, lv8, nib, out, rc.out_location));
+    else GTS_TRY(deliver(c, g, value, out, rc.out_location, false));
     if (st) {
         std::memset(st, 0, sizeof(*st));
         st->wall_s = now_s() - t_start;

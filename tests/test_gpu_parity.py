@@ -97,6 +97,23 @@ def test_bfs_pid16_entries(G, ctx, name):
         assert np.array_equal(got, oracle.bfs(g.row_ptr, g.col, src))
 
 
+@pytest.mark.parametrize("name", ["fig1", "path", "bintree", "rmat16_4k", "rmat20", "twitter20"])
+@pytest.mark.parametrize("k", ["0", "3", "5", "64"])
+def test_bfs_level_slots(G, ctx, name, k, monkeypatch):
+    """Level-slot LV construction (GTS_BFS_SLOTS=K): LV written once from the per-level
+    frontier bitmaps; traversals deeper than K switch to per-level LV writes mid-way.
+    K=0 is per-level writes throughout.  Resident, streamed and degree-ordered pages."""
+    monkeypatch.setenv("GTS_BFS_SLOTS", k)
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
+    go = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+    for src in _sources(g)[:2]:
+        want = oracle.bfs(g.row_ptr, g.col, src)
+        for gg, kw in ((gr, {}), (go, {}), (gr, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3))):
+            got, st = G.gts_bfs(ctx, gg, src, **kw)
+            assert np.array_equal(got, want), (name, k, src, kw, int(np.sum(got != want)))
+
+
 def test_bfs_deterministic_and_device_output(G, ctx):
     import torch
     g, pb = graph("rmat20")
@@ -170,7 +187,7 @@ def test_pagerank_tolerance(G, ctx, name):
 @pytest.mark.parametrize("order", [False, True])
 def test_pagerank_in_star_hub(G, ctx, k, order):
     """Hub stress pin: k leaves -> dangling hub; closed-form recurrence in fp64.
-    order=True runs the degree-ordered binned scatter (hub in the shared-memory hot set)."""
+    order=True runs the degree-ordered scatter (hub in the shared-memory hot set)."""
     n = k + 1
     row_ptr = np.concatenate([[0, 0], np.arange(1, k + 1)]).astype(np.uint64)
     col = np.zeros(k, np.uint32)
