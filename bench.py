@@ -59,6 +59,11 @@ class ClockSampler:
         self.proc = None
 
     def start(self):
+        mode = os.environ.get("GTS_BENCH_CLOCKS", "smi")
+        if mode == "nvml":
+            return self._start_nvml()
+        if mode == "off":
+            return
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
                                           "-lms", "200", "-i", str(self.device)], stdout=subprocess.PIPE,
@@ -72,14 +77,43 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.lines.append(line.strip())
 
+    # in-process NVML sampling (GTS_BENCH_CLOCKS=nvml): the same fields as the
+    # nvidia-smi line, without a second process polling the driver
+    def _start_nvml(self):
+        import pynvml
+        pynvml.nvmlInit()
+        self.nv = pynvml
+        self.h = pynvml.nvmlDeviceGetHandleByIndex(self.device)
+        self.stop_ev = threading.Event()
+        bits = {"hw_slowdown": pynvml.nvmlClocksEventReasonHwSlowdown,
+                "hw_thermal_slowdown": pynvml.nvmlClocksEventReasonHwThermalSlowdown,
+                "sw_thermal_slowdown": pynvml.nvmlClocksEventReasonSwThermalSlowdown,
+                "sw_power_cap": pynvml.nvmlClocksEventReasonSwPowerCap}
+
+        def run():
+            while not self.stop_ev.is_set():
+                sm = pynvml.nvmlDeviceGetClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+                mx = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+                r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                act = ["Active" if r & b else "Not Active" for b in bits.values()]
+                self.lines.append(", ".join([str(sm), str(mx), "0", hex(r)] + act))
+                self.stop_ev.wait(0.2)
+        self.t = threading.Thread(target=run, daemon=True)
+        self.t.start()
+        self.proc = "nvml"
+
     def stop(self):
         if not self.proc:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=5)
-        except Exception:
-            self.proc.kill()
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["clock sampling off"]}
+        if self.proc == "nvml":
+            self.stop_ev.set()
+            self.t.join(timeout=5)
+        else:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
         sm, mx, reasons = [], [], set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in self.lines:

@@ -154,7 +154,8 @@ bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visite
     block_add_u64(op.nedges, edges_out);
 }
 
-__global__ void __launch_bounds__(kThreads, 2)
+template <int MB = 2>
+__global__ void __launch_bounds__(kThreads, MB)
 sssp_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* dist, uint32_t* next,
                    uint32_t* work_ctr, unsigned long long* edges_out, uint32_t* ovf_flag, uint32_t T) {
     __shared__ TileSmem sm;
@@ -546,7 +547,11 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         bfs_kern = g->weighted ? bfs_expand_kernel<true, kMicroTile, 3> : bfs_expand_kernel<false, kMicroTile, 3>;
     const char* hde = getenv("GTS_HYBRID_DEG");
     const uint32_t hybrid_deg = hde ? (uint32_t)std::max(1L, atol(hde)) : 8u;
-    const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_expand_kernel;
+    // GTS_SSSP_OCC=3: three 512-thread CTAs per SM for the SSSP expansion (RMAT-27: 35.7 vs
+    // 35.1 ms for two -- the weighted walk spills 124 bytes at 40 registers -- so off by default)
+    const char* soe = getenv("GTS_SSSP_OCC");
+    auto sssp_kern = (soe && atoi(soe) == 3) ? sssp_expand_kernel<3> : sssp_expand_kernel<2>;
+    const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_kern;
     int grid = 0;
     GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
     const int fin_grid = c->num_sms * 4;
@@ -590,7 +595,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                     bfs_kern<<<std::min(grid, cap), kThreads, 0, s>>>(
                                         p2, cur, visited, next, &ctr->work, &ctr->edges, vprefix);
                                 } else
-                                    sssp_expand_kernel<<<std::min(grid, cap), kThreads, 0, s>>>(
+                                    sssp_kern<<<std::min(grid, cap), kThreads, 0, s>>>(
                                         ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T);
                                 if (timing) cudaEventRecord(ev.second, s);
                                 GTS_CUDA(cudaGetLastError());

@@ -149,8 +149,8 @@ wcc_sample_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t ks)
     }
 }
 
-template <bool W>
-__global__ void __launch_bounds__(kThreads, 2)
+template <bool W, int MB = 2>
+__global__ void __launch_bounds__(kThreads, MB)
 wcc_sweep_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t* changed, const uint32_t* gbm,
                  const uint32_t* rstar) {
     __shared__ TileSmem sm;
@@ -213,7 +213,12 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     const int eg = c->num_sms * 4;
     wcc_init_kernel<<<eg, 256, 0, s>>>(label, n);
     int grid = 0;
-    auto sweep_k = g->weighted ? wcc_sweep_kernel<true> : wcc_sweep_kernel<false>;
+    // three 512-thread CTAs per SM for the sweep by default (40 registers; RMAT-27 sweep
+    // 17.4 -> 14.6 ms: the third CTA covers the per-tile barriers); GTS_WCC_OCC=2 = two
+    const char* oce = getenv("GTS_WCC_OCC");
+    const bool occ3 = !oce || atoi(oce) != 2;
+    auto sweep_k = g->weighted ? (occ3 ? wcc_sweep_kernel<true, 3> : wcc_sweep_kernel<true, 2>)
+                               : (occ3 ? wcc_sweep_kernel<false, 3> : wcc_sweep_kernel<false, 2>);
     GTS_TRY(sms_grid(c, (const void*)sweep_k, kThreads, 0, &grid));
     uint64_t launches = 1, main_launches = 0, nccl_bytes = 0;
     uint32_t sweeps = 0;

@@ -114,6 +114,24 @@ def test_bfs_level_slots(G, ctx, name, k, monkeypatch):
             assert np.array_equal(got, want), (name, k, src, kw, int(np.sum(got != want)))
 
 
+@pytest.mark.parametrize("name", ["fig1", "rmat16_4k", "rmat20", "twitter20", "instar"])
+@pytest.mark.parametrize("occ", ["2", "3"])
+def test_occupancy_variants(G, ctx, name, occ, monkeypatch):
+    """Two- and three-CTA-per-SM builds of the BFS, WCC and SSSP expansion kernels
+    (GTS_BFS_OCC / GTS_WCC_OCC / GTS_SSSP_OCC), resident and degree-ordered pages."""
+    for k in ("GTS_BFS_OCC", "GTS_WCC_OCC", "GTS_SSSP_OCC"):
+        monkeypatch.setenv(k, occ)
+    g, pb = graph(name)
+    w = inputs.edge_weights(g)
+    for order in (False, True):
+        gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
+        src = _sources(g)[1]
+        assert np.array_equal(G.gts_bfs(ctx, gr, src)[0], oracle.bfs(g.row_ptr, g.col, src))
+        assert np.array_equal(G.gts_wcc(ctx, gr)[0], oracle.wcc(g.row_ptr, g.col))
+        grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb, order=order)
+        assert np.array_equal(G.gts_sssp(ctx, grw, src)[0], oracle.sssp(g.row_ptr, g.col, w, src))
+
+
 def test_bfs_deterministic_and_device_output(G, ctx):
     import torch
     g, pb = graph("rmat20")
@@ -184,10 +202,12 @@ def test_pagerank_tolerance(G, ctx, name):
 
 
 @pytest.mark.parametrize("k", [1_300_000, 4_600_000])
-@pytest.mark.parametrize("order", [False, True])
-def test_pagerank_in_star_hub(G, ctx, k, order):
+@pytest.mark.parametrize("order,lean", [(False, "0"), (True, "0"), (True, "1")])
+def test_pagerank_in_star_hub(G, ctx, k, order, lean, monkeypatch):
     """Hub stress pin: k leaves -> dangling hub; closed-form recurrence in fp64.
-    order=True runs the degree-ordered scatter (hub in the shared-memory hot set)."""
+    order=True runs the degree-ordered scatter (hub in the shared-memory hot set), with the
+    tile walk (lean=0) or the lean warp-window scatter (lean=1)."""
+    monkeypatch.setenv("GTS_PR_LEAN", lean)
     n = k + 1
     row_ptr = np.concatenate([[0, 0], np.arange(1, k + 1)]).astype(np.uint64)
     col = np.zeros(k, np.uint32)
@@ -300,10 +320,15 @@ def test_degree_ordered_device_outputs(G, ctx):
 
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "instar", "multi"])
-@pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow"])
+@pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow", "lean", "tilewalk"])
 def test_pagerank_ordered_variants(G, ctx, name, mode, monkeypatch):
     """Degree-ordered PageRank with and without the L2 persistence window (GTS_L2_PERSIST=0),
-    and with the warp-window walk (record-start masks) instead of the tile walk."""
+    with the warp-window walk (record-start masks), the lean warp-window scatter
+    (GTS_PR_LEAN=1) and the tile walk (GTS_PR_LEAN=0)."""
+    if mode == "lean":
+        monkeypatch.setenv("GTS_PR_LEAN", "1")
+    if mode == "tilewalk":
+        monkeypatch.setenv("GTS_PR_LEAN", "0")
     if mode == "nopersist":
         monkeypatch.setenv("GTS_L2_PERSIST", "0")
     if mode == "warpwindow":
