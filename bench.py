@@ -454,6 +454,7 @@ def main():
                 "wcc_s": out["wcc"]["s"] / K if "wcc" in algos else None,
                 "wcc_sweeps": out.get("wcc", {}).get("iters"),
                 "kernel_s_per_step": {a: out[a]["main_s"] / K for a in algos},
+                "call_ms_each_step": {a: [round(1e3 * t, 3) for t, _ in rec[a]] for a in algos},
                 "merge_s_per_step": {a: out[a]["merge_s"] / K for a in algos},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": int(sum(out[a]["launches"] for a in algos))}

@@ -474,157 +474,6 @@ pr_scatter_ww_kernel(PageSet ps, const float* __restrict__ x, float* acc, float 
     if ((tid & 31) == 0 && dang != 0.0) atomicAdd(dang_out, dang);
 }
 
-// Lean scatter for unweighted VID32 pages with a dense hot set (degree-ordered):
-// the warp-window walk of pr_scatter_ww_kernel, with the per-edge work cut to
-// what Alg 4 l.16 needs.  A lane's 4 words have owners jb + c (c = record
-// starts up to the word; every non-start word of an unweighted record is an
-// entry), so there is no per-word popcount search; there is no run combiner
-// (consecutive equal destinations are < 1% of RMAT edges, and the combiner's
-// deferred emit made every edge branchy); each edge is one predicated global
-// red.add or one shared-memory add into the hot set.
-template <int T, int kMinBlocks, uint32_t H>
-__global__ void __launch_bounds__(T, kMinBlocks)
-pr_scatter_lean_kernel(PageSet ps, const float* __restrict__ x, float* acc, float d, double* dang_out,
-                       uint32_t* work_ctr, uint32_t n_hot) {
-    __shared__ PrSmem<T> sm;
-    extern __shared__ uint4 dyn_smem[];
-    float* hacc = reinterpret_cast<float*>(dyn_smem);
-    constexpr int kW = T / 32;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    for (uint32_t i = tid; i < H; i += T) hacc[i] = 0.f;
-    __syncthreads();
-    const uint64_t pol = policy_evict_first();
-    const uint32_t count = ps.count;
-    double dang = 0.0;
-    auto emit = [&](uint32_t dst, float c) {
-        if (dst < H) atomicAdd(hacc + dst, c);
-        else atomicAdd(acc + dst, c);                   // REDG.E.ADD.F32 (result unused)
-    };
-    for (;;) {
-        if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
-        __syncthreads();
-        const uint32_t it = sm.item;
-        __syncthreads();
-        if (it >= count) break;
-        uint32_t pid;
-        const uint8_t* data;
-        page_at(ps, it, pid, data);
-        const uint8_t* end = data + ps.page_bytes;
-        const uint32_t kind = ld32(end - 4);
-        const uint32_t nslots = ld32(end - 8);
-        const uint4* q4 = reinterpret_cast<const uint4*>(data);
-        if (kind == GTS_PAGE_LP) {
-            const uint32_t vid = ld32(end - kLpFooter - kSlotBytes);
-            const uint32_t total = ld32(end - 16);
-            const uint32_t len = ld32(data);
-            const float c = d * __ldg(x + vid) / (float)total;
-            const uint32_t wend = 1 + len, qend = (wend + 3) >> 2;
-            for (uint32_t qb = tid; qb < qend; qb += T * kPrUnroll) {
-                uint4 v[kPrUnroll];
-#pragma unroll
-                for (int u = 0; u < kPrUnroll; ++u) {
-                    const uint32_t q = qb + u * T;
-                    if (q < qend) v[u] = ld_stream_v4(q4 + q, pol);
-                }
-#pragma unroll
-                for (int u = 0; u < kPrUnroll; ++u) {
-                    const uint32_t q = qb + u * T;
-                    if (q >= qend) break;
-#pragma unroll
-                    for (int k = 0; k < 4; ++k) {
-                        const uint32_t w = 4 * q + k;
-                        if (w >= 1 && w < wend) emit(word_of(v[u], k), c);
-                    }
-                }
-            }
-        } else {
-            const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
-            for (uint32_t t0 = 0; t0 < nslots; t0 += T) {
-                const uint32_t nv = min((uint32_t)T, nslots - t0);
-                if ((uint32_t)tid < nv) {
-                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
-                    sm.off[tid] = ld_stream_u32(slot + 4, pol) >> 2;
-                    if ((uint32_t)tid == nv - 1) {
-                        if (t0 + nv < nslots) {
-                            sm.off[nv] = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
-                        } else {
-                            const uint32_t o = ld_stream_u32(slot + 4, pol);
-                            sm.off[nv] = (o >> 2) + 1 + ld32(data + o);
-                        }
-                    }
-                }
-                __syncthreads();
-                if ((uint32_t)tid < nv) {
-                    const uint32_t deg = sm.off[tid + 1] - sm.off[tid] - 1;
-                    const float xv = ld_stream_f32(x + start + t0 + tid, pol);
-                    float c = 0.f;
-                    if (deg == 0) dang += (double)xv;      // dangling mass (R3)
-                    else c = d * xv / (float)deg;
-                    sm.c[tid] = c;
-                }
-                __syncthreads();
-                const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
-                const uint32_t wbase = W0 & ~3u;
-                const uint32_t nwin = (W1 - wbase + 127) >> 7;
-                const uint32_t per = (nwin + kW - 1) / kW;
-                const uint32_t wa = min(nwin, warp * per), wb = min(nwin, wa + per);
-                if (wa < wb) {
-                    const uint32_t base = wbase + (wa << 7);
-                    int lo = -1, hi = (int)nv;               // off[lo] < base <= off[hi]
-                    while (hi - lo > 1) {
-                        const int mid = (lo + hi) >> 1;
-                        if (sm.off[mid] < base) lo = mid; else hi = mid;
-                    }
-                    int j0 = lo;
-                    for (uint32_t wi = wa; wi < wb; wi += kPrUnroll) {
-                        uint4 v[kPrUnroll];
-#pragma unroll
-                        for (int u = 0; u < kPrUnroll; ++u) {
-                            const uint32_t q = ((wbase + ((wi + u) << 7)) >> 2) + lane;
-                            v[u] = make_uint4(0u, 0u, 0u, 0u);
-                            if (wi + u < wb && 4 * q < W1) v[u] = ld_stream_v4(q4 + q, pol);
-                        }
-#pragma unroll
-                        for (int u = 0; u < kPrUnroll; ++u) {
-                            if (wi + u >= wb) break;
-                            const uint32_t bw = wbase + ((wi + u) << 7);
-                            const uint32_t q = (bw >> 2) + lane;
-                            int ns;
-                            const WinMask wm = win_mask(sm.off, j0, nv, bw, ns);
-                            const uint32_t mw = lane >> 3;
-                            uint32_t before = 0;
-#pragma unroll
-                            for (int k = 0; k < 4; ++k) before += (uint32_t)k < mw ? __popc(wm.m[k]) : 0u;
-                            const uint32_t mword = mw == 0 ? wm.m[0] : mw == 1 ? wm.m[1] : mw == 2 ? wm.m[2] : wm.m[3];
-                            const uint32_t bpos0 = (4 * lane) & 31;
-                            const uint32_t nb = (mword >> bpos0) & 0xFu;
-                            const int jb = j0 + (int)(before + __popc(mword & ((1u << bpos0) - 1u)));
-                            uint32_t cnt = 0;
-#pragma unroll
-                            for (int k = 0; k < 4; ++k) {
-                                const uint32_t w = 4 * q + k;
-                                const uint32_t st = (nb >> k) & 1u;
-                                cnt += st;
-                                if (!st && w >= W0 && w < W1) emit(word_of(v[u], k), sm.c[jb + (int)cnt]);
-                            }
-                            j0 += ns;
-                        }
-                    }
-                }
-                __syncthreads();
-            }
-        }
-    }
-    __syncthreads();
-    for (uint32_t i = tid; i < n_hot; i += T) {
-        const float v = hacc[i];
-        if (v != 0.f) atomicAdd(acc + i, v);
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) dang += __shfl_down_sync(0xFFFFFFFFu, dang, o);
-    if ((tid & 31) == 0 && dang != 0.0) atomicAdd(dang_out, dang);
-}
-
 // Plain push PageRank (Alg 4/5: c = d x[u] / deg(u), one red.add per edge, no
 // hot set) on the generic page engine, for the micro-level comparison of App E
 // (GTS_MICRO_EDGE / VERTEX / HYBRID / TILE).  Same arguments as pr_scatter_kernel.
@@ -1315,10 +1164,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     // (measured on RMAT-27: 12.48 vs 12.24 ms for the tile walk, so opt-in: GTS_PR_WW=1)
     const char* wwe = getenv("GTS_PR_WW");
     const bool ww = mode == kDense && big && wwe && atoi(wwe) > 0;
-    // lean warp-window scatter (unweighted VID32 degree-ordered pages): GTS_PR_LEAN=1
-    const char* lne = getenv("GTS_PR_LEAN");
-    const bool lean = mode == kDense && big && !ww && !g->weighted && g->entry_encoding == GTS_ENTRY_VID32 &&
-                      lne && atoi(lne) > 0;
     const void* kern;
     size_t dyn;
     int threads;
@@ -1352,11 +1197,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         dyn = pr_dyn_smem<kDense, kHotDense>();
         threads = kThreads;
         n_hot = (uint32_t)std::min<uint64_t>(n, kHotDense);
-    } else if (lean) {
-        kern = (const void*)pr_scatter_lean_kernel<1024, 1, kHotDenseBig>;
-        dyn = pr_dyn_smem<kDense, kHotDenseBig>();
-        threads = 1024;
-        n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
     } else if (ww) {
         kern = g->weighted ? (const void*)pr_scatter_ww_kernel<true, 1024, 1, kHotDenseBig>
                            : (const void*)pr_scatter_ww_kernel<false, 1024, 1, kHotDenseBig>;
@@ -1405,7 +1245,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         void* args_full[] = {(void*)&p2, (void*)&x, (void*)&acc, (void*)&hk, (void*)&dmp, (void*)&D,
                              (void*)&ctr, (void*)&n_hot, (void*)&rp};
         void* args_ww[] = {(void*)&p2, (void*)&x, (void*)&acc, (void*)&dmp, (void*)&D, (void*)&ctr, (void*)&n_hot};
-        void** args = (ww || lean) && !micro ? args_ww : args_full;
+        void** args = ww && !micro ? args_ww : args_full;
         cudaLaunchConfig_t lc;
         std::memset(&lc, 0, sizeof(lc));
         lc.gridDim = dim3(std::min(grid, cap));

@@ -202,12 +202,10 @@ def test_pagerank_tolerance(G, ctx, name):
 
 
 @pytest.mark.parametrize("k", [1_300_000, 4_600_000])
-@pytest.mark.parametrize("order,lean", [(False, "0"), (True, "0"), (True, "1")])
-def test_pagerank_in_star_hub(G, ctx, k, order, lean, monkeypatch):
+@pytest.mark.parametrize("order", [False, True])
+def test_pagerank_in_star_hub(G, ctx, k, order):
     """Hub stress pin: k leaves -> dangling hub; closed-form recurrence in fp64.
-    order=True runs the degree-ordered scatter (hub in the shared-memory hot set), with the
-    tile walk (lean=0) or the lean warp-window scatter (lean=1)."""
-    monkeypatch.setenv("GTS_PR_LEAN", lean)
+    order=True runs the degree-ordered scatter (hub in the shared-memory hot set)."""
     n = k + 1
     row_ptr = np.concatenate([[0, 0], np.arange(1, k + 1)]).astype(np.uint64)
     col = np.zeros(k, np.uint32)
@@ -320,15 +318,10 @@ def test_degree_ordered_device_outputs(G, ctx):
 
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "instar", "multi"])
-@pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow", "lean", "tilewalk"])
+@pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow"])
 def test_pagerank_ordered_variants(G, ctx, name, mode, monkeypatch):
     """Degree-ordered PageRank with and without the L2 persistence window (GTS_L2_PERSIST=0),
-    with the warp-window walk (record-start masks), the lean warp-window scatter
-    (GTS_PR_LEAN=1) and the tile walk (GTS_PR_LEAN=0)."""
-    if mode == "lean":
-        monkeypatch.setenv("GTS_PR_LEAN", "1")
-    if mode == "tilewalk":
-        monkeypatch.setenv("GTS_PR_LEAN", "0")
+    and with the warp-window walk (record-start masks) instead of the tile walk."""
     if mode == "nopersist":
         monkeypatch.setenv("GTS_L2_PERSIST", "0")
     if mode == "warpwindow":
