@@ -48,7 +48,14 @@ def measured_peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """SM clocks + throttle reasons during the timed region.
+
+    Default (GTS_BENCH_CLOCKS=kick): in-process NVML, one sample taken by a helper
+    thread each time the step starts its PageRank call (kick()), i.e. while the
+    GPU is loaded and the host is not on the critical path: a poller running
+    concurrently (nvidia-smi -lms 200, the "smi" mode) stalls the per-level host
+    synchronisations of SSSP/WCC through the driver lock and measured +0-40 ms
+    per call.  "nvml" polls in-process every 200 ms, "off" disables sampling."""
     FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
               "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
               "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
@@ -59,9 +66,9 @@ class ClockSampler:
         self.proc = None
 
     def start(self):
-        mode = os.environ.get("GTS_BENCH_CLOCKS", "smi")
-        if mode == "nvml":
-            return self._start_nvml()
+        mode = os.environ.get("GTS_BENCH_CLOCKS", "kick")
+        if mode in ("nvml", "kick"):
+            return self._start_nvml(kicked=mode == "kick")
         if mode == "off":
             return
         try:
@@ -79,12 +86,21 @@ class ClockSampler:
 
     # in-process NVML sampling (GTS_BENCH_CLOCKS=nvml): the same fields as the
     # nvidia-smi line, without a second process polling the driver
-    def _start_nvml(self):
-        import pynvml
-        pynvml.nvmlInit()
+    def kick(self):
+        if getattr(self, "kick_ev", None) is not None:
+            self.kick_ev.set()
+
+    def _start_nvml(self, kicked=False):
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+        except Exception as e:  # pragma: no cover
+            log("NVML unavailable:", e)
+            return
         self.nv = pynvml
         self.h = pynvml.nvmlDeviceGetHandleByIndex(self.device)
         self.stop_ev = threading.Event()
+        self.kick_ev = threading.Event() if kicked else None
         bits = {"hw_slowdown": pynvml.nvmlClocksEventReasonHwSlowdown,
                 "hw_thermal_slowdown": pynvml.nvmlClocksEventReasonHwThermalSlowdown,
                 "sw_thermal_slowdown": pynvml.nvmlClocksEventReasonSwThermalSlowdown,
@@ -92,12 +108,18 @@ class ClockSampler:
 
         def run():
             while not self.stop_ev.is_set():
+                if self.kick_ev is not None:
+                    if not self.kick_ev.wait(0.05):
+                        continue
+                    self.kick_ev.clear()
+                    time.sleep(0.01)          # inside the PageRank call
                 sm = pynvml.nvmlDeviceGetClockInfo(self.h, pynvml.NVML_CLOCK_SM)
                 mx = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
                 r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
                 act = ["Active" if r & b else "Not Active" for b in bits.values()]
                 self.lines.append(", ".join([str(sm), str(mx), "0", hex(r)] + act))
-                self.stop_ev.wait(0.2)
+                if self.kick_ev is None:
+                    self.stop_ev.wait(0.2)
         self.t = threading.Thread(target=run, daemon=True)
         self.t.start()
         self.proc = "nvml"
@@ -304,6 +326,8 @@ def main():
             if a == "bfs":
                 _, st = G.gts_bfs(ctx, gr, src, out=lv, timing=True)
             elif a == "pr":
+                if sampler is not None:
+                    sampler.kick()
                 _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=pr, timing=True)
             elif a == "sssp":
                 _, st = G.gts_sssp(ctx, grw, src, out=ds, timing=True)
@@ -322,11 +346,18 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
+    sampler = None
     for i in range(args.warmup):
         step(None)
         log(f"[rank {rank}] warmup {i} done")
     sampler = ClockSampler(local_rank)
     sampler.start()
+    if "pr" not in algos:             # no PageRank call to sample inside: sample at each step start
+        _step = step
+
+        def step(record):
+            sampler.kick()
+            _step(record)
     rec = {}
     barrier()
     t_start = torch.cuda.Event(enable_timing=True)
