@@ -106,6 +106,8 @@ class ClockSampler:
                 "sw_thermal_slowdown": pynvml.nvmlClocksEventReasonSwThermalSlowdown,
                 "sw_power_cap": pynvml.nvmlClocksEventReasonSwPowerCap}
 
+        mx = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)   # once: this query takes ms
+
         def run():
             while not self.stop_ev.is_set():
                 if self.kick_ev is not None:
@@ -114,7 +116,6 @@ class ClockSampler:
                     self.kick_ev.clear()
                     time.sleep(0.01)          # inside the PageRank call
                 sm = pynvml.nvmlDeviceGetClockInfo(self.h, pynvml.NVML_CLOCK_SM)
-                mx = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
                 r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
                 act = ["Active" if r & b else "Not Active" for b in bits.values()]
                 self.lines.append(", ".join([str(sm), str(mx), "0", hex(r)] + act))

@@ -61,7 +61,6 @@ struct RouteParams {
     uint64_t lo, hi;
     int nranks;
     int drop_remote;                   // paper-literal Strategy-S (broadcast pages): ignore remote updates
-    int dang_all;                      // count the dangling mass of every source (single-rank tail deferral)
 };
 
 __device__ __forceinline__ int route_owner(const RouteParams& rp, uint32_t v) {
@@ -249,8 +248,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                     float c = 0.f;
                     // dangling mass (R3); a routed rank counts only its own WA range (under
                     // S_BCAST every rank sees every page)
-                    if (deg == 0 && (kMode != kRoute || rp.dang_all ||
-                                     (uint64_t)(start + t0 + tid) - rp.lo < rp.hi - rp.lo))
+                    if (deg == 0 && (kMode != kRoute || (uint64_t)(start + t0 + tid) - rp.lo < rp.hi - rp.lo))
                         dang += (double)xv;
                     else c = d * xv / (float)deg;
                     sm.c[tid] = c;
@@ -1166,14 +1164,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     // (measured on RMAT-27: 12.48 vs 12.24 ms for the tile walk, so opt-in: GTS_PR_WW=1)
     const char* wwe = getenv("GTS_PR_WW");
     const bool ww = mode == kDense && big && wwe && atoi(wwe) > 0;
-    // tail deferral (GTS_PR_TAIL=<first deferred internal ID>): on one rank, updates
-    // for destinations >= C are appended as (dst, value) pairs to 7 ID-range bins by the
-    // routed scatter and applied bin by bin after it (each bin's WA range L2-sized), instead
-    // of one L2-missing reduction each; [0, C) keeps the hot set + direct reductions
-    const char* tle = getenv("GTS_PR_TAIL");
-    const uint64_t tailC = tle ? (uint64_t)std::max(0L, atol(tle)) : 0;
-    const bool tail = tailC >= kHotDenseBig && tailC < n && mode == kDense && big && !ww && !micro && !streamed &&
-                      c->world == 1 && !(getenv("GTS_PR_BINNED") && atoi(getenv("GTS_PR_BINNED")) > 0);
     const void* kern;
     size_t dyn;
     int threads;
@@ -1207,12 +1197,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         dyn = pr_dyn_smem<kDense, kHotDense>();
         threads = kThreads;
         n_hot = (uint32_t)std::min<uint64_t>(n, kHotDense);
-    } else if (tail) {
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kRoute, 1024, 1, kHotDenseBig>
-                           : (const void*)pr_scatter_kernel<false, kRoute, 1024, 1, kHotDenseBig>;
-        dyn = pr_dyn_smem<kRoute, kHotDenseBig>();
-        threads = 1024;
-        n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
     } else if (ww) {
         kern = g->weighted ? (const void*)pr_scatter_ww_kernel<true, 1024, 1, kHotDenseBig>
                            : (const void*)pr_scatter_ww_kernel<false, 1024, 1, kHotDenseBig>;
@@ -1303,72 +1287,15 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         ++launches;
         return GTS_OK;
     };
-    uint2* t_send = nullptr;
-    uint32_t *t_cnt = nullptr, *t_off = nullptr;
-    if (tail && !route && !binned) {
-        rp0.nranks = kMaxRanks;
-        rp0.vr[0] = 0;
-        rp0.vr[1] = tailC;
-        const uint64_t bw = (n - tailC + kMaxRanks - 2) / (kMaxRanks - 1);
-        for (int k = 2; k <= kMaxRanks; ++k) rp0.vr[k] = std::min<uint64_t>(n, tailC + (k - 1) * bw);
-        rp0.lo = 0;
-        rp0.hi = tailC;
-        rp0.acc_loc = acc;
-        rp0.dang_all = 1;
-        unsigned long long* d_c64;
-        GTS_TRY(c->buf(kBufRouteCnt, sizeof(unsigned long long) * kMaxRanks + (8 + 2 * kMaxRanks) * 4, (void**)&d_c64));
-        GTS_CUDA(cudaMemsetAsync(d_c64, 0, sizeof(unsigned long long) * kMaxRanks + (8 + 2 * kMaxRanks) * 4, s));
-        const void* kcount = g->weighted ? (const void*)route_count_kernel<true> : (const void*)route_count_kernel<false>;
-        int cgrid = 0;
-        GTS_TRY(sms_grid(c, kcount, kThreads, 0, &cgrid));
-        const uint32_t* dl0 = c->dg.all_local ? nullptr : c->dg.local_list;
-        GTS_TRY(sweep_pages(c, g, rc, false, &c->dg.h_local_list, dl0, c->dg.n_local, nullptr,
-                            [&](const PageSet& ps, int cap) -> int {
-                                GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
-                                void* ca[] = {(void*)&ps, (void*)&rp0, (void*)&n_hot, (void*)&d_c64, (void*)&ctr};
-                                GTS_CUDA(cudaLaunchKernel(kcount, dim3(std::min(cgrid, cap)), dim3(kThreads), ca, 0, s));
-                                ++launches;
-                                return GTS_OK;
-                            }, &ss));
-        std::vector<unsigned long long> cap(kMaxRanks);
-        GTS_CUDA(cudaMemcpyAsync(cap.data(), d_c64, kMaxRanks * 8, cudaMemcpyDeviceToHost, s));
-        GTS_CUDA(cudaStreamSynchronize(s));
-        uint64_t tot = 0;
-        std::vector<uint32_t> off(kMaxRanks);
-        for (int k = 0; k < kMaxRanks; ++k) {
-            off[k] = (uint32_t)tot;
-            rp0.send_off[k] = (uint32_t)tot;
-            rp0.send_cap[k] = (uint32_t)cap[k];
-            tot += cap[k];
-        }
-        if (tot >= (1ull << 32)) return fail(GTS_EOVERFLOW, "tail buffer exceeds 2^32 pairs");
-        GTS_TRY(c->buf(kBufRouteSend, std::max<uint64_t>(tot, 1) * 8, (void**)&t_send));
-        uint32_t* fl = reinterpret_cast<uint32_t*>(d_c64 + kMaxRanks);
-        rp0.overflow = fl;
-        t_cnt = fl + 8;
-        t_off = t_cnt + kMaxRanks;
-        GTS_CUDA(cudaMemcpyAsync(t_off, off.data(), kMaxRanks * 4, cudaMemcpyHostToDevice, s));
-        rp0.send = t_send;
-        rp0.send_cnt = t_cnt;
-    }
     if (!route) {
         const uint32_t* d_list = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
         for (uint32_t it = 0; it < iters; ++it) {
             double* D = dang + (it & 1);
             std::pair<cudaEvent_t, cudaEvent_t> ev;
-            if (t_send) GTS_CUDA(cudaMemsetAsync(t_cnt, 0, kMaxRanks * 4, s));
             GTS_TRY(sweep_pages(c, g, rc, streamed, &c->dg.h_local_list, d_list, c->dg.n_local, nullptr,
                                 [&](const PageSet& ps, int cap) -> int {
                                     return binned ? binned_scatter(ps, D) : scatter(ps, cap, D, rp0);
                                 }, &ss));
-            if (t_send) {           // deferred tail updates, bin by bin (same additions as Alg 4 l.16)
-                std::pair<cudaEvent_t, cudaEvent_t> e3;
-                if (timing) { e3 = c->t_main.next(); cudaEventRecord(e3.first, s); }
-                route_apply_kernel<<<c->num_sms * 8, 256, 0, s>>>(t_send, t_off, t_cnt, kMaxRanks, acc, 0);
-                if (timing) cudaEventRecord(e3.second, s);
-                GTS_CUDA(cudaGetLastError());
-                ++launches;
-            }
             if (c->world > 1) {         // Strategy-P: every replica receives the full sum
                 if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
                 GTS_NCCL(ncclGroupStart());

@@ -318,13 +318,10 @@ def test_degree_ordered_device_outputs(G, ctx):
 
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "instar", "multi"])
-@pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow", "tail"])
+@pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow"])
 def test_pagerank_ordered_variants(G, ctx, name, mode, monkeypatch):
     """Degree-ordered PageRank with and without the L2 persistence window (GTS_L2_PERSIST=0),
-    with the warp-window walk (record-start masks) instead of the tile walk, and with the
-    tail deferral (GTS_PR_TAIL: updates into IDs >= 60,000 binned and applied after the scatter)."""
-    if mode == "tail":
-        monkeypatch.setenv("GTS_PR_TAIL", "60000")
+    and with the warp-window walk (record-start masks) instead of the tile walk."""
     if mode == "nopersist":
         monkeypatch.setenv("GTS_L2_PERSIST", "0")
     if mode == "warpwindow":

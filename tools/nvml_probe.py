@@ -33,6 +33,13 @@ def loop():
         time.sleep(0.02)
 
 
+lat0 = []
+for _ in range(200):                       # control: no sampling thread
+    t = time.perf_counter()
+    b = a @ a
+    torch.cuda.synchronize()
+    lat0.append((time.perf_counter() - t) * 1e3)
+print("control matmul+sync ms: median", sorted(lat0)[len(lat0) // 2], "max", max(lat0))
 th = threading.Thread(target=loop)
 th.start()
 lat = []
