@@ -405,15 +405,17 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
 
 template <class Op, int kMicro = kMicroTile>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
-    const uint32_t count = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
+    const uint32_t S = ps.split;                 // >= 1 work items per page
+    const uint32_t count = (ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count) * S;
     const int tid = threadIdx.x;
     const uint64_t pol = policy_evict_first();
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
         __syncthreads();
-        const uint32_t i = sm.item;
+        const uint32_t item = sm.item;
         __syncthreads();
-        if (i >= count) break;
+        if (item >= count) break;
+        const uint32_t i = S == 1 ? item : item / S, sub = S == 1 ? 0u : item % S;
         uint32_t pid;
         const uint8_t* data;
         page_at(ps, i, pid, data);
@@ -425,16 +427,18 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             const uint32_t vid = ld32(end - kLpFooter - kSlotBytes);
             const uint32_t total = ld32(end - 16);
             const uint32_t len = ld32(data);
+            // slice `sub` of S of the chunk (high-degree split across CTAs)
+            const uint32_t klo = (uint32_t)((uint64_t)len * sub / S), khi = (uint32_t)((uint64_t)len * (sub + 1) / S);
             uint32_t payload = 0;
-            if (op.select_lp(vid, total, len, payload)) {
+            if (khi > klo && op.select_lp(vid, total, khi - klo, payload)) {
                 const uint32_t* adj = words + 1;
-                for (uint32_t k0 = tid; k0 < len; k0 += kThreads * kEdgesPerThread) {
+                for (uint32_t k0 = klo + tid; k0 < khi; k0 += kThreads * kEdgesPerThread) {
                     uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
                     bool valid[kEdgesPerThread];
 #pragma unroll
                     for (int q = 0; q < kEdgesPerThread; ++q) {
                         const uint32_t k = k0 + q * kThreads;
-                        valid[q] = k < len;
+                        valid[q] = k < khi;
                         dst[q] = valid[q] ? ld_stream_u32(adj + k, pol) : 0u;
                         w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_u32(adj + len + k, pol) : 0u;
                         pl[q] = payload;
@@ -445,6 +449,8 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     op.edges(dst, w, pl, src, valid);
                 }
             }
+        } else if (sub != 0) {
+            continue;                           // an SP is one work item (slice 0)
         } else if (kMicro != kMicroTile) {
             expand_sp_micro<Op, kMicro>(ps, op, data, end, nslots, pol);
         } else {

@@ -584,19 +584,28 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
             persist = true;
         }
     }
+    const char* spe = getenv("GTS_SPLIT");
+    const bool split_on = !spe || atoi(spe) > 0;
+    uint32_t cur_pages = (uint32_t)l0.size();       // pages in this level's list (host copy of the count)
     for (uint32_t L = 0;; ++L) {
         auto launch = [&](const PageSet& ps, int cap) -> int {
                                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+                                PageSet p2 = ps;
+                                p2.hybrid_deg = hybrid_deg;
+                                // few pages in this level (e.g. the source hub's LPs): slice LPs so
+                                // every CTA gets work (GTS_SPLIT=0 disables)
+                                const uint32_t pc = ps.d_count ? cur_pages : ps.count;
+                                const int gl = std::min(grid, cap);
+                                if (split_on && pc > 0 && 2 * pc < (uint32_t)gl)
+                                    p2.split = std::min<uint32_t>(64u, (uint32_t)gl / pc);
                                 if (algo == kBFS) {
-                                    PageSet p2 = ps;
-                                    p2.hybrid_deg = hybrid_deg;
-                                    bfs_kern<<<std::min(grid, cap), kThreads, 0, s>>>(
+                                    bfs_kern<<<gl, kThreads, 0, s>>>(
                                         p2, cur, visited, next, &ctr->work, &ctr->edges, vprefix);
                                 } else
-                                    sssp_kern<<<std::min(grid, cap), kThreads, 0, s>>>(
-                                        ps, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T);
+                                    sssp_kern<<<gl, kThreads, 0, s>>>(
+                                        p2, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T);
                                 if (timing) cudaEventRecord(ev.second, s);
                                 GTS_CUDA(cudaGetLastError());
                                 ++main_launches;
@@ -647,6 +656,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
             T = (uint32_t)std::min<uint64_t>(nt, 0xFFFFFFFEull);
         }
         pages_processed += h.list_count;
+        cur_pages = h.list_count;
         if (streamed) {                          // the host drives the copies: fetch and sort the page set
             h_list.resize(h.list_count);
             if (h.list_count) {

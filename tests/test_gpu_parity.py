@@ -132,6 +132,27 @@ def test_occupancy_variants(G, ctx, name, occ, monkeypatch):
         assert np.array_equal(G.gts_sssp(ctx, grw, src)[0], oracle.sssp(g.row_ptr, g.col, w, src))
 
 
+@pytest.mark.parametrize("name", ["fig1", "outstar", "instar", "rmat16_4k", "rmat16_256", "twitter20"])
+@pytest.mark.parametrize("split", ["0", "1"])
+def test_lp_slicing(G, ctx, name, split, monkeypatch):
+    """LP slicing for small page sets (GTS_SPLIT): BFS and SSSP from the max-degree
+    vertex (its LPs are the whole first level) and from vertex 0, resident and streamed,
+    bit-exact either way."""
+    monkeypatch.setenv("GTS_SPLIT", split)
+    g, pb = graph(name)
+    w = inputs.edge_weights(g)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
+    grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb)
+    for src in (int(np.argmax(np.diff(g.row_ptr))), 0):
+        want = oracle.bfs(g.row_ptr, g.col, src)
+        for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=2)):
+            got, st = G.gts_bfs(ctx, gr, src, **kw)
+            assert np.array_equal(got, want), (name, split, src, kw)
+            reached = want != oracle.UNREACHED
+            assert st["edges_traversed"] == int(np.diff(g.row_ptr)[reached].sum())
+            assert np.array_equal(G.gts_sssp(ctx, grw, src, **kw)[0], oracle.sssp(g.row_ptr, g.col, w, src))
+
+
 def test_bfs_deterministic_and_device_output(G, ctx):
     import torch
     g, pb = graph("rmat20")
