@@ -513,7 +513,12 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 uint32_t pos, nf, excl, total;
                 tile_scan(sel, sel ? deg : 0u, pos, nf, excl, total, sm);
                 const uint32_t W0 = sm.soff[0], W1 = sm.soff[nv];
-                if (2 * total >= W1 - W0 && ps.ww) {
+                // dense: the selected records' words are >= half of the tile's record region
+                // (weighted records hold 2 words per edge; ps.wdense = 0 restores the
+                // edges-only count, which made weighted tiles dense only when ~all selected)
+                const uint32_t selw = (Op::kWeighted && ps.wdense) ? 2 * total : total;
+                const bool dense = 2 * selw >= W1 - W0;
+                if (dense && ps.ww) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
                     // 128-word windows; owners from record-start masks (no binary search)
                     if (ps.entry_encoding == GTS_ENTRY_VID32)
@@ -523,7 +528,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     __syncthreads();
                     continue;
                 }
-                if (2 * total >= W1 - W0) {
+                if (dense) {
                     // dense tile: stream the whole record region with 16-byte loads and
                     // act on the words of selected owners (hybrid micro-level, App E)
                     const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;

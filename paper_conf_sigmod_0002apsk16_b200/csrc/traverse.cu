@@ -584,6 +584,8 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
             persist = true;
         }
     }
+    const char* wde = getenv("GTS_WDENSE");
+    const uint32_t wdense = (!wde || atoi(wde) > 0) ? 1u : 0u;
     const char* spe = getenv("GTS_SPLIT");
     const bool split_on = !spe || atoi(spe) > 0;
     uint32_t cur_pages = (uint32_t)l0.size();       // pages in this level's list (host copy of the count)
@@ -594,6 +596,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
                                 PageSet p2 = ps;
                                 p2.hybrid_deg = hybrid_deg;
+                                p2.wdense = wdense;
                                 // few pages in this level (e.g. the source hub's LPs): slice LPs so
                                 // every CTA gets work (GTS_SPLIT=0 disables)
                                 const uint32_t pc = ps.d_count ? cur_pages : ps.count;
