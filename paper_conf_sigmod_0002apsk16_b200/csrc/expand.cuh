@@ -184,6 +184,68 @@ __device__ __forceinline__ void gather_items(const PageSet& ps, Op& op, TileSmem
     }
 }
 
+// Same expansion by warp windows: the item edge space [0, total) is cut into
+// 128-edge windows, each warp walks a contiguous run of them, and the owner of
+// a lane's edges comes from an item-start mask (win_mask over sm.pre) instead of
+// a binary search per 4 edges.  Requires every item to have >= 1 edge (starts
+// are distinct).  The item data of the lane's first two owners is read once.
+template <class Op>
+__device__ __forceinline__ void gather_items_ww(const PageSet& ps, Op& op, TileSmem& sm, const uint32_t* words,
+                                                uint32_t nf, uint32_t total, uint64_t pol) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t nwin = (total + 127) >> 7;
+    const uint32_t per = (nwin + kWarps - 1) / kWarps;
+    const uint32_t wa = min(nwin, warp * per), wb = min(nwin, wa + per);
+    if (wa >= wb) return;
+    const uint32_t base0 = wa << 7;
+    int lo = -1, hi = (int)nf;                       // pre[lo] < base0 <= pre[hi]
+    while (hi - lo > 1) {
+        const int mid = (lo + hi) >> 1;
+        if (sm.pre[mid] < base0) lo = mid; else hi = mid;
+    }
+    int j0 = lo;
+    for (uint32_t wi = wa; wi < wb; ++wi) {
+        const uint32_t bw = wi << 7;
+        int ns;
+        const WinMask wm = win_mask(sm.pre, j0, nf, bw, ns);
+        const uint32_t mw = lane >> 3;
+        uint32_t before = 0;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) before += (uint32_t)k < mw ? __popc(wm.m[k]) : 0u;
+        const uint32_t mword = mw == 0 ? wm.m[0] : mw == 1 ? wm.m[1] : mw == 2 ? wm.m[2] : wm.m[3];
+        const uint32_t bpos0 = (4 * lane) & 31;
+        const uint32_t nb = (mword >> bpos0) & 0xFu;     // items starting at my edges
+        const int jb = j0 + (int)(before + __popc(mword & ((1u << bpos0) - 1u)));
+        // owners jb (if >= 0) and jb + 1
+        const int ja = jb < 0 ? 0 : jb;
+        const uint32_t preA = sm.pre[ja], offA = sm.off[ja], degA = sm.deg[ja], payA = sm.payload[ja], srcA = sm.src[ja];
+        const uint32_t preB = sm.pre[jb + 1], offB = sm.off[jb + 1], degB = sm.deg[jb + 1], payB = sm.payload[jb + 1],
+                       srcB = sm.src[jb + 1];
+        uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
+        bool valid[kEdgesPerThread];
+        uint32_t c = 0;
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            const uint32_t e = bw + 4 * lane + q;
+            c += (nb >> q) & 1u;
+            const int j = jb + (int)c;
+            valid[q] = e < total;
+            uint32_t pj, oj, dj;
+            if (c == 0) { pj = preA; oj = offA; dj = degA; pl[q] = payA; src[q] = srcA; }
+            else if (c == 1) { pj = preB; oj = offB; dj = degB; pl[q] = payB; src[q] = srcB; }
+            else { pj = sm.pre[j]; oj = sm.off[j]; dj = sm.deg[j]; pl[q] = sm.payload[j]; src[q] = sm.src[j]; }
+            const uint32_t* adj = words + oj;
+            const uint32_t local = e - pj;
+            dst[q] = valid[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
+            w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_l1_u32(adj + dj + local, pol) : 0u;
+        }
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) dst[q] = decode_entry(ps, dst[q]);
+        op.edges(dst, w, pl, src, valid);
+        j0 += ns;
+    }
+}
+
 // Sparse page (frontier-driven ops, < 1/4 of the page's vertices selected):
 // compact the page's frontier vertices from the bitmap in passes of
 // kListWords words, then expand them in batches of kTile with gather_items.
@@ -223,9 +285,10 @@ __device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, cons
             }
             const uint32_t v = start + j;
             const uint32_t pay = sel ? op.payload(v, deg) : 0u;
+            const bool item = sel && deg > 0;            // items with edges only
             uint32_t p2, nf, ex2, total;
-            tile_scan(sel, deg, p2, nf, ex2, total, sm);
-            if (sel) {
+            tile_scan(item, item ? deg : 0u, p2, nf, ex2, total, sm);
+            if (item) {
                 sm.off[p2] = off / 4 + 1;
                 sm.deg[p2] = deg;
                 sm.src[p2] = v;
@@ -234,7 +297,8 @@ __device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, cons
             }
             if (tid == 0) sm.pre[nf] = total;
             __syncthreads();
-            gather_items(ps, op, sm, words, nf, total, pol);
+            if (ps.ww & 2u) gather_items_ww(ps, op, sm, words, nf, total, pol);
+            else gather_items(ps, op, sm, words, nf, total, pol);
             __syncthreads();
         }
     }
@@ -379,16 +443,28 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
                 j0 += ns;
                 continue;
             }
+            // Weighted records (sz, adj[sz], w[sz]): a word is an entry iff it lies in
+            // the first sz words after its owner's header.  The lane's words have owners
+            // jb + c; the record bounds of jb and jb + 1 (all but a few lanes) are loaded
+            // once per lane, others on demand.
+            const uint32_t bpos0 = (4 * lane) & 31;
+            const uint32_t nb = (mword >> bpos0) & 0xFu;
+            const int jb = j0 + (int)(before + __popc(mword & ((1u << bpos0) - 1u)));
+            const uint32_t oA = jb >= 0 ? sm.soff[jb] : 0u;   // jb = -1: only words before W0 have c = 0
+            const uint32_t oB = sm.soff[jb + 1], oC = sm.soff[jb + 2];
+            uint32_t c = 0;
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
                 const uint32_t w = 4 * q + k;
-                const uint32_t bpos = (4 * lane + k) & 31;
-                const int j = j0 + (int)(before + __popc(mword & ((2u << bpos) - 1u)));
-                bool ok = w >= W0 && w < W1 && !((mword >> bpos) & 1u);
+                const uint32_t st = (nb >> k) & 1u;
+                c += st;
+                const int j = jb + (int)c;
+                bool ok = !st && w >= W0 && w < W1;
                 uint32_t dj = 0;
                 if (ok) {                              // adjacency words only, not the weights after them
-                    const uint32_t o = sm.soff[j];
-                    dj = (sm.soff[j + 1] - o - 1) >> wsh;
+                    const uint32_t o = c == 0 ? oA : c == 1 ? oB : sm.soff[j];
+                    const uint32_t oe = c == 0 ? oB : c == 1 ? oC : sm.soff[j + 1];
+                    dj = (oe - o - 1) >> wsh;
                     ok = w - o <= dj && sm.sel[j];
                 }
                 wt[k] = (Op::kReadWeights && ok) ? ld_stream_l1_u32(words + w + dj, pol) : 0u;
@@ -511,14 +587,17 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     sm.paytile[tid] = pay;
                 }
                 uint32_t pos, nf, excl, total;
-                tile_scan(sel, sel ? deg : 0u, pos, nf, excl, total, sm);
+                const bool item = sel && deg > 0;        // sparse tiles compact items with edges only
+                tile_scan(item, item ? deg : 0u, pos, nf, excl, total, sm);
                 const uint32_t W0 = sm.soff[0], W1 = sm.soff[nv];
-                // dense: the selected records' words are >= half of the tile's record region
-                // (weighted records hold 2 words per edge; ps.wdense = 0 restores the
-                // edges-only count, which made weighted tiles dense only when ~all selected)
-                const uint32_t selw = (Op::kWeighted && ps.wdense) ? 2 * total : total;
-                const bool dense = 2 * selw >= W1 - W0;
-                if (dense && ps.ww) {
+                // dense: the selected edges are >= half of the tile's record words.  Weighted
+                // records hold 2 words per edge, so there a tile is dense only when nearly
+                // every vertex is selected -- measured the better choice for SSSP (RMAT-27
+                // 35.7 ms vs 42.8 ms when the words are counted, ps.wdense = 1; ps.wdense = 2
+                // never streams weighted tiles)
+                const uint32_t selw = (Op::kWeighted && ps.wdense == 1) ? 2 * total : total;
+                const bool dense = 2 * selw >= W1 - W0 && !(Op::kWeighted && ps.wdense == 2);
+                if (dense && (ps.ww & 1u)) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
                     // 128-word windows; owners from record-start masks (no binary search)
                     if (ps.entry_encoding == GTS_ENTRY_VID32)
@@ -581,7 +660,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     continue;
                 }
                 // sparse tile: compacted selected vertices, edge-parallel gather
-                if (sel) {
+                if (item) {
                     sm.off[pos] = sm.soff[tid] + 1;
                     sm.deg[pos] = deg;
                     sm.src[pos] = v;
@@ -590,7 +669,8 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 }
                 if (tid == 0) sm.pre[nf] = total;
                 __syncthreads();
-                gather_items(ps, op, sm, words, nf, total, pol);
+                if (ps.ww & 2u) gather_items_ww(ps, op, sm, words, nf, total, pol);
+                else gather_items(ps, op, sm, words, nf, total, pol);
                 __syncthreads();
             }
         }

@@ -54,7 +54,7 @@ struct PageSet {
     const uint32_t* rvt_start; // START_VID per page (PID16 decode)
     uint32_t hybrid_deg = 8;   // GTS_MICRO_HYBRID: vertex-centric below this many edges per vertex (R24)
     uint32_t ww = 0;           // dense tiles by warp windows (expand.cuh dense_tile_ww)
-    uint32_t wdense = 1;       // weighted pages: count 2 words per selected edge in the dense-tile test
+    uint32_t wdense = 0;       // weighted pages' dense-tile test: 0 edges vs words, 1 words vs words, 2 never
     uint32_t split = 1;        // work items per page: an LP's chunk is cut into `split` slices
                                // (small page sets, e.g. a hub's LPs at BFS level 0); SPs use slice 0
 };
@@ -155,9 +155,12 @@ void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t
 
 // dense tiles by warp windows unless GTS_WW=0 (read per call so tests can switch it);
 // RMAT-27: SSSP 33.8 vs 36.2 ms, WCC 13.7 vs 14.2, BFS equal (profiles/r01_ww_dense.txt)
+// PageSet::ww bits: 1 = dense tiles by warp windows (GTS_WW=0 clears), 2 = sparse
+// tiles' item gather by warp windows (GTS_GWW=0 clears)
 inline uint32_t env_ww() {
     const char* e = getenv("GTS_WW");
-    return e && atoi(e) == 0 ? 0u : 1u;
+    const char* g = getenv("GTS_GWW");
+    return (e && atoi(e) == 0 ? 0u : 1u) | (g && atoi(g) == 0 ? 0u : 2u);
 }
 
 inline double now_s() {

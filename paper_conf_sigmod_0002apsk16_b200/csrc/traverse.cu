@@ -585,7 +585,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         }
     }
     const char* wde = getenv("GTS_WDENSE");
-    const uint32_t wdense = (!wde || atoi(wde) > 0) ? 1u : 0u;
+    const uint32_t wdense = wde ? (uint32_t)std::min(2, std::max(0, atoi(wde))) : 0u;
     const char* spe = getenv("GTS_SPLIT");
     const bool split_on = !spe || atoi(spe) > 0;
     uint32_t cur_pages = (uint32_t)l0.size();       // pages in this level's list (host copy of the count)

@@ -153,6 +153,40 @@ def test_lp_slicing(G, ctx, name, split, monkeypatch):
             assert np.array_equal(G.gts_sssp(ctx, grw, src, **kw)[0], oracle.sssp(g.row_ptr, g.col, w, src))
 
 
+@pytest.mark.parametrize("name", ["fig1", "rmat16_4k", "rmat16_64k", "rmat20", "twitter20", "bintree"])
+@pytest.mark.parametrize("wdense", ["0", "1", "2"])
+def test_weighted_dense_tiles(G, ctx, name, wdense, monkeypatch):
+    """Weighted pages under the three dense-tile tests (GTS_WDENSE): SSSP and BFS bit-exact,
+    warp-window and tile walks."""
+    monkeypatch.setenv("GTS_WDENSE", wdense)
+    g, pb = graph(name)
+    w = inputs.edge_weights(g)
+    src = _sources(g)[1]
+    for ww in ("1", "0"):
+        monkeypatch.setenv("GTS_WW", ww)
+        for order in (False, True):
+            grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb, order=order)
+            assert np.array_equal(G.gts_sssp(ctx, grw, src)[0], oracle.sssp(g.row_ptr, g.col, w, src))
+            assert np.array_equal(G.gts_bfs(ctx, grw, src)[0], oracle.bfs(g.row_ptr, g.col, src))
+
+
+@pytest.mark.parametrize("name", ["fig1", "multi", "path", "outstar", "rand", "rmat16_4k", "rmat16_256", "rmat20", "twitter20"])
+@pytest.mark.parametrize("gww", ["0", "1"])
+def test_sparse_gather_walks(G, ctx, name, gww, monkeypatch):
+    """Sparse tiles' item gather: per-thread binary search (GTS_GWW=0) or warp windows over
+    the item-start mask (GTS_GWW=1); BFS / SSSP / WCC bit-exact, natural and degree order."""
+    monkeypatch.setenv("GTS_GWW", gww)
+    g, pb = graph(name)
+    w = inputs.edge_weights(g)
+    for order in (False, True):
+        gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
+        grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb, order=order)
+        for src in _sources(g)[:3]:
+            assert np.array_equal(G.gts_bfs(ctx, gr, src)[0], oracle.bfs(g.row_ptr, g.col, src))
+            assert np.array_equal(G.gts_sssp(ctx, grw, src)[0], oracle.sssp(g.row_ptr, g.col, w, src))
+        assert np.array_equal(G.gts_wcc(ctx, gr)[0], oracle.wcc(g.row_ptr, g.col))
+
+
 def test_bfs_deterministic_and_device_output(G, ctx):
     import torch
     g, pb = graph("rmat20")
