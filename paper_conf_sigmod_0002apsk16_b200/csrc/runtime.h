@@ -155,12 +155,13 @@ void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t
 
 // dense tiles by warp windows unless GTS_WW=0 (read per call so tests can switch it);
 // RMAT-27: SSSP 33.8 vs 36.2 ms, WCC 13.7 vs 14.2, BFS equal (profiles/r01_ww_dense.txt)
-// PageSet::ww bits: 1 = dense tiles by warp windows (GTS_WW=0 clears), 2 = sparse
-// tiles' item gather by warp windows (GTS_GWW=0 clears)
+// PageSet::ww bits: 1 = dense tiles by warp windows (default; GTS_WW=0 clears), 2 =
+// sparse tiles' item gather by warp windows (opt-in GTS_GWW=1: RMAT-27 BFS 7.79 vs
+// 7.62 ms, SSSP 36.0 vs 36.3 ms, WCC 12.8 vs 12.7 ms against the binary search)
 inline uint32_t env_ww() {
     const char* e = getenv("GTS_WW");
     const char* g = getenv("GTS_GWW");
-    return (e && atoi(e) == 0 ? 0u : 1u) | (g && atoi(g) == 0 ? 0u : 2u);
+    return (e && atoi(e) == 0 ? 0u : 1u) | (g && atoi(g) > 0 ? 2u : 0u);
 }
 
 inline double now_s() {
