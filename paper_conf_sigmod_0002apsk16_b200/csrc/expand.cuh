@@ -481,8 +481,12 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
 
 template <class Op, int kMicro = kMicroTile>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
-    const uint32_t S = ps.split;                 // >= 1 work items per page
-    const uint32_t count = (ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count) * S;
+    const uint32_t npages = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
+    // work items per page: ps.split, or 0 = automatic: slice LPs when the set has fewer
+    // than half as many pages as the grid has CTAs (same value in every CTA)
+    const uint32_t S = ps.split ? ps.split
+                                : (npages > 0 && 2 * npages < gridDim.x ? min(64u, gridDim.x / npages) : 1u);
+    const uint32_t count = npages * S;
     const int tid = threadIdx.x;
     const uint64_t pol = policy_evict_first();
     for (;;) {

@@ -147,9 +147,13 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 template <bool W, int M = kMicroTile, int MB = 2>
 __global__ void __launch_bounds__(kThreads, MB)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
-                  uint32_t* work_ctr, unsigned long long* edges_out, uint32_t vprefix) {
+                  uint32_t* work_ctr, unsigned long long* edges_out, const unsigned int* vprefix_words,
+                  uint64_t n) {
     __shared__ TileSmem sm;
-    BfsOp<W> op{cur, visited, next, 0ull, vprefix};
+    // all-visited prefix from the previous level's visited_prefix_kernel (device-side,
+    // so levels can be enqueued without a host round trip)
+    const uint64_t vw = min((uint64_t)*vprefix_words, (n + 31) / 32);
+    BfsOp<W> op{cur, visited, next, 0ull, (uint32_t)min(vw * 32, n)};
     expand_pages<BfsOp<W>, M>(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
@@ -418,7 +422,7 @@ struct Counters {               // device scratch, slot kCtr
     unsigned int vprefix_words;    // BFS: all-visited prefix of the bitmap (words)
 };
 
-enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather, kBufLvSlots, kBufLv8 };
+enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather, kBufLvSlots, kBufLv8, kBufLvCnt };
 
 // deliver() for byte levels of a degree-ordered graph: out[v] = lv8[new_of_old[v]]
 static int deliver_levels8(Context* c, const Graph* g, const uint8_t* lv8, bool nibbles, void* out,
@@ -561,7 +565,6 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     SweepStats ss;
     std::vector<uint32_t> h_list = l0;             // streamed mode: this level's pages on the host (ascending)
     const bool cached = streamed && rc.cache_mib > 0;
-    uint32_t vprefix = 0;
     // SSSP near-far bucketing: expand only pending vertices with dist <= T; T
     // advances by delta past the nearest pending distance when no pending vertex
     // is within it.  Label-correcting, so any delta gives the exact distances.
@@ -588,7 +591,23 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     const uint32_t wdense = wde ? (uint32_t)std::min(2, std::max(0, atoi(wde))) : 0u;
     const char* spe = getenv("GTS_SPLIT");
     const bool split_on = !spe || atoi(spe) > 0;
-    uint32_t cur_pages = (uint32_t)l0.size();       // pages in this level's list (host copy of the count)
+    // BFS on resident pages, one rank: levels are enqueued GTS_BFS_BATCH (default 8) at a
+    // time without a host round trip (per-level new-vertex counts and page-list counts go
+    // to device arrays; the levels after the last non-empty one run on an empty frontier)
+    const char* bbe = getenv("GTS_BFS_BATCH");
+    const uint32_t B = (algo == kBFS && !streamed && c->world == 1 && K > 0)
+                           ? (uint32_t)std::max(1L, bbe ? atol(bbe) : 8L) : 1u;
+    unsigned long long* lvl_cnt = nullptr;           // [K] new vertices per level (BFS)
+    uint32_t* lvl_pages = nullptr;                   // [K] pages in the list of level L
+    if (algo == kBFS) {
+        const uint32_t nl = std::max<uint32_t>(K, 1) + 1;
+        GTS_TRY(c->buf(kBufLvCnt, (size_t)nl * 12, (void**)&lvl_cnt));
+        lvl_pages = reinterpret_cast<uint32_t*>(lvl_cnt + nl);
+        GTS_CUDA(cudaMemsetAsync(lvl_cnt, 0, (size_t)nl * 12, s));
+    }
+    std::vector<unsigned long long> h_cnt;
+    std::vector<uint32_t> h_pages;
+    uint32_t synced = 0;                             // levels whose counts the host has read
     for (uint32_t L = 0;; ++L) {
         auto launch = [&](const PageSet& ps, int cap) -> int {
                                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
@@ -598,14 +617,12 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                 p2.hybrid_deg = hybrid_deg;
                                 p2.wdense = wdense;
                                 // few pages in this level (e.g. the source hub's LPs): slice LPs so
-                                // every CTA gets work (GTS_SPLIT=0 disables)
-                                const uint32_t pc = ps.d_count ? cur_pages : ps.count;
+                                // every CTA gets work, decided on the device (GTS_SPLIT=0 disables)
+                                p2.split = split_on ? 0u : 1u;
                                 const int gl = std::min(grid, cap);
-                                if (split_on && pc > 0 && 2 * pc < (uint32_t)gl)
-                                    p2.split = std::min<uint32_t>(64u, (uint32_t)gl / pc);
                                 if (algo == kBFS) {
                                     bfs_kern<<<gl, kThreads, 0, s>>>(
-                                        p2, cur, visited, next, &ctr->work, &ctr->edges, vprefix);
+                                        p2, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n);
                                 } else
                                     sssp_kern<<<gl, kThreads, 0, s>>>(
                                         p2, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T);
@@ -631,7 +648,8 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         GTS_CUDA(cudaMemsetAsync(&ctr->list_count, 0, 4, s));
         if (algo == kBFS) {
             frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, next,
-                                                            visited, slots ? nullptr : value, L + 1, &ctr->count);
+                                                            visited, slots ? nullptr : value, L + 1,
+                                                            L < K ? lvl_cnt + L : &ctr->count);
             GTS_CUDA(cudaMemsetAsync(&ctr->vprefix_words, 0xFF, 4, s));
             visited_prefix_kernel<<<fin_grid, 256, 0, s>>>(visited, words, &ctr->vprefix_words);
             ++launches;
@@ -648,18 +666,51 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         if (timing) cudaEventRecord(ev.second, s);
         launches += 2;
         GTS_CUDA(cudaGetLastError());
-        GTS_CUDA(cudaMemcpyAsync(&h, ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
-        GTS_CUDA(cudaStreamSynchronize(s));
+        if (algo == kBFS && L < K)                    // pages of level L+1's list (lvl_pages has K+1 entries)
+            GTS_CUDA(cudaMemcpyAsync(lvl_pages + L + 1, &ctr->list_count, 4, cudaMemcpyDeviceToDevice, s));
         ++levels;
-        if (algo == kBFS)
-            vprefix = (uint32_t)std::min<uint64_t>((uint64_t)std::min<uint64_t>(h.vprefix_words, words) * 32, n);
+        // host round trip: every level (SSSP, streamed, multi-rank), else every B levels and
+        // before the level slots run out
+        const bool sync = B == 1 || (L + 1) % B == 0 || !(slots && L + 3 < K);
+        if (!sync) {
+            if (slots && L + 2 < K) {
+                cur = next;
+                next = lvb + (uint64_t)(L + 2) * words;
+                GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
+                continue;
+            }
+        }
+        GTS_CUDA(cudaMemcpyAsync(&h, ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
+        if (algo == kBFS && L < K) {
+            h_cnt.resize(L + 1);
+            h_pages.resize(L + 2);
+            GTS_CUDA(cudaMemcpyAsync(h_cnt.data() + synced, lvl_cnt + synced, (size_t)(L + 1 - synced) * 8,
+                                     cudaMemcpyDeviceToHost, s));
+            GTS_CUDA(cudaMemcpyAsync(h_pages.data() + synced + 1, lvl_pages + synced + 1, (size_t)(L + 1 - synced) * 4,
+                                     cudaMemcpyDeviceToHost, s));
+        }
+        GTS_CUDA(cudaStreamSynchronize(s));
+        if (algo == kBFS && L < K) {
+            bool done = false;
+            for (uint32_t l = synced; l <= L; ++l) {
+                if (h_cnt[l] == 0) {                  // level l discovered nothing: BFS ends there
+                    levels = l + 1;
+                    done = true;
+                    break;
+                }
+                pages_processed += h_pages[l + 1];
+            }
+            synced = L + 1;
+            h.count = done ? 0 : h_cnt[L];
+            h.list_count = h_pages[L + 1];
+            if (done) break;
+        }
         if (h.count == 0) break;
         if (algo == kSSSP && h.near == 0) {      // nothing pending within T: open the next bucket
             const uint64_t nt = (uint64_t)h.minpend + delta;
             T = (uint32_t)std::min<uint64_t>(nt, 0xFFFFFFFEull);
         }
-        pages_processed += h.list_count;
-        cur_pages = h.list_count;
+        if (algo != kBFS || L >= K) pages_processed += h.list_count;
         if (streamed) {                          // the host drives the copies: fetch and sort the page set
             h_list.resize(h.list_count);
             if (h.list_count) {
@@ -960,8 +1011,8 @@ static int betweenness(gts_context* c, const gts_graph* g, const uint64_t* sourc
                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, 0u);
-                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, 0u);
+                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n);
+                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n);
                 if (timing) cudaEventRecord(ev.second, s);
                 GTS_CUDA(cudaGetLastError());
                 ++main_launches;

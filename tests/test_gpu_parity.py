@@ -99,19 +99,26 @@ def test_bfs_pid16_entries(G, ctx, name):
 
 @pytest.mark.parametrize("name", ["fig1", "path", "bintree", "rmat16_4k", "rmat20", "twitter20"])
 @pytest.mark.parametrize("k", ["0", "3", "5", "64"])
-def test_bfs_level_slots(G, ctx, name, k, monkeypatch):
+@pytest.mark.parametrize("batch", ["1", "3", "8"])
+def test_bfs_level_slots(G, ctx, name, k, batch, monkeypatch):
     """Level-slot LV construction (GTS_BFS_SLOTS=K): LV written once from the per-level
     frontier bitmaps; traversals deeper than K switch to per-level LV writes mid-way.
-    K=0 is per-level writes throughout.  Resident, streamed and degree-ordered pages."""
+    K=0 is per-level writes throughout.  Levels enqueued GTS_BFS_BATCH at a time between
+    host round trips.  Resident, streamed and degree-ordered pages; edge and level counts."""
     monkeypatch.setenv("GTS_BFS_SLOTS", k)
+    monkeypatch.setenv("GTS_BFS_BATCH", batch)
     g, pb = graph(name)
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
     go = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
     for src in _sources(g)[:2]:
         want = oracle.bfs(g.row_ptr, g.col, src)
+        reached = want != oracle.UNREACHED
+        depth = int(want[reached].max()) + 1
         for gg, kw in ((gr, {}), (go, {}), (gr, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3))):
             got, st = G.gts_bfs(ctx, gg, src, **kw)
             assert np.array_equal(got, want), (name, k, src, kw, int(np.sum(got != want)))
+            assert st["levels_or_iters"] == depth, (st["levels_or_iters"], depth)
+            assert st["edges_traversed"] == int(np.diff(g.row_ptr)[reached].sum())
 
 
 @pytest.mark.parametrize("name", ["fig1", "rmat16_4k", "rmat20", "twitter20", "instar"])
