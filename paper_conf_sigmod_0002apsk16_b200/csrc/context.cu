@@ -351,10 +351,13 @@ __global__ void label_min_kernel(uint32_t* minorig, const uint32_t* __restrict__
     if (cl != 0xFFFFFFFFu) label_min_flush(minorig, cl, cm);
 }
 
-__global__ void label_map_kernel(uint32_t* tmp, const uint32_t* __restrict__ label, const uint32_t* __restrict__ minorig,
-                                 uint64_t n) {
+// label_map + gather in one pass: out[v] = minorig[label[new_of_old[v]]] (caller order)
+__global__ void label_gather_kernel(uint32_t* out, const uint32_t* __restrict__ label,
+                                    const uint32_t* __restrict__ minorig, const uint32_t* __restrict__ idx,
+                                    uint64_t n) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) tmp[i] = minorig[label[i]];
+    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+        out[v] = minorig[label[idx[v]]];
 }
 
 int ensure_old_of_new(Context* c, const Graph* g, const uint32_t** out) {
@@ -370,22 +373,19 @@ int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_
     const uint64_t n = g->n;
     if (!g->ordered) return copy_out(c, vals, out, n * 4, out_location);
     const int eg = c->num_sms * 4;
-    const uint32_t* src = vals;
+    uint32_t* minorig = nullptr;
     if (labels) {             // internal min-ID label -> min caller VID of the component
         const uint32_t* onew;
         GTS_TRY(ensure_old_of_new(c, g, &onew));
-        uint32_t *minorig, *tmp;
         GTS_TRY(c->buf(70, n * 4, (void**)&minorig));
-        GTS_TRY(c->buf(71, n * 4, (void**)&tmp));
         GTS_CUDA(cudaMemsetAsync(minorig, 0xFF, n * 4, c->stream));
         label_min_kernel<<<eg, 256, 0, c->stream>>>(minorig, vals, c->dg.old_of_new, n);
-        label_map_kernel<<<eg, 256, 0, c->stream>>>(tmp, vals, minorig, n);
-        src = tmp;
     }
     uint32_t* dst;
     if (out_location == GTS_OUT_DEVICE) dst = static_cast<uint32_t*>(out);
     else GTS_TRY(c->buf(72, n * 4, (void**)&dst));
-    gather_kernel<<<eg, 256, 0, c->stream>>>(dst, src, c->dg.new_of_old, n);
+    if (labels) label_gather_kernel<<<eg, 256, 0, c->stream>>>(dst, vals, minorig, c->dg.new_of_old, n);
+    else gather_kernel<<<eg, 256, 0, c->stream>>>(dst, vals, c->dg.new_of_old, n);
     GTS_CUDA(cudaGetLastError());
     if (out_location == GTS_OUT_DEVICE) {
         GTS_CUDA(cudaStreamSynchronize(c->stream));
