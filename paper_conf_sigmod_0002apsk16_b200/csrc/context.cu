@@ -12,6 +12,7 @@
 #include <cstring>
 #include <new>
 
+#include "memops.cuh"
 #include "runtime.h"
 
 namespace gts {
@@ -323,8 +324,7 @@ int copy_out(Context* c, const void* dsrc, void* dst, size_t bytes, uint32_t out
 
 __global__ void gather_kernel(uint32_t* out, const uint32_t* __restrict__ vals, const uint32_t* __restrict__ idx,
                               uint64_t n) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) out[v] = vals[idx[v]];
+    gather_x4(out, idx, n, [&](uint32_t i) { return __ldg(vals + i); });
 }
 
 // min caller VID per component.  Each thread folds runs of equal labels in a
@@ -355,9 +355,7 @@ __global__ void label_min_kernel(uint32_t* minorig, const uint32_t* __restrict__
 __global__ void label_gather_kernel(uint32_t* out, const uint32_t* __restrict__ label,
                                     const uint32_t* __restrict__ minorig, const uint32_t* __restrict__ idx,
                                     uint64_t n) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
-        out[v] = minorig[label[idx[v]]];
+    gather_x4(out, idx, n, [&](uint32_t i) { return __ldg(minorig + __ldg(label + i)); });
 }
 
 int ensure_old_of_new(Context* c, const Graph* g, const uint32_t** out) {
@@ -384,8 +382,8 @@ int deliver(Context* c, const Graph* g, const uint32_t* vals, void* out, uint32_
     uint32_t* dst;
     if (out_location == GTS_OUT_DEVICE) dst = static_cast<uint32_t*>(out);
     else GTS_TRY(c->buf(72, n * 4, (void**)&dst));
-    if (labels) label_gather_kernel<<<eg, 256, 0, c->stream>>>(dst, vals, minorig, c->dg.new_of_old, n);
-    else gather_kernel<<<eg, 256, 0, c->stream>>>(dst, vals, c->dg.new_of_old, n);
+    if (labels) label_gather_kernel<<<2 * eg, 256, 0, c->stream>>>(dst, vals, minorig, c->dg.new_of_old, n);
+    else gather_kernel<<<2 * eg, 256, 0, c->stream>>>(dst, vals, c->dg.new_of_old, n);
     GTS_CUDA(cudaGetLastError());
     if (out_location == GTS_OUT_DEVICE) {
         GTS_CUDA(cudaStreamSynchronize(c->stream));

@@ -348,21 +348,18 @@ __global__ void level_fill4_kernel(uint8_t* lv4, const uint32_t* __restrict__ sl
 
 __global__ void gather4_kernel(uint32_t* out, const uint8_t* __restrict__ lv4, const uint32_t* __restrict__ idx,
                                uint64_t n) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
-        const uint32_t i = idx[v];
-        const uint32_t l = (lv4[i >> 1] >> (4 * (i & 1))) & 0xFu;
-        out[v] = l == 0xFu ? GTS_UNREACHED : l;
-    }
+    gather_x4(out, idx, n, [&](uint32_t i) {
+        const uint32_t l = (__ldg(lv4 + (i >> 1)) >> (4 * (i & 1))) & 0xFu;
+        return l == 0xFu ? GTS_UNREACHED : l;
+    });
 }
 
 __global__ void gather8_kernel(uint32_t* out, const uint8_t* __restrict__ lv8, const uint32_t* __restrict__ idx,
                                uint64_t n) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
-        const uint32_t l = lv8[idx[v]];
-        out[v] = l == 0xFFu ? GTS_UNREACHED : l;
-    }
+    gather_x4(out, idx, n, [&](uint32_t i) {
+        const uint32_t l = __ldg(lv8 + i);
+        return l == 0xFFu ? GTS_UNREACHED : l;
+    });
 }
 
 // Length of the all-visited prefix of the bitmap, in words: the first word that
@@ -431,8 +428,8 @@ static int deliver_levels8(Context* c, const Graph* g, const uint8_t* lv8, bool 
     uint32_t* dst;
     if (out_location == GTS_OUT_DEVICE) dst = static_cast<uint32_t*>(out);
     else GTS_TRY(c->buf(72, n * 4, (void**)&dst));     // deliver()'s staging slot
-    if (nibbles) gather4_kernel<<<c->num_sms * 4, 256, 0, c->stream>>>(dst, lv8, c->dg.new_of_old, n);
-    else gather8_kernel<<<c->num_sms * 4, 256, 0, c->stream>>>(dst, lv8, c->dg.new_of_old, n);
+    if (nibbles) gather4_kernel<<<c->num_sms * 8, 256, 0, c->stream>>>(dst, lv8, c->dg.new_of_old, n);
+    else gather8_kernel<<<c->num_sms * 8, 256, 0, c->stream>>>(dst, lv8, c->dg.new_of_old, n);
     GTS_CUDA(cudaGetLastError());
     if (out_location == GTS_OUT_DEVICE) {
         GTS_CUDA(cudaStreamSynchronize(c->stream));

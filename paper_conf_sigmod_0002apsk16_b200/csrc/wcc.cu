@@ -178,9 +178,31 @@ __global__ void wcc_giant_kernel(const uint32_t* parent, uint64_t n, uint32_t* g
 }
 
 // every vertex points at its root (the component's minimum VID)
+// Four consecutive vertices per thread per step, their root walks interleaved
+// so four pointer-chasing reads are in flight (one per vertex per hop).
 __global__ void wcc_finalize_kernel(uint32_t* parent, uint64_t n) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t n4 = n >> 2;
+    uint4* p4 = reinterpret_cast<uint4*>(parent);
+    for (uint64_t q = t; q < n4; q += stride) {
+        const uint4 v = __ldcg(p4 + q);
+        uint32_t r[4] = {v.x, v.y, v.z, v.w};
+        bool more = true;
+        while (more) {
+            uint32_t p[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) p[k] = __ldcg(parent + r[k]);
+            more = false;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                more |= p[k] != r[k];
+                r[k] = p[k];
+            }
+        }
+        p4[q] = make_uint4(r[0], r[1], r[2], r[3]);
+    }
+    for (uint64_t i = 4 * n4 + t; i < n; i += stride) {
         uint32_t r = __ldcg(parent + i);
         while (r != __ldcg(parent + r)) r = __ldcg(parent + r);
         parent[i] = r;
