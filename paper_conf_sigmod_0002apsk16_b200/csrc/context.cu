@@ -337,9 +337,9 @@ __device__ __forceinline__ void label_min_flush(uint32_t* minorig, uint32_t l, u
 __global__ void label_min_kernel(uint32_t* minorig, const uint32_t* __restrict__ label,
                                  const uint32_t* __restrict__ old_of_new, uint64_t n) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     uint32_t cl = 0xFFFFFFFFu, cm = 0xFFFFFFFFu;
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-        const uint32_t l = label[i], o = old_of_new[i];
+    auto fold = [&](uint32_t l, uint32_t o) {
         if (l == cl) {
             cm = min(cm, o);
         } else {
@@ -347,7 +347,20 @@ __global__ void label_min_kernel(uint32_t* minorig, const uint32_t* __restrict__
             cl = l;
             cm = o;
         }
+    };
+    // four consecutive vertices per step with 16-byte loads; the tail (or
+    // everything, if an array is not 16-byte aligned) element by element
+    const bool al = ((((uintptr_t)label) | ((uintptr_t)old_of_new)) & 15u) == 0;
+    const uint64_t n4 = al ? n >> 2 : 0;
+    for (uint64_t q = t; q < n4; q += stride) {
+        const uint4 l = __ldcs(reinterpret_cast<const uint4*>(label) + q);
+        const uint4 o = __ldcs(reinterpret_cast<const uint4*>(old_of_new) + q);
+        fold(l.x, o.x);
+        fold(l.y, o.y);
+        fold(l.z, o.z);
+        fold(l.w, o.w);
     }
+    for (uint64_t i = 4 * n4 + t; i < n; i += stride) fold(label[i], old_of_new[i]);
     if (cl != 0xFFFFFFFFu) label_min_flush(minorig, cl, cm);
 }
 

@@ -1306,7 +1306,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                 nccl_bytes += n * 4 + 8;
             }
             if (timing) { ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
-            pr_finish_kernel<<<eg, 256, 0, s>>>(x, acc, n, 0, n, damping, D, dang + ((it + 1) & 1),
+            pr_finish_kernel<<<2 * eg, 256, 0, s>>>(x, acc, n, 0, n, damping, D, dang + ((it + 1) & 1),
                                                  dangling == GTS_DANGLING_UNIFORM ? 1 : 0, 0);
             if (timing) cudaEventRecord(ev.second, s);
             ++launches;
@@ -1490,7 +1490,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
             }
             if (timing) { cudaEventRecord(ev.second, s); ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
             const uint64_t flo = virt ? 0 : vr[me], fhi = virt ? n : vr[me + 1];
-            pr_finish_kernel<<<eg, 256, 0, s>>>(x, acc, n, flo, fhi, damping, D, dang + ((it + 1) & 1),
+            pr_finish_kernel<<<2 * eg, 256, 0, s>>>(x, acc, n, flo, fhi, damping, D, dang + ((it + 1) & 1),
                                                  dangling == GTS_DANGLING_UNIFORM ? 1 : 0, 0);
             if (timing) cudaEventRecord(ev.second, s);
             ++launches;

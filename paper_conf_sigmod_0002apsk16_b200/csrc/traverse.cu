@@ -739,7 +739,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     const bool nib = levels < 15;
     if (slots && g->ordered && nib) {
         GTS_TRY(c->buf(kBufLv8, words * 32, (void**)&lv8));
-        level_fill4_kernel<<<fin_grid, 256, 0, s>>>(lv8, lvb, levels, words);
+        level_fill4_kernel<<<2 * fin_grid, 256, 0, s>>>(lv8, lvb, levels, words);
         GTS_CUDA(cudaGetLastError());
         launches += 2;
     } else if (slots && g->ordered && levels < 255) {
