@@ -379,6 +379,29 @@ def test_degree_ordered_device_outputs(G, ctx):
     _pr_check(f.cpu().numpy(), oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, "ordered-device")
 
 
+@pytest.mark.parametrize("name", ["rmat16_4k", "instar", "multi"])
+def test_degree_ordered_unaligned_device_outputs(G, ctx, name):
+    """Caller-order gathers into a device output 4 bytes past a 16-byte boundary
+    (the scalar fallback of gather_x4) and into an aligned one whose length is not
+    a multiple of 4 (the tail): every result equals the oracle."""
+    import torch
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+    w = inputs.edge_weights(g)
+    grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb, order=True)
+    for off in (1, 0):
+        d = torch.empty(g.n + 1, dtype=torch.int32, device="cuda")[off:off + g.n]
+        G.gts_bfs(ctx, gr, 0, out=d)
+        assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.bfs(g.row_ptr, g.col, 0)), (name, off)
+        G.gts_sssp(ctx, grw, 0, out=d)
+        assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.sssp(g.row_ptr, g.col, w, 0)), (name, off)
+        G.gts_wcc(ctx, gr, out=d)
+        assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.wcc(g.row_ptr, g.col)), (name, off)
+        f = torch.empty(g.n + 1, dtype=torch.float32, device="cuda")[off:off + g.n]
+        G.gts_pagerank(ctx, gr, 10, out=f)
+        _pr_check(f.cpu().numpy(), oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, "unaligned", off))
+
+
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "instar", "multi"])
 @pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow"])
 def test_pagerank_ordered_variants(G, ctx, name, mode, monkeypatch):
