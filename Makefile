@@ -12,12 +12,12 @@ NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 --expt-relaxed-constexpr -Xcompiler
             -Iinclude -I$(CSRC) -I$(NCCL_DIR)/include -Xptxas -v
 CU_SRC   := $(CSRC)/context.cu $(CSRC)/traverse.cu $(CSRC)/pagerank.cu $(CSRC)/wcc.cu
 CPP_SRC  := $(CSRC)/builder.cpp $(CSRC)/capi.cpp
-HDRS     := include/gts.h $(CSRC)/gts_internal.h $(CSRC)/runtime.h $(CSRC)/expand.cuh
+HDRS     := include/gts.h $(wildcard $(CSRC)/*.h) $(wildcard $(CSRC)/*.cuh)
 OBJDIR   := build/obj
 CU_OBJ   := $(patsubst $(CSRC)/%.cu,$(OBJDIR)/%.o,$(CU_SRC))
 CPP_OBJ  := $(patsubst $(CSRC)/%.cpp,$(OBJDIR)/%.o,$(CPP_SRC))
 
-all: $(LIBDIR)/libgts.so oracle/liboracle.so inputs/libgtsgen.so
+all: $(LIBDIR)/libgts.so oracle/liboracle.so oracle/liboracle_omp.so inputs/libgtsgen.so
 
 $(OBJDIR)/%.o: $(CSRC)/%.cu $(HDRS)
 	@mkdir -p $(OBJDIR)
@@ -35,10 +35,13 @@ $(LIBDIR)/libgts.so: $(CU_OBJ) $(CPP_OBJ)
 oracle/liboracle.so: oracle/oracle.c
 	gcc -O2 -fPIC -shared -o $@ $<
 
+oracle/liboracle_omp.so: oracle/oracle.c
+	gcc -O2 -fopenmp -fPIC -shared -o $@ $<
+
 inputs/libgtsgen.so: inputs/gen.c
 	gcc -O3 -march=x86-64-v2 -fopenmp -fPIC -shared -o $@ $< -lm
 
 clean:
-	rm -rf build $(LIBDIR) oracle/liboracle.so inputs/libgtsgen.so
+	rm -rf build $(LIBDIR) oracle/liboracle.so oracle/liboracle_omp.so inputs/libgtsgen.so
 
 .PHONY: all clean

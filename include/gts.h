@@ -67,7 +67,7 @@ typedef enum {
     GTS_ECUDA = -3,         /* CUDA runtime error or no usable device */
     GTS_ENCCL = -4,         /* NCCL error (world_size > 1) */
     GTS_EUNSUPPORTED = -5,  /* valid but unsupported combination (e.g. SSSP on an unweighted graph) */
-    GTS_EOVERFLOW = -6      /* n > 2^32, a degree >= 2^32, SSSP distance >= 2^32-1, PID16 limits */
+    GTS_EOVERFLOW = -6      /* n >= 2^32, a degree >= 2^32, SSSP distance >= 2^32-1, PID16 limits */
 } gts_status;
 
 enum { GTS_PAGE_SP = 0, GTS_PAGE_LP = 1 };
@@ -137,7 +137,7 @@ typedef struct gts_graph gts_graph;   /* opaque; owns the host pages + directory
  * VIDs < n; weights: m values or NULL (a weighted graph is required by
  * gts_sssp).  cfg may be NULL (defaults).  The graph owns a copy of
  * everything; inputs may be freed on return.  Pure host code (no CUDA call).
- * Errors: EINVAL (bad CSR / config), EOVERFLOW (n > 2^32, degree >= 2^32,
+ * Errors: EINVAL (bad CSR / config), EOVERFLOW (n >= 2^32, degree >= 2^32,
  * PID16 limits: > 65536 pages or > 65536 slots per page), ENOMEM. */
 int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, const uint32_t* col_idx,
                     const uint32_t* weights, const gts_page_config* cfg, gts_graph** out);

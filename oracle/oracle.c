@@ -1,8 +1,8 @@
 /*
  * oracle/oracle.c -- TEST INFRASTRUCTURE ONLY.
  *
- * A plain, slow, single-threaded CPU implementation of what the GTS hot path
- * computes, over CSR (never over the slotted pages, except the page decoder at
+ * A plain, slow CPU implementation of what the GTS hot path computes, over
+ * CSR (never over the slotted pages, except the page decoder at
  * the bottom, which reads page bytes by the format's definition).  It shares
  * no code, header, table or constant generator with the CUDA path
  * (paper_conf_sigmod_0002apsk16_b200/csrc) and neither side includes the
@@ -15,10 +15,20 @@
  * Every function here is pinned by tests/test_oracle_*.py to something other
  * than itself (brute force, closed forms, scipy / networkx / numpy library
  * routines, invariants); see DESIGN.md "Oracle pins".
+ *
+ * Built twice: liboracle.so (plain, single-threaded: the
+ * pragmas below are ignored) and liboracle_omp.so (-fopenmp).  The OpenMP
+ * pragmas only split loops whose iterations write disjoint outputs, each
+ * computed in the same fixed order as the plain build (PageRank: y[v] sums
+ * its in-edges in ascending u), so the two builds are byte-identical
+ * (tests/test_oracle_pagerank.py::test_openmp_build_byte_identical).
  */
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 #define UNREACHED 0xFFFFFFFFu
 
@@ -49,6 +59,72 @@ int oracle_bfs(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, uint64_
     }
     free(queue);
     return 0;
+}
+
+/* Level-synchronous BFS: the same hop levels as oracle_bfs, organised the way
+ * Alg 1 drives the GPU (level by level, every vertex of the current
+ * level L sets its unvisited out-neighbours to L+1, Alg 2 lines 17-18).  The
+ * level sets are unique, so the result equals the FIFO-queue BFS (pinned in
+ * tests/test_oracle_bfs.py).  Written so the OpenMP build splits each level's
+ * frontier over the host cores (the all-core CPU baseline of SURVEY 8(d)): a
+ * compare-and-swap on level[v] lets exactly one discoverer append v to the
+ * next frontier. */
+int oracle_bfs_levelsync(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, uint64_t src,
+                         uint32_t* level /* n */) {
+    if (src >= n) return -1;
+    for (uint64_t v = 0; v < n; ++v) level[v] = UNREACHED;
+    uint32_t* cur = (uint32_t*)malloc((n ? n : 1) * sizeof(uint32_t));
+    uint32_t* nxt = (uint32_t*)malloc((n ? n : 1) * sizeof(uint32_t));
+    if (!cur || !nxt) return -2;
+    level[src] = 0;
+    cur[0] = (uint32_t)src;
+    uint64_t ncur = 1;
+    for (uint32_t L = 0; ncur > 0; ++L) {
+        uint64_t nnext = 0;
+        #pragma omp parallel
+        {
+            uint32_t buf[1024];
+            uint64_t nb = 0;
+            #pragma omp for schedule(dynamic, 64)
+            for (uint64_t i = 0; i < ncur; ++i) {
+                uint32_t u = cur[i];
+                for (uint64_t k = row_ptr[u]; k < row_ptr[u + 1]; ++k) {
+                    uint32_t v = col[k];
+                    if (level[v] == UNREACHED && __sync_bool_compare_and_swap(&level[v], UNREACHED, L + 1)) {
+                        buf[nb++] = v;
+                        if (nb == 1024) {
+                            uint64_t at = __atomic_fetch_add(&nnext, nb, __ATOMIC_RELAXED);
+                            memcpy(nxt + at, buf, nb * sizeof(uint32_t));
+                            nb = 0;
+                        }
+                    }
+                }
+            }
+            if (nb) {
+                uint64_t at = __atomic_fetch_add(&nnext, nb, __ATOMIC_RELAXED);
+                memcpy(nxt + at, buf, nb * sizeof(uint32_t));
+            }
+        }
+        uint32_t* t = cur; cur = nxt; nxt = t;
+        ncur = nnext;
+    }
+    free(cur); free(nxt);
+    return 0;
+}
+
+/* Threads the OpenMP build runs with (1 in the plain build). */
+int oracle_num_threads(void) {
+#ifdef _OPENMP
+    int t = 1;
+    #pragma omp parallel
+    {
+        #pragma omp single
+        t = omp_get_num_threads();
+    }
+    return t;
+#else
+    return 1;
+#endif
 }
 
 /* ------------------------------------------------------------- PageRank ---
@@ -82,19 +158,23 @@ int oracle_pagerank(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, ui
 
     for (uint64_t v = 0; v < n; ++v) x[v] = 1.0 / (double)n;
     for (uint32_t t = 0; t < iters; ++t) {
-        double D = 0.0;
+        double D = 0.0;                            /* sequential: fixed summation order */
+        for (uint64_t u = 0; u < n; ++u)
+            if (row_ptr[u + 1] == row_ptr[u]) D += x[u];
+        #pragma omp parallel for schedule(static)
         for (uint64_t u = 0; u < n; ++u) {
             uint64_t deg = row_ptr[u + 1] - row_ptr[u];
-            if (deg == 0) { D += x[u]; contrib[u] = 0.0; }
-            else contrib[u] = x[u] / (double)deg;
+            contrib[u] = deg == 0 ? 0.0 : x[u] / (double)deg;
         }
         double base = (1.0 - d) / (double)n + (dangling_uniform ? d * D / (double)n : 0.0);
+        #pragma omp parallel for schedule(dynamic, 4096)
         for (uint64_t v = 0; v < n; ++v) {
             double s = 0.0;
             for (uint64_t k = in_ptr[v]; k < in_ptr[v + 1]; ++k) s += contrib[in_src[k]];
             y[v] = base + d * s;
         }
-        memcpy(x, y, n * sizeof(double));
+        #pragma omp parallel for schedule(static)
+        for (uint64_t v = 0; v < n; ++v) x[v] = y[v];
     }
     free(in_ptr); free(in_src); free(y); free(contrib);
     return 0;

@@ -135,7 +135,7 @@ extern "C" int gts_plan_pages(uint64_t n, const uint64_t* row_ptr, int weighted,
     clear_error();
     if (!row_ptr || !out) return fail(GTS_EINVAL, "NULL argument");
     if (n == 0) return fail(GTS_EINVAL, "n must be >= 1");
-    if (n > (1ull << 32)) return fail(GTS_EOVERFLOW, "n > 2^32");
+    if (n >= (1ull << 32)) return fail(GTS_EOVERFLOW, "n >= 2^32 (VID 0xFFFFFFFF is the NULL/empty sentinel)");
     uint32_t pb = (cfg && cfg->page_bytes) ? cfg->page_bytes : kDefaultPageBytes;
     uint32_t enc = cfg ? cfg->entry_encoding : GTS_ENTRY_VID32;
     if (!valid_page_bytes(pb)) return fail(GTS_EINVAL, "page_bytes %u must be a power of two in [256, 2^30]", pb);
@@ -154,7 +154,7 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
     if (cfg && cfg->struct_size && cfg->struct_size < sizeof(gts_page_config))
         return fail(GTS_EINVAL, "gts_page_config.struct_size too small");
     if (n == 0) return fail(GTS_EINVAL, "n must be >= 1");
-    if (n > (1ull << 32)) return fail(GTS_EOVERFLOW, "n > 2^32 (u32 VIDs)");
+    if (n >= (1ull << 32)) return fail(GTS_EOVERFLOW, "n >= 2^32 (u32 VIDs; 0xFFFFFFFF is the NULL/empty sentinel)");
     uint32_t pb = (cfg && cfg->page_bytes) ? cfg->page_bytes : kDefaultPageBytes;
     uint32_t enc = cfg ? cfg->entry_encoding : GTS_ENTRY_VID32;
     if (!valid_page_bytes(pb)) return fail(GTS_EINVAL, "page_bytes %u must be a power of two in [256, 2^30]", pb);

@@ -145,9 +145,9 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
     }
     if (c->dg.uid != g->uid) {
         DevGraph& d = c->dg;
-        d.uid = g->uid;
-        d.strategy = strat_key;
-        d.world = c->world;
+        // d.uid is set only after every allocation and upload below succeeded: a failed
+        // setup leaves uid = 0, and its partial allocations are freed on the next call
+        free_devgraph(d);
         std::vector<uint64_t> vrange;
         partition(g, strategy, c->world, d.h_owner, vrange);
         d.vlo = vrange[c->rank];
@@ -183,6 +183,9 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
             GTS_CUDA(cudaMemcpyAsync(d.new_of_old, g->new_of_old.data(), g->n * 4, cudaMemcpyHostToDevice, c->stream));
         }
         GTS_CUDA(cudaStreamSynchronize(c->stream));   // host vectors above are temporaries
+        d.uid = g->uid;
+        d.strategy = strat_key;
+        d.world = c->world;
     }
     DevGraph& d = c->dg;
     if (need_resident && !d.resident) {

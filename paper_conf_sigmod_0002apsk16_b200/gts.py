@@ -266,27 +266,32 @@ def _run_config(strategy, residency, ring_slots, batch_pages, out_location, timi
                      (GTS_RUN_TIMING if timing else 0) | micro, int(cache_mib))
 
 
-def _out(out, n, dtype):
-    """Host numpy array, or a CUDA tensor (anything with data_ptr() and is_cuda) -> (obj, ptr, location)."""
+def _out(out, n, dtype, ctx=None):
+    """Host numpy array, or a torch tensor (CUDA on the context's device, or CPU) -> (obj, ptr, location).
+    Every buffer must be contiguous, of the result's element size, with >= n elements: libgts writes
+    n elements through the pointer."""
     if out is None:
         out = np.empty(n, dtype=dtype)
+    isz = np.dtype(dtype).itemsize
     if isinstance(out, np.ndarray):
-        if out.dtype != dtype or out.size < n or not out.flags.c_contiguous:
-            raise ValueError(f"output must be a contiguous {dtype} array of >= {n} elements")
+        if out.dtype != dtype or out.size < n or not out.flags.c_contiguous or not out.flags.writeable:
+            raise ValueError(f"output must be a writeable contiguous {dtype} array of >= {n} elements")
         return out, ctypes.c_void_p(out.ctypes.data), GTS_OUT_HOST
+    if not (hasattr(out, "data_ptr") and hasattr(out, "numel") and hasattr(out, "element_size")):
+        raise TypeError("unsupported output buffer (numpy array or torch tensor)")
+    if out.numel() < n or out.element_size() != isz or not out.is_contiguous():
+        raise ValueError(f"output tensor must be contiguous, {isz}-byte elements, >= {n} elements")
     if getattr(out, "is_cuda", False):
-        if out.numel() < n or out.element_size() != np.dtype(dtype).itemsize or not out.is_contiguous():
-            raise ValueError(f"device output must be contiguous, {np.dtype(dtype).itemsize}-byte, >= {n} elements")
+        if ctx is not None and out.device.index is not None and out.device.index != ctx.device:
+            raise ValueError(f"device output is on cuda:{out.device.index}, the context on cuda:{ctx.device}")
         return out, ctypes.c_void_p(out.data_ptr()), GTS_OUT_DEVICE
-    if hasattr(out, "data_ptr"):   # pinned/pageable host tensor
-        return out, ctypes.c_void_p(out.data_ptr()), GTS_OUT_HOST
-    raise TypeError("unsupported output buffer")
+    return out, ctypes.c_void_p(out.data_ptr()), GTS_OUT_HOST     # pinned/pageable host tensor
 
 
 def gts_bfs(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
             batch_pages=0, timing=False, cache_mib=0, micro=GTS_MICRO_DEFAULT):
     """Returns (levels, stats dict).  micro: GTS_MICRO_* or "default"/"edge"/"vertex"/"hybrid"."""
-    out, ptr, loc = _out(out, graph.n, np.uint32)
+    out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib, micro)
     st = RunStats()
     _check(_lib.gts_bfs(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
@@ -296,7 +301,7 @@ def gts_bfs(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RE
 def gts_pagerank(ctx, graph, iters=10, damping=0.85, dangling=GTS_DANGLING_UNIFORM, out=None,
                  strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0, batch_pages=0, timing=False,
                  micro=GTS_MICRO_DEFAULT):
-    out, ptr, loc = _out(out, graph.n, np.float32)
+    out, ptr, loc = _out(out, graph.n, np.float32, ctx)
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, 0, micro)
     st = RunStats()
     _check(_lib.gts_pagerank(ctx.handle, graph.handle, int(iters), float(damping), int(dangling),
@@ -306,7 +311,7 @@ def gts_pagerank(ctx, graph, iters=10, damping=0.85, dangling=GTS_DANGLING_UNIFO
 
 def gts_sssp(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
              batch_pages=0, timing=False, cache_mib=0):
-    out, ptr, loc = _out(out, graph.n, np.uint32)
+    out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib)
     st = RunStats()
     _check(_lib.gts_sssp(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
@@ -315,7 +320,7 @@ def gts_sssp(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_R
 
 def gts_wcc(ctx, graph, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
             batch_pages=0, timing=False):
-    out, ptr, loc = _out(out, graph.n, np.uint32)
+    out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing)
     st = RunStats()
     _check(_lib.gts_wcc(ctx.handle, graph.handle, ctypes.byref(cfg), ptr, ctypes.byref(st)))
@@ -325,7 +330,7 @@ def gts_wcc(ctx, graph, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDEN
 def gts_bc(ctx, graph, sources, out=None, residency=GTS_RESIDENCY_AUTO, ring_slots=0, batch_pages=0, timing=False):
     """Betweenness centrality summed over `sources` (fp64, unnormalised).  Returns (bc, stats)."""
     src = np.ascontiguousarray(sources, dtype=np.uint64)
-    out, ptr, loc = _out(out, graph.n, np.float64)
+    out, ptr, loc = _out(out, graph.n, np.float64, ctx)
     cfg = _run_config(GTS_STRATEGY_P, residency, ring_slots, batch_pages, loc, timing)
     st = RunStats()
     _check(_lib.gts_bc(ctx.handle, graph.handle, _np_ptr(src), len(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))

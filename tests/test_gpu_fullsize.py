@@ -8,9 +8,9 @@ device outputs, persistent grids).
   dist[src] = 0, feasibility dist[v] <= dist[u] + w(u,v) on every edge, and a
   tight in-edge (dist[v] = dist[u] + w) for every reached v != src; plus the
   reached set equals the oracle BFS reached set.
-* PageRank: sum = 1 (UNIFORM), x_v >= (1-d)/n, and the last iteration
-  recomputed in fp64 from the GPU's own x^9 for a sample of vertices that
-  includes the top in-degree hubs (x^10_v = (1-d)/n + d*(sum_u x^9_u/deg u + D/n)).
+* PageRank: element-wise against the fp64 oracle (its OpenMP build), max
+  relative error <= 1e-4 and L1 <= 1e-5 (north_star), on RMAT-27 and on the
+  Twitter-shaped graph.
 """
 import numpy as np
 import pytest
@@ -83,41 +83,38 @@ def test_sssp_full_properties(big):
     assert np.all(tight[reach])
 
 
-def test_pagerank_full_properties(big):
+def pr_gates(got, want, g, tag):
+    """North_star PageRank gates vs the fp64 oracle: max_v |g-o|/o <= 1e-4 and
+    sum_v |g-o| <= 1e-5 (SURVEY 8(c) comparison rules); logs the argmax vertex
+    and its in-degree (the hub drift check)."""
+    got = got.astype(np.float64)
+    rel = np.abs(got - want) / want
+    l1 = float(np.sum(np.abs(got - want)))
+    i = int(np.argmax(rel))
+    indeg = np.bincount(g.col, minlength=g.n)
+    hub = int(np.argmax(indeg))
+    print(f"[{tag}] PageRank vs fp64 oracle: max rel {rel.max():.3e} at v={i} (in-degree {int(indeg[i])}), "
+          f"L1 {l1:.3e}; top hub v={hub} in-degree {int(indeg[hub])} rel {rel[hub]:.3e}")
+    assert rel.max() <= 1e-4, (float(rel.max()), i, int(indeg[i]))
+    assert l1 <= 1e-5, l1
+
+
+def test_pagerank_full_vs_oracle(big):
+    """Alg 4/5, x^0 = 1/n, 10 iterations, d = 0.85, UNIFORM
+    dangling (R1-R3): the GPU's fp32 result at full RMAT-27 against the
+    OpenMP build of the fp64 oracle (byte-identical to the plain build)."""
     G, g, gr, ctx, torch = big
-    n, dmp = g.n, 0.85
-    x9 = torch.empty(n, dtype=torch.float32, device="cuda")
-    x10 = torch.empty(n, dtype=torch.float32, device="cuda")
-    G.gts_pagerank(ctx, gr, 9, dmp, out=x9)
-    G.gts_pagerank(ctx, gr, 10, dmp, out=x10)
-    a9 = x9.cpu().numpy().astype(np.float64)
-    a10 = x10.cpu().numpy().astype(np.float64)
-    assert abs(np.sum(np.sort(a10)) - 1.0) <= 1e-4
-    assert np.all(a10 >= (1 - dmp) / n * (1 - 1e-4))
-    deg = np.diff(g.row_ptr).astype(np.float64)
-    D = a9[deg == 0].sum()
-    indeg = np.bincount(g.col, minlength=n)
-    rng = np.random.default_rng(27)
-    sample = np.unique(np.concatenate([np.argsort(indeg)[-64:], rng.integers(0, n, 512)]))
-    pos = np.full(n, -1, dtype=np.int64)
-    pos[sample] = np.arange(len(sample))
-    acc = np.zeros(len(sample))
-    chunk = 1 << 26
-    src_all = np.repeat(np.arange(n, dtype=np.int64), np.diff(g.row_ptr).astype(np.int64))
-    for a in range(0, g.m, chunk):
-        t = g.col[a:a + chunk].astype(np.int64)
-        hit = pos[t] >= 0
-        s = src_all[a:a + chunk][hit]
-        np.add.at(acc, pos[t[hit]], a9[s] / deg[s])
-    want = (1 - dmp) / n + dmp * (acc + D / n)
-    rel = np.abs(a10[sample] - want) / want
-    assert rel.max() <= 1e-4, (float(rel.max()), int(sample[np.argmax(rel)]))
+    x = torch.empty(g.n, dtype=torch.float32, device="cuda")
+    G.gts_pagerank(ctx, gr, 10, 0.85, out=x)
+    got = x.cpu().numpy()
+    want = oracle.pagerank(g.row_ptr, g.col, 10, 0.85, omp=True)
+    pr_gates(got, want, g, "rmat27")
 
 
 def test_twitter_shaped_full_size(gpu):
     """BASELINE configs[1]: Twitter-shaped graph at full size (n = 41.65 M,
     m = 1.47 B, degree-ordered 1 MiB pages): BFS and WCC bit-exact, PageRank
-    sum and lower-bound invariants."""
+    element-wise against the fp64 oracle."""
     import torch
     import paper_conf_sigmod_0002apsk16_b200 as G
     g = inputs.twitter_like()
@@ -134,8 +131,6 @@ def test_twitter_shaped_full_size(gpu):
         assert np.array_equal(out.cpu().numpy().view(np.uint32), oracle.wcc(g.row_ptr, g.col))
         x = torch.empty(g.n, dtype=torch.float32, device="cuda")
         G.gts_pagerank(ctx, gr, 10, 0.85, out=x)
-        a = x.cpu().numpy().astype(np.float64)
-        assert abs(np.sum(np.sort(a)) - 1.0) <= 1e-4
-        assert np.all(a >= 0.15 / g.n * (1 - 1e-4))
+        pr_gates(x.cpu().numpy(), oracle.pagerank(g.row_ptr, g.col, 10, 0.85, omp=True), g, "twitter")
     finally:
         ctx.free()

@@ -144,3 +144,19 @@ def test_generator_lean_mode_same_graph():
     a = inputs.rmat(13)
     b = inputs.rmat(13, lean=True)
     assert np.array_equal(a.row_ptr, b.row_ptr) and np.array_equal(a.col, b.col)
+
+
+@pytest.mark.parametrize("omp", [False, True])
+def test_levelsync_equals_queue_bfs(omp):
+    """The level-synchronous BFS (plain and OpenMP builds) returns the FIFO-queue
+    BFS levels: the level sets of a BFS are unique (Alg 1 P:330-334 drives the
+    GPU level by level)."""
+    cases = [inputs.rmat(16), inputs.random_graph(20000, 60000, 3), inputs.path(5000), inputs.in_star(1000),
+             inputs.out_star(1000), inputs.twitter_like(n=1 << 16, m=1 << 20)]
+    for g in cases:
+        deg = np.diff(g.row_ptr)
+        for src in {0, int(np.argmax(deg)), g.n - 1}:
+            assert np.array_equal(oracle.bfs_levelsync(g.row_ptr, g.col, src, omp=omp),
+                                  oracle.bfs(g.row_ptr, g.col, src))
+    with pytest.raises(ValueError):
+        oracle.bfs_levelsync(cases[0].row_ptr, cases[0].col, cases[0].n, omp=omp)

@@ -130,3 +130,18 @@ def test_multiedges_count_with_multiplicity():
     g = inputs.from_edges(3, [(0, 1), (0, 1), (0, 2), (1, 0), (2, 0)])
     x = oracle.pagerank(g.row_ptr, g.col, 10, D)
     assert np.max(np.abs(x - _dense_pagerank(g, 10, D))) < 1e-15
+
+
+@pytest.mark.parametrize("maker", [lambda: inputs.rmat(16), lambda: inputs.random_graph(30000, 200000, 5),
+                                   lambda: inputs.in_star(100000)])
+@pytest.mark.parametrize("dangling", [oracle.DANGLING_UNIFORM, oracle.DANGLING_DROP])
+def test_openmp_build_byte_identical(maker, dangling):
+    """the oracle is compiled plain and with OpenMP; every y[v]
+    sums its in-edges in ascending u in both builds and D is summed
+    sequentially, so the outputs are byte-identical (the OpenMP build is the
+    parity reference at full size and the all-core CPU baseline)."""
+    g = maker()
+    a = oracle.pagerank(g.row_ptr, g.col, 10, D, dangling=dangling, omp=False)
+    b = oracle.pagerank(g.row_ptr, g.col, 10, D, dangling=dangling, omp=True)
+    assert a.tobytes() == b.tobytes()
+    assert oracle.num_threads(omp=False) == 1

@@ -1,0 +1,38 @@
+#!/bin/bash
+# One parameterised GPU-box job (run under gpurun from the repo root):
+#   tools/gpu/run.sh <what> [args...]
+# what:
+#   tests [pytest args]       pytest -m gpu (default -x -q), log -> gpurun_out/tests.log
+#   bench [bench args]        bench.py, JSON line -> gpurun_out/bench.json, stderr -> bench.log
+#   launches [bench args]     ncu launch list of one bench step (cold-cache, serialised: shares only)
+#   ncu <kernel-regex> [n] [bench args]   ncu --set full of the n-th launch matching the regex
+#   sanitize <tool>           compute-sanitizer <tool> over tools/sanitize_run.py (RMAT-16, every kernel)
+#   py <script> [args]        any python script, stdout -> gpurun_out/<script basename>.out
+set -u
+cd "${GRAFT_REPO_ROOT:-/root/repo}"
+O=gpurun_out
+mkdir -p $O
+what=${1:-tests}; shift || true
+case "$what" in
+  tests)
+    timeout 3000 python -m pytest tests -m gpu ${@:--x -q} > $O/tests.log 2>&1; echo "pytest rc=$?"; tail -5 $O/tests.log ;;
+  bench)
+    timeout 1500 python bench.py "$@" > $O/bench.json 2> $O/bench.log; echo "bench rc=$?"; tail -c 3000 $O/bench.json ;;
+  launches)
+    timeout 1500 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv \
+      python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e "$@" > /dev/null 2> $O/launches.log
+    echo "ncu rc=$?"; python tools/launch_summary.py $O/launches.csv > $O/launches.txt; head -40 $O/launches.txt ;;
+  ncu)
+    k=$1; shift; c=${1:-1}; shift || true
+    timeout 2400 ncu --set full --clock-control none --import-source on -k "regex:$k" -s $((c - 1)) -c 1 \
+      -o $O/ncu_full -f python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e "$@" > $O/ncu.log 2>&1
+    echo "ncu rc=$?"; tail -3 $O/ncu.log ;;
+  sanitize)
+    tool=${1:-memcheck}
+    timeout 2400 compute-sanitizer --tool $tool --print-limit 50 python tools/sanitize_run.py > $O/sanitize_$tool.log 2>&1
+    echo "sanitizer rc=$?"; tail -8 $O/sanitize_$tool.log ;;
+  py)
+    s=$1; shift
+    timeout 3000 python "$s" "$@" > $O/$(basename "$s" .py).out 2>&1; echo "py rc=$?"; tail -40 $O/$(basename "$s" .py).out ;;
+  *) echo "unknown job $what"; exit 2 ;;
+esac
