@@ -10,7 +10,7 @@ NCCL_DIR := $(SITE)/nvidia/nccl
 ARCH     := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 --expt-relaxed-constexpr -Xcompiler -fPIC,-fopenmp,-O3 \
             -Iinclude -I$(CSRC) -I$(NCCL_DIR)/include -Xptxas -v
-CU_SRC   := $(CSRC)/context.cu $(CSRC)/traverse.cu $(CSRC)/pagerank.cu $(CSRC)/wcc.cu
+CU_SRC   := $(CSRC)/context.cu $(CSRC)/comm.cu $(CSRC)/traverse.cu $(CSRC)/pagerank.cu $(CSRC)/wcc.cu
 CPP_SRC  := $(CSRC)/builder.cpp $(CSRC)/capi.cpp
 HDRS     := include/gts.h $(wildcard $(CSRC)/*.h) $(wildcard $(CSRC)/*.cuh)
 OBJDIR   := build/obj

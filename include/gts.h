@@ -72,13 +72,20 @@ typedef enum {
 
 enum { GTS_PAGE_SP = 0, GTS_PAGE_LP = 1 };
 enum { GTS_ENTRY_VID32 = 0, GTS_ENTRY_PID16_SLOT16 = 1 };
-/* Strategy-P: pages partitioned h(j) = j mod N, WA replicated.
- * Strategy-S: WA range-partitioned, each rank holds the pages of its range and
- *             routes updates to their owners (north_star "routes updates").
+/* Strategy-P: pages partitioned h(j) = j mod N, WA replicated, merged after
+ *             every iteration / level: PageRank all-reduce(sum),
+ *             BFS all-gather + OR of the next frontiers, SSSP all-reduce(min)
+ *             + OR, WCC all-reduce(min) of the union-find forests.
+ * Strategy-S: WA range-partitioned into N contiguous VID ranges cut at page
+ *             boundaries; each rank holds the pages whose sources lie in its
+ *             range and routes updates for other ranges to their owners
+ *             (north_star "routes updates"): PageRank (dst, value), BFS dst,
+ *             SSSP (dst, dist), WCC (dst, label) on GTS_BUILD_SYMMETRIC pages.
+ *             Each rank allocates its WA range only (n/N entries).
  * Strategy-S_BCAST: the paper-literal Strategy-S: every rank
- *             processes every page and keeps only the updates of its own WA
- *             range; no exchange until the final gather (PageRank; the other
- *             algorithms run replicated). */
+ *             processes every page and applies only the updates of its own WA
+ *             range (PageRank, BFS, SSSP; WA ranges re-broadcast after each
+ *             step); WCC runs the full union-find on every rank (replicated). */
 enum { GTS_STRATEGY_P = 0, GTS_STRATEGY_S = 1, GTS_STRATEGY_S_BCAST = 2 };
 enum { GTS_RESIDENCY_AUTO = 0, GTS_RESIDENT = 1, GTS_STREAMED = 2 };
 enum { GTS_DANGLING_UNIFORM = 0, GTS_DANGLING_DROP = 1 };
@@ -103,6 +110,21 @@ enum { GTS_MICRO_DEFAULT = 0u, GTS_MICRO_EDGE = 1u << 8, GTS_MICRO_VERTEX = 2u <
  * IDs (gts_graph_order gives the mapping).  Used by the B200 PageRank kernel
  * to keep the most-updated WA entries contiguous. */
 enum { GTS_BUILD_DEGREE_ORDER = 1u };
+/* gts_page_config.flags: also store every edge reversed (the pages hold the
+ * symmetrised multigraph, 2m entries).  gts_wcc under GTS_STRATEGY_S needs it:
+ * its routed label propagation pushes along both directions of an edge from
+ * the source's owner only (WCC caveat). */
+enum { GTS_BUILD_SYMMETRIC = 2u };
+/* gts_page_config.flags: build (and hold in host memory) only the pages that
+ * rank owner_rank of an owner_world-rank job processes under owner_strategy
+ * (Strategy-P: page j with j mod N == rank; Strategy-S: the rank's
+ * contiguous page range).  The directory (RVT) still covers every
+ * page.  Such a graph can only be used by a context of that rank and world
+ * with that strategy (EINVAL otherwise); gts_graph_pages returns the held
+ * pages in ascending page ID.  S_BCAST ranks process every page, so the
+ * filter keeps all pages for it. */
+enum { GTS_BUILD_OWNER_FILTER = 4u };
+#define GTS_OFF 0xFFFFFFFFu
 
 #define GTS_UNREACHED 0xFFFFFFFFu
 
@@ -112,10 +134,13 @@ int gts_version(void);
 /* ------------------------------------------------------------- graphs --- */
 
 typedef struct {
-    uint32_t struct_size;     /* sizeof(gts_page_config) */
+    uint32_t struct_size;     /* sizeof(gts_page_config); 16 (version 1.0 layout) is accepted */
     uint32_t page_bytes;      /* power of two, 256 B .. 1 GiB; default (0) = 1 MiB (R14) */
     uint32_t entry_encoding;  /* GTS_ENTRY_VID32 (default) | GTS_ENTRY_PID16_SLOT16 */
-    uint32_t flags;           /* 0 or GTS_BUILD_DEGREE_ORDER */
+    uint32_t flags;           /* GTS_BUILD_DEGREE_ORDER | GTS_BUILD_SYMMETRIC | GTS_BUILD_OWNER_FILTER */
+    /* GTS_BUILD_OWNER_FILTER only: */
+    uint32_t owner_rank, owner_world, owner_strategy;
+    uint32_t reserved;
 } gts_page_config;
 
 typedef struct {
@@ -128,6 +153,10 @@ typedef struct {
     uint32_t weighted, entry_encoding;
     uint32_t n_hot;           /* entries in the hot-destination table (PageRank, DESIGN.md K-PR) */
     uint32_t ordered;         /* 1 if built with GTS_BUILD_DEGREE_ORDER */
+    uint64_t host_page_bytes; /* page bytes this graph holds in host memory (< topo_bytes with an owner filter) */
+    uint32_t symmetric;       /* 1 if built with GTS_BUILD_SYMMETRIC (m counts both directions) */
+    int32_t owner_rank;       /* GTS_BUILD_OWNER_FILTER: the rank; -1: every page is held */
+    uint32_t owner_world, owner_strategy;
 } gts_graph_stats;
 
 typedef struct gts_graph gts_graph;   /* opaque; owns the host pages + directory (RVT) */
@@ -195,6 +224,18 @@ typedef struct {
     uint32_t flags;           /* GTS_RUN_TIMING | one GTS_MICRO_* value */
     uint32_t cache_mib;       /* streamed BFS/SSSP: device LRU cache of topology pages across levels,
                                  in MiB (cachedPIDMap, Alg 1 lines 8/16/29); 0 = none */
+    /* ---- version 1.1 (struct_size >= 64; a 32-byte 1.0 config gets the defaults) ---- */
+    uint32_t virtual_ranks;   /* 0/1 = off.  V in [2, 8] on a world-1 context: run the V-rank job of
+                                 `strategy` on this one GPU -- every rank's page set, WA buffers, kernels
+                                 and merge kernels as on V GPUs, the collectives done in device memory
+                                 (DESIGN.md "Virtual ranks").  Results equal the real V-rank job's. */
+    uint32_t sssp_delta;      /* SSSP near-far bucket width; 0 = unbounded (frontier Bellman-Ford) */
+    uint32_t levels_per_sync; /* BFS on one rank, resident: levels enqueued per host round trip; 0 = 8 */
+    uint32_t l2_persist_mib;  /* persisting-L2 window on the probed head of WA; 0 = 96 MiB, GTS_OFF = none */
+    uint32_t bfs_level_slots; /* BFS level-slot store (one bitmap per level); 0 = 32, GTS_OFF = off */
+    uint32_t wcc_sample;      /* WCC sampling pass: first k out-neighbours; 0 = 1, GTS_OFF = no pass */
+    uint32_t hybrid_deg;      /* GTS_MICRO_HYBRID: vertex-centric below this many edges/vertex; 0 = 8 */
+    uint32_t reserved;
 } gts_run_config;
 
 typedef struct {
@@ -214,6 +255,8 @@ typedef struct {
     uint32_t reserved;
     uint64_t cache_hits;      /* streamed + cache: page visits served from the device cache */
     uint64_t cache_misses;    /* streamed + cache: page visits copied from host memory */
+    uint64_t wa_bytes;        /* device bytes of the attribute vectors (WA + RA) one rank allocated */
+    uint64_t routed_msgs;     /* Strategy-S: update messages sent to other ranks */
 } gts_run_stats;
 
 /* BFS (App B.1, Alg 2/3 P:1494-1514; Alg 1 BFS-like path P:330-334).

@@ -21,6 +21,39 @@ namespace gts {
 
 static std::atomic<uint64_t> g_next_uid{1};
 
+void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t>& owner,
+               std::vector<uint64_t>& vrange) {
+    const uint64_t P = g->num_pages;
+    owner.assign(P, 0);
+    vrange.assign(world + 1, g->n);
+    vrange[0] = 0;
+    if (world <= 1) return;
+    if (strategy == GTS_STRATEGY_P) {
+        for (uint64_t j = 0; j < P; ++j) owner[j] = (int32_t)(j % (uint64_t)world);   // h(j) = j mod N
+        return;
+    }
+    // Strategy-S and S_BCAST share the WA ranges; under S_BCAST owner[j] is the
+    // WA owner of the page's sources, but every rank processes every page.
+    // Strategy-S: contiguous VID ranges cut at page boundaries (never inside an
+    // LP run) with ~equal page counts; rank r owns WA[vrange[r], vrange[r+1]).
+    uint64_t p = 0;
+    for (int r = 0; r < world; ++r) {
+        uint64_t target = (P * (uint64_t)(r + 1)) / (uint64_t)world;
+        if (r == world - 1) target = P;
+        uint64_t first = p;
+        while (p < target || (p < P && p > 0 && g->kind[p] == GTS_PAGE_LP && g->lp_first[p] != (int64_t)p)) {
+            owner[p] = r;
+            ++p;
+        }
+        vrange[r] = first < P ? g->start_vid[first] : g->n;
+        if (r == 0) vrange[0] = 0;
+    }
+    // ranks left without pages own an empty range at the end
+    for (int r = 1; r <= world; ++r) vrange[r] = std::max(vrange[r], vrange[r - 1]);
+    vrange[world] = g->n;
+}
+
+
 static inline void wr32(uint8_t* p, uint32_t v) { std::memcpy(p, &v, 4); }
 
 static bool valid_page_bytes(uint32_t pb) {
@@ -146,17 +179,64 @@ extern "C" int gts_plan_pages(uint64_t n, const uint64_t* row_ptr, int weighted,
     return plan_pages(n, row_ptr, weighted != 0, pb, enc, plan, out);
 }
 
+// Symmetrised multigraph (GTS_BUILD_SYMMETRIC): row u = out(u) followed by in(u)
+// (every edge u->v also stored as v->u), each row sorted (by (dst, weight)).
+static void symmetrise(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, const uint32_t* w,
+                       std::vector<uint64_t>& s_row, std::vector<uint32_t>& s_col, std::vector<uint32_t>& s_w) {
+    const uint64_t m = row_ptr[n];
+    std::vector<uint64_t> indeg(n + 1, 0);
+    for (uint64_t k = 0; k < m; ++k) indeg[col[k]]++;
+    s_row.assign(n + 1, 0);
+    for (uint64_t v = 0; v < n; ++v) s_row[v + 1] = s_row[v] + (row_ptr[v + 1] - row_ptr[v]) + indeg[v];
+    s_col.resize(2 * m);
+    if (w) s_w.resize(2 * m);
+    std::vector<uint64_t> cur(n);
+    for (uint64_t v = 0; v < n; ++v) {
+        const uint64_t d = row_ptr[v + 1] - row_ptr[v];
+        std::memcpy(s_col.data() + s_row[v], col + row_ptr[v], d * 4);
+        if (w) std::memcpy(s_w.data() + s_row[v], w + row_ptr[v], d * 4);
+        cur[v] = s_row[v] + d;
+    }
+    for (uint64_t u = 0; u < n; ++u)
+        for (uint64_t k = row_ptr[u]; k < row_ptr[u + 1]; ++k) {
+            const uint64_t at = cur[col[k]]++;
+            s_col[at] = (uint32_t)u;
+            if (w) s_w[at] = w[k];
+        }
+    #pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t v = 0; v < (int64_t)n; ++v) {
+        const uint64_t b = s_row[v], len = s_row[v + 1] - b;
+        if (!w) {
+            std::sort(s_col.begin() + b, s_col.begin() + b + len);
+        } else {
+            std::vector<std::pair<uint32_t, uint32_t>> e(len);
+            for (uint64_t k = 0; k < len; ++k) e[k] = {s_col[b + k], s_w[b + k]};
+            std::sort(e.begin(), e.end());
+            for (uint64_t k = 0; k < len; ++k) {
+                s_col[b + k] = e[k].first;
+                s_w[b + k] = e[k].second;
+            }
+        }
+    }
+}
+
 extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, const uint32_t* col_idx,
                                const uint32_t* weights, const gts_page_config* cfg, gts_graph** out) {
     clear_error();
     if (!row_ptr || !out || (m > 0 && !col_idx)) return fail(GTS_EINVAL, "NULL argument");
     *out = nullptr;
-    if (cfg && cfg->struct_size && cfg->struct_size < sizeof(gts_page_config))
-        return fail(GTS_EINVAL, "gts_page_config.struct_size too small");
+    // struct_size: 16 = the 1.0 layout (no owner fields), sizeof = current; 0 = current
+    gts_page_config pc;
+    std::memset(&pc, 0, sizeof(pc));
+    if (cfg) {
+        const uint32_t sz = cfg->struct_size ? cfg->struct_size : (uint32_t)sizeof(gts_page_config);
+        if (sz < 16) return fail(GTS_EINVAL, "gts_page_config.struct_size too small");
+        std::memcpy(&pc, cfg, std::min<size_t>(sz, sizeof(pc)));
+    }
     if (n == 0) return fail(GTS_EINVAL, "n must be >= 1");
     if (n >= (1ull << 32)) return fail(GTS_EOVERFLOW, "n >= 2^32 (u32 VIDs; 0xFFFFFFFF is the NULL/empty sentinel)");
-    uint32_t pb = (cfg && cfg->page_bytes) ? cfg->page_bytes : kDefaultPageBytes;
-    uint32_t enc = cfg ? cfg->entry_encoding : GTS_ENTRY_VID32;
+    uint32_t pb = pc.page_bytes ? pc.page_bytes : kDefaultPageBytes;
+    uint32_t enc = pc.entry_encoding;
     if (!valid_page_bytes(pb)) return fail(GTS_EINVAL, "page_bytes %u must be a power of two in [256, 2^30]", pb);
     if (enc > GTS_ENTRY_PID16_SLOT16) return fail(GTS_EINVAL, "unknown entry encoding %u", enc);
     if (row_ptr[0] != 0 || row_ptr[n] != m) return fail(GTS_EINVAL, "row_ptr[0] must be 0 and row_ptr[n] == m");
@@ -169,9 +249,26 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
     for (int64_t k = 0; k < (int64_t)m; ++k) bad_col = bad_col || (col_idx[k] >= n);
     if (bad_col) return fail(GTS_EINVAL, "col_idx has an entry >= n");
 
+    const uint32_t known = GTS_BUILD_DEGREE_ORDER | GTS_BUILD_SYMMETRIC | GTS_BUILD_OWNER_FILTER;
+    if (pc.flags & ~known) return fail(GTS_EINVAL, "unknown page_config flags 0x%x", pc.flags);
     const bool weighted = weights != nullptr;
-    const bool ordered = cfg && (cfg->flags & GTS_BUILD_DEGREE_ORDER);
-    if (cfg && (cfg->flags & ~(uint32_t)GTS_BUILD_DEGREE_ORDER)) return fail(GTS_EINVAL, "unknown page_config flags");
+    const bool ordered = pc.flags & GTS_BUILD_DEGREE_ORDER;
+    const bool symmetric = pc.flags & GTS_BUILD_SYMMETRIC;
+    const bool filtered = pc.flags & GTS_BUILD_OWNER_FILTER;
+    if (filtered) {
+        if (pc.owner_world < 1 || pc.owner_rank >= pc.owner_world)
+            return fail(GTS_EINVAL, "owner filter: rank %u of world %u", pc.owner_rank, pc.owner_world);
+        if (pc.owner_strategy > GTS_STRATEGY_S_BCAST) return fail(GTS_EINVAL, "owner filter: unknown strategy");
+    }
+    std::vector<uint64_t> s_row;
+    std::vector<uint32_t> s_col, s_w;
+    if (symmetric) {
+        symmetrise(n, row_ptr, col_idx, weights, s_row, s_col, s_w);
+        row_ptr = s_row.data();
+        col_idx = s_col.data();
+        if (weighted) weights = s_w.data();
+        m = 2 * m;
+    }
     // Degree ordering (GTS_BUILD_DEGREE_ORDER): rename vertices by descending
     // in-degree (ties by VID) and build the pages of the renamed graph.
     std::vector<uint32_t> new_of_old, old_of_new;
@@ -238,11 +335,7 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
     g->used_bytes = st.used_bytes;
     g->max_outdeg = st.max_outdeg;
     g->uid = g_next_uid.fetch_add(1);
-    g->pages_alloc = (size_t)g->num_pages * pb;
-    size_t alloc = (g->pages_alloc + 4095) & ~(size_t)4095;
-    if (alloc == 0) alloc = 4096;
-    g->pages = (uint8_t*)std::aligned_alloc(4096, alloc);
-    if (!g->pages) { delete g; return fail(GTS_ENOMEM, "cannot allocate %zu bytes of pages", alloc); }
+    g->symmetric = symmetric;
     g->start_vid.resize(g->num_pages);
     g->nslots.resize(g->num_pages);
     g->kind.resize(g->num_pages);
@@ -255,6 +348,30 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
         g->lp_first[p] = plan[p].lp_first;
         g->lp_last[p] = plan[p].lp_last;
     }
+    // the pages this graph holds: all, or (owner filter) the pages of one rank
+    std::vector<uint32_t> held;
+    if (filtered && pc.owner_strategy != GTS_STRATEGY_S_BCAST && pc.owner_world > 1) {
+        std::vector<int32_t> owner;
+        std::vector<uint64_t> vr;
+        partition(g, pc.owner_strategy, (int)pc.owner_world, owner, vr);
+        g->host_loc.assign(g->num_pages, UINT32_MAX);
+        for (uint64_t p = 0; p < g->num_pages; ++p)
+            if (owner[p] == (int32_t)pc.owner_rank) {
+                g->host_loc[p] = (uint32_t)held.size();
+                held.push_back((uint32_t)p);
+            }
+    }
+    if (filtered) {
+        g->owner_rank = (int32_t)pc.owner_rank;
+        g->owner_world = pc.owner_world;
+        g->owner_strategy = pc.owner_strategy;
+    }
+    g->n_host_pages = g->host_loc.empty() ? g->num_pages : held.size();
+    g->pages_alloc = (size_t)g->n_host_pages * pb;
+    size_t alloc = (g->pages_alloc + 4095) & ~(size_t)4095;
+    if (alloc == 0) alloc = 4096;
+    g->pages = (uint8_t*)std::aligned_alloc(4096, alloc);
+    if (!g->pages) { delete g; return fail(GTS_ENOMEM, "cannot allocate %zu bytes of pages", alloc); }
 
     // PID16_SLOT16: physical ID of every vertex = (first page holding it, slot)
     std::vector<uint32_t> phys;
@@ -272,8 +389,9 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
     const uint64_t lp_cap = (pb - kLpFooter - kSlotBytes - 4) / (4 * wpe);
 
     #pragma omp parallel for schedule(dynamic, 4)
-    for (int64_t p = 0; p < (int64_t)g->num_pages; ++p) {
-        uint8_t* pg = g->pages + (size_t)p * pb;
+    for (int64_t hp = 0; hp < (int64_t)g->n_host_pages; ++hp) {
+        const int64_t p = g->host_loc.empty() ? hp : (int64_t)held[hp];
+        uint8_t* pg = g->pages + (size_t)hp * pb;
         std::memset(pg, 0, pb);
         const PagePlanEntry& e = plan[p];
         auto put_entries = [&](uint8_t* dst, uint64_t k0, uint64_t len) {
@@ -342,6 +460,11 @@ extern "C" int gts_graph_get_stats(const gts_graph* g, gts_graph_stats* out) {
     out->entry_encoding = g->entry_encoding;
     out->n_hot = g->ordered ? (uint32_t)std::min<uint64_t>(g->n, kHotDense) : g->n_hot;
     out->ordered = g->ordered ? 1 : 0;
+    out->host_page_bytes = g->n_host_pages * (uint64_t)g->page_bytes;
+    out->symmetric = g->symmetric ? 1 : 0;
+    out->owner_rank = g->owner_rank;
+    out->owner_world = g->owner_world;
+    out->owner_strategy = g->owner_strategy;
     return GTS_OK;
 }
 

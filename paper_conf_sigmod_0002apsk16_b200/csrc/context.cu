@@ -56,38 +56,6 @@ int Context::buf(int slot, size_t bytes, void** out) {
     return GTS_OK;
 }
 
-void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t>& owner,
-               std::vector<uint64_t>& vrange) {
-    const uint64_t P = g->num_pages;
-    owner.assign(P, 0);
-    vrange.assign(world + 1, g->n);
-    vrange[0] = 0;
-    if (world <= 1) return;
-    if (strategy == GTS_STRATEGY_P) {
-        for (uint64_t j = 0; j < P; ++j) owner[j] = (int32_t)(j % (uint64_t)world);   // h(j) = j mod N
-        return;
-    }
-    // Strategy-S and S_BCAST share the WA ranges; under S_BCAST owner[j] is the
-    // WA owner of the page's sources, but every rank processes every page.
-    // Strategy-S: contiguous VID ranges cut at page boundaries (never inside an
-    // LP run) with ~equal page counts; rank r owns WA[vrange[r], vrange[r+1]).
-    uint64_t p = 0;
-    for (int r = 0; r < world; ++r) {
-        uint64_t target = (P * (uint64_t)(r + 1)) / (uint64_t)world;
-        if (r == world - 1) target = P;
-        uint64_t first = p;
-        while (p < target || (p < P && p > 0 && g->kind[p] == GTS_PAGE_LP && g->lp_first[p] != (int64_t)p)) {
-            owner[p] = r;
-            ++p;
-        }
-        vrange[r] = first < P ? g->start_vid[first] : g->n;
-        if (r == 0) vrange[0] = 0;
-    }
-    // ranks left without pages own an empty range at the end
-    for (int r = 1; r <= world; ++r) vrange[r] = std::max(vrange[r], vrange[r - 1]);
-    vrange[world] = g->n;
-}
-
 // Pin the graph's host pages (and, for ordered graphs, the VID maps) once, so
 // uploads and streamed sweeps run at the link rate.  Failure is not an error:
 // pageable sources are still correct, only slower.
@@ -204,13 +172,15 @@ int ensure_graph(Context* c, const Graph* gc, uint32_t strategy, bool need_resid
             return fail(GTS_ENOMEM, "resident pages: cudaMalloc(%zu) failed: %s", d.pages_bytes,
                         cudaGetErrorString(e));
         }
-        // copy runs of consecutive local pages in one cudaMemcpyAsync each
+        // copy runs of pages adjacent in host memory in one cudaMemcpyAsync each
         uint32_t i = 0;
         while (i < d.n_local) {
+            const uint8_t* h0 = host_page(g, d.h_local_list[i]);
+            if (!h0) return fail(GTS_EINVAL, "graph does not hold page %u of this rank", d.h_local_list[i]);
             uint32_t j = i + 1;
-            while (j < d.n_local && d.h_local_list[j] == d.h_local_list[j - 1] + 1) ++j;
-            GTS_CUDA(cudaMemcpyAsync(d.pages + (size_t)i * pb, g->pages + (size_t)d.h_local_list[i] * pb,
-                                     (size_t)(j - i) * pb, cudaMemcpyHostToDevice, c->stream));
+            while (j < d.n_local && host_page(g, d.h_local_list[j]) == h0 + (size_t)(j - i) * pb) ++j;
+            GTS_CUDA(cudaMemcpyAsync(d.pages + (size_t)i * pb, h0, (size_t)(j - i) * pb, cudaMemcpyHostToDevice,
+                                     c->stream));
             i = j;
         }
         GTS_CUDA(cudaStreamSynchronize(c->stream));
@@ -254,14 +224,29 @@ int validate_common(gts_context* ctx, const gts_graph* g, const gts_run_config* 
     d.struct_size = sizeof(d);
     d.strategy = GTS_STRATEGY_P;
     d.residency = GTS_RESIDENCY_AUTO;
-    if (cfg) {
-        if (cfg->struct_size && cfg->struct_size < sizeof(gts_run_config))
-            return fail(GTS_EINVAL, "gts_run_config.struct_size too small");
-        d = *cfg;
+    if (cfg) {   // struct_size 32 = the 1.0 layout (the 1.1 fields take their defaults); 0 = current
+        const uint32_t sz = cfg->struct_size ? cfg->struct_size : (uint32_t)sizeof(gts_run_config);
+        if (sz < 32) return fail(GTS_EINVAL, "gts_run_config.struct_size too small");
+        std::memcpy(&d, cfg, std::min<size_t>(sz, sizeof(d)));
+        d.struct_size = sizeof(d);
     }
     if (d.strategy > GTS_STRATEGY_S_BCAST) return fail(GTS_EINVAL, "unknown strategy %u", d.strategy);
     if (d.residency > GTS_STREAMED) return fail(GTS_EINVAL, "unknown residency %u", d.residency);
     if (d.out_location > GTS_OUT_DEVICE) return fail(GTS_EINVAL, "unknown out_location %u", d.out_location);
+    if (d.virtual_ranks > 8) return fail(GTS_EINVAL, "virtual_ranks must be <= 8");
+    if (d.virtual_ranks > 1 && ctx->world > 1) return fail(GTS_EINVAL, "virtual_ranks needs a world-1 context");
+    const bool multi = ctx->world > 1 || d.virtual_ranks > 1;
+    if (multi && (d.flags & GTS_MICRO_MASK))
+        return fail(GTS_EUNSUPPORTED, "GTS_MICRO_* techniques run on one rank");
+    if (multi && d.cache_mib) return fail(GTS_EUNSUPPORTED, "the page cache (cache_mib) runs on one rank");
+    // an owner-filtered graph holds one rank's pages: only that rank of that job can use it
+    if (g->owner_rank >= 0 && g->owner_world > 1 && g->owner_strategy != GTS_STRATEGY_S_BCAST) {
+        if (ctx->world != (int)g->owner_world || ctx->rank != g->owner_rank ||
+            (ctx->world > 1 && d.strategy != g->owner_strategy))
+            return fail(GTS_EINVAL, "graph holds the pages of rank %d/%u (strategy %u); context is rank %d/%d "
+                        "(strategy %u)", g->owner_rank, g->owner_world, g->owner_strategy, ctx->rank, ctx->world,
+                        d.strategy);
+    }
     if (d.ring_slots == 0) d.ring_slots = 4;
     if (d.batch_pages == 0) {   // >= 64 MiB per batch: enough pages in flight to keep the link busy
         const uint32_t pb = g->page_bytes;

@@ -184,68 +184,6 @@ __device__ __forceinline__ void gather_items(const PageSet& ps, Op& op, TileSmem
     }
 }
 
-// Same expansion by warp windows: the item edge space [0, total) is cut into
-// 128-edge windows, each warp walks a contiguous run of them, and the owner of
-// a lane's edges comes from an item-start mask (win_mask over sm.pre) instead of
-// a binary search per 4 edges.  Requires every item to have >= 1 edge (starts
-// are distinct).  The item data of the lane's first two owners is read once.
-template <class Op>
-__device__ __forceinline__ void gather_items_ww(const PageSet& ps, Op& op, TileSmem& sm, const uint32_t* words,
-                                                uint32_t nf, uint32_t total, uint64_t pol) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint32_t nwin = (total + 127) >> 7;
-    const uint32_t per = (nwin + kWarps - 1) / kWarps;
-    const uint32_t wa = min(nwin, warp * per), wb = min(nwin, wa + per);
-    if (wa >= wb) return;
-    const uint32_t base0 = wa << 7;
-    int lo = -1, hi = (int)nf;                       // pre[lo] < base0 <= pre[hi]
-    while (hi - lo > 1) {
-        const int mid = (lo + hi) >> 1;
-        if (sm.pre[mid] < base0) lo = mid; else hi = mid;
-    }
-    int j0 = lo;
-    for (uint32_t wi = wa; wi < wb; ++wi) {
-        const uint32_t bw = wi << 7;
-        int ns;
-        const WinMask wm = win_mask(sm.pre, j0, nf, bw, ns);
-        const uint32_t mw = lane >> 3;
-        uint32_t before = 0;
-#pragma unroll
-        for (int k = 0; k < 4; ++k) before += (uint32_t)k < mw ? __popc(wm.m[k]) : 0u;
-        const uint32_t mword = mw == 0 ? wm.m[0] : mw == 1 ? wm.m[1] : mw == 2 ? wm.m[2] : wm.m[3];
-        const uint32_t bpos0 = (4 * lane) & 31;
-        const uint32_t nb = (mword >> bpos0) & 0xFu;     // items starting at my edges
-        const int jb = j0 + (int)(before + __popc(mword & ((1u << bpos0) - 1u)));
-        // owners jb (if >= 0) and jb + 1
-        const int ja = jb < 0 ? 0 : jb;
-        const uint32_t preA = sm.pre[ja], offA = sm.off[ja], degA = sm.deg[ja], payA = sm.payload[ja], srcA = sm.src[ja];
-        const uint32_t preB = sm.pre[jb + 1], offB = sm.off[jb + 1], degB = sm.deg[jb + 1], payB = sm.payload[jb + 1],
-                       srcB = sm.src[jb + 1];
-        uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
-        bool valid[kEdgesPerThread];
-        uint32_t c = 0;
-#pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q) {
-            const uint32_t e = bw + 4 * lane + q;
-            c += (nb >> q) & 1u;
-            const int j = jb + (int)c;
-            valid[q] = e < total;
-            uint32_t pj, oj, dj;
-            if (c == 0) { pj = preA; oj = offA; dj = degA; pl[q] = payA; src[q] = srcA; }
-            else if (c == 1) { pj = preB; oj = offB; dj = degB; pl[q] = payB; src[q] = srcB; }
-            else { pj = sm.pre[j]; oj = sm.off[j]; dj = sm.deg[j]; pl[q] = sm.payload[j]; src[q] = sm.src[j]; }
-            const uint32_t* adj = words + oj;
-            const uint32_t local = e - pj;
-            dst[q] = valid[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
-            w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_l1_u32(adj + dj + local, pol) : 0u;
-        }
-#pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q) dst[q] = decode_entry(ps, dst[q]);
-        op.edges(dst, w, pl, src, valid);
-        j0 += ns;
-    }
-}
-
 // Sparse page (frontier-driven ops, < 1/4 of the page's vertices selected):
 // compact the page's frontier vertices from the bitmap in passes of
 // kListWords words, then expand them in batches of kTile with gather_items.
@@ -297,8 +235,7 @@ __device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, cons
             }
             if (tid == 0) sm.pre[nf] = total;
             __syncthreads();
-            if (ps.ww & 2u) gather_items_ww(ps, op, sm, words, nf, total, pol);
-            else gather_items(ps, op, sm, words, nf, total, pol);
+            gather_items(ps, op, sm, words, nf, total, pol);
             __syncthreads();
         }
     }
@@ -597,69 +534,17 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 // dense: the selected edges are >= half of the tile's record words.  Weighted
                 // records hold 2 words per edge, so there a tile is dense only when nearly
                 // every vertex is selected -- measured the better choice for SSSP (RMAT-27
-                // 35.7 ms vs 42.8 ms when the words are counted, ps.wdense = 1; ps.wdense = 2
-                // never streams weighted tiles)
-                const uint32_t selw = (Op::kWeighted && ps.wdense == 1) ? 2 * total : total;
-                const bool dense = 2 * selw >= W1 - W0 && !(Op::kWeighted && ps.wdense == 2);
-                if (dense && (ps.ww & 1u)) {
+                // 35.7 ms vs 42.8 ms when the selected words are counted instead)
+                const bool dense = 2 * total >= W1 - W0;
+                if (dense) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
-                    // 128-word windows; owners from record-start masks (no binary search)
+                    // 128-word windows; owners from record-start masks (no binary search;
+                    // RMAT-27 SSSP 33.8 vs 36.2 ms, WCC 13.7 vs 14.2 ms against a binary
+                    // search per 16 bytes, BFS equal)
                     if (ps.entry_encoding == GTS_ENTRY_VID32)
                         dense_tile_ww<Op, true>(ps, op, sm, q4, words, start + t0, nv, W0, W1, pol);
                     else
                         dense_tile_ww<Op, false>(ps, op, sm, q4, words, start + t0, nv, W0, W1, pol);
-                    __syncthreads();
-                    continue;
-                }
-                if (dense) {
-                    // dense tile: stream the whole record region with 16-byte loads and
-                    // act on the words of selected owners (hybrid micro-level, App E)
-                    const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
-                    for (uint32_t qb = qbeg + tid; qb < qend; qb += kThreads * kDenseUnroll) {
-                        uint4 vv[kDenseUnroll];
-#pragma unroll
-                        for (int u = 0; u < kDenseUnroll; ++u) {
-                            const uint32_t q = qb + u * kThreads;
-                            if (q < qend) vv[u] = ld_stream_v4(q4 + q, pol);
-                        }
-#pragma unroll
-                        for (int u = 0; u < kDenseUnroll; ++u) {
-                            const uint32_t q = qb + u * kThreads;
-                            if (q >= qend) break;
-                            const uint32_t w0 = 4 * q;
-                            uint32_t lo = 0, hi = nv;
-                            while (hi - lo > 1) {
-                                const uint32_t mid = (lo + hi) >> 1;
-                                if (sm.soff[mid] <= w0) lo = mid; else hi = mid;
-                            }
-                            uint32_t j = lo, cur = sm.soff[j], nxt = sm.soff[j + 1];
-                            uint32_t dst[kEdgesPerThread], wt[kEdgesPerThread], pl[kEdgesPerThread],
-                                src[kEdgesPerThread];
-                            bool valid[kEdgesPerThread];
-#pragma unroll
-                            for (int k = 0; k < 4; ++k) {
-                                const uint32_t w = w0 + k;
-                                bool ok = w >= W0 && w < W1;
-                                if (ok) {
-                                    while (w >= nxt) {
-                                        ++j;
-                                        cur = nxt;
-                                        nxt = sm.soff[j + 1];
-                                    }
-                                    const uint32_t rel = w - cur, dj = (nxt - cur - 1) >> (Op::kWeighted ? 1 : 0);
-                                    ok = rel >= 1 && rel <= dj && sm.sel[j];
-                                    wt[k] = (Op::kReadWeights && ok) ? ld_stream_l1_u32(words + w + dj, pol) : 0u;
-                                } else {
-                                    wt[k] = 0u;
-                                }
-                                valid[k] = ok;
-                                dst[k] = decode_entry(ps, word_of(vv[u], k));
-                                pl[k] = sm.paytile[j];
-                                src[k] = start + t0 + j;
-                            }
-                            op.edges(dst, wt, pl, src, valid);
-                        }
-                    }
                     __syncthreads();
                     continue;
                 }
@@ -673,8 +558,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 }
                 if (tid == 0) sm.pre[nf] = total;
                 __syncthreads();
-                if (ps.ww & 2u) gather_items_ww(ps, op, sm, words, nf, total, pol);
-                else gather_items(ps, op, sm, words, nf, total, pol);
+                gather_items(ps, op, sm, words, nf, total, pol);
                 __syncthreads();
             }
         }

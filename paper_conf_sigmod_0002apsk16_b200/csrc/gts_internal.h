@@ -64,7 +64,30 @@ struct Graph {
     std::vector<uint32_t> old_of_new;  // internal ID -> caller VID
     bool host_registered = false;      // pages cudaHostRegister'ed by a context
     bool maps_registered = false;      // new_of_old / old_of_new registered too
+    bool symmetric = false;            // GTS_BUILD_SYMMETRIC: every edge stored in both directions
+    // GTS_BUILD_OWNER_FILTER: only the pages rank owner_rank of owner_world processes under
+    // owner_strategy are held, compacted in ascending page ID; host_loc[pid] = index in pages
+    // (UINT32_MAX: not held).  owner_rank = -1: every page held, host_loc empty (identity).
+    int32_t owner_rank = -1;
+    uint32_t owner_world = 1, owner_strategy = 0;
+    std::vector<uint32_t> host_loc;
+    uint64_t n_host_pages = 0;
 };
+
+// host address of page pid (nullptr if this graph does not hold it)
+inline const uint8_t* host_page(const Graph* g, uint64_t pid) {
+    if (g->host_loc.empty()) return g->pages + pid * (uint64_t)g->page_bytes;
+    const uint32_t l = g->host_loc[pid];
+    return l == UINT32_MAX ? nullptr : g->pages + (uint64_t)l * g->page_bytes;
+}
+
+// Page -> rank assignment of a strategy (P:352-354 Strategy-P h(j) = j mod N;
+// P:430-434 Strategy-S contiguous WA ranges cut at page boundaries with ~equal
+// page counts, never inside an LP run).  vrange[world+1]: rank r owns WA
+// [vrange[r], vrange[r+1]).  Needs only the directory (n, num_pages, start_vid,
+// kind, lp_first).
+void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t>& owner,
+               std::vector<uint64_t>& vrange);
 
 struct PagePlanEntry {
     uint32_t start_vid;

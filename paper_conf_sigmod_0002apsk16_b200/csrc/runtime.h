@@ -5,6 +5,7 @@
 #include <nccl.h>
 
 #include <chrono>
+#include <map>
 #include <cstdlib>
 #include <utility>
 #include <vector>
@@ -53,8 +54,6 @@ struct PageSet {
     uint32_t entry_encoding;
     const uint32_t* rvt_start; // START_VID per page (PID16 decode)
     uint32_t hybrid_deg = 8;   // GTS_MICRO_HYBRID: vertex-centric below this many edges per vertex (R24)
-    uint32_t ww = 0;           // dense tiles by warp windows (expand.cuh dense_tile_ww)
-    uint32_t wdense = 0;       // weighted pages' dense-tile test: 0 edges vs words, 1 words vs words, 2 never
     uint32_t split = 1;        // work items per page: an LP's chunk is cut into `split` slices
                                // (small page sets, e.g. a hub's LPs at BFS level 0); SPs use slice 0
 };
@@ -83,6 +82,8 @@ struct DevGraph {
     std::vector<unsigned long long> pb_count;
     uint64_t pb_key = 0;
     std::vector<uint64_t> h_vrange;    // all ranks' WA ranges (world + 1)
+    // Strategy-S route capacities (comm.cu route_capacities), per (skip, world, strategy)
+    std::map<uint64_t, std::vector<uint64_t>> route_caps;
 };
 
 // LRU cache of topology pages in device memory for streamed BFS-like sweeps
@@ -149,19 +150,10 @@ void free_cache(PageCache& pc);
 // residency decision (GTS_RESIDENCY_AUTO: resident iff this rank's pages + attributes fit in free HBM)
 bool choose_streamed(Context* c, const Graph* g, const gts_run_config& rc, uint64_t attr_bytes);
 
-// P-strategy page ownership (h(j) = j mod N) and S ranges.
-void partition(const Graph* g, uint32_t strategy, int world, std::vector<int32_t>& owner,
-               std::vector<uint64_t>& vrange);
 
-// dense tiles by warp windows unless GTS_WW=0 (read per call so tests can switch it);
-// RMAT-27: SSSP 33.8 vs 36.2 ms, WCC 13.7 vs 14.2, BFS equal (profiles/r01_ww_dense.txt)
-// PageSet::ww bits: 1 = dense tiles by warp windows (default; GTS_WW=0 clears), 2 =
-// sparse tiles' item gather by warp windows (opt-in GTS_GWW=1: RMAT-27 BFS 7.79 vs
-// 7.62 ms, SSSP 36.0 vs 36.3 ms, WCC 12.8 vs 12.7 ms against the binary search)
-inline uint32_t env_ww() {
-    const char* e = getenv("GTS_WW");
-    const char* g = getenv("GTS_GWW");
-    return (e && atoi(e) == 0 ? 0u : 1u) | (g && atoi(g) > 0 ? 2u : 0u);
+// persisting-L2 window size of a call (gts_run_config.l2_persist_mib: 0 = 96 MiB, GTS_OFF = none)
+inline size_t l2_persist_mib(const gts_run_config& rc) {
+    return rc.l2_persist_mib == GTS_OFF ? 0 : rc.l2_persist_mib ? rc.l2_persist_mib : 96;
 }
 
 inline double now_s() {

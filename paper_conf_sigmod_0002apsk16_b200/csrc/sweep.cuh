@@ -48,7 +48,6 @@ int sweep_pages(Context* c, const Graph* g, const gts_run_config& rc, bool strea
         ps.mode = d.all_local ? kAddrByPid : kAddrByLoc;
         ps.entry_encoding = g->entry_encoding;
         ps.rvt_start = d.rvt_start;
-        ps.ww = env_ww();
         GTS_TRY(launch(ps, 1 << 30));
         ss->launches++;
         return GTS_OK;
@@ -70,11 +69,13 @@ int sweep_pages(Context* c, const Graph* g, const gts_run_config& rc, bool strea
             cudaEventRecord(ev.first, c->copy_stream);
         }
         uint32_t i = 0;
-        while (i < nb) {
+        while (i < nb) {             // runs of pages adjacent in host memory: one copy each
+            const uint8_t* h0 = host_page(g, L[b0 + i]);
+            if (!h0) return fail(GTS_EINVAL, "graph does not hold page %u", L[b0 + i]);
             uint32_t j = i + 1;
-            while (j < nb && L[b0 + j] == L[b0 + j - 1] + 1) ++j;
-            GTS_CUDA(cudaMemcpyAsync(dst + (size_t)i * pb, g->pages + (size_t)L[b0 + i] * pb, (size_t)(j - i) * pb,
-                                     cudaMemcpyHostToDevice, c->copy_stream));
+            while (j < nb && host_page(g, L[b0 + j]) == h0 + (size_t)(j - i) * pb) ++j;
+            GTS_CUDA(cudaMemcpyAsync(dst + (size_t)i * pb, h0, (size_t)(j - i) * pb, cudaMemcpyHostToDevice,
+                                     c->copy_stream));
             i = j;
         }
         if (timing) cudaEventRecord(ev.second, c->copy_stream);
@@ -90,7 +91,6 @@ int sweep_pages(Context* c, const Graph* g, const gts_run_config& rc, bool strea
         ps.mode = kAddrByPos;
         ps.entry_encoding = g->entry_encoding;
         ps.rvt_start = d.rvt_start;
-        ps.ww = env_ww();
         GTS_TRY(launch(ps, (int)nb));
         GTS_CUDA(cudaEventRecord(c->ring_free[slot], c->stream));
         ss->h2d_bytes += (uint64_t)nb * pb;
@@ -180,7 +180,6 @@ int sweep_pages_cached(Context* c, const Graph* g, const gts_run_config& rc, con
         ps.mode = kAddrByLoc;
         ps.entry_encoding = g->entry_encoding;
         ps.rvt_start = c->dg.rvt_start;
-        ps.ww = env_ww();
         return ps;
     };
     if (!hits.empty()) {                          // overlaps the miss copies below
@@ -194,8 +193,9 @@ int sweep_pages_cached(Context* c, const Graph* g, const gts_run_config& rc, con
         const uint32_t ev = bi % rc.ring_slots;
         for (uint32_t k = 0; k < nb; ++k) {
             const uint32_t p = miss[b0 + k];
-            GTS_CUDA(cudaMemcpyAsync(pc.buf + (size_t)pc.loc[p] * pb, g->pages + (size_t)p * pb, pb,
-                                     cudaMemcpyHostToDevice, c->copy_stream));
+            const uint8_t* hp = host_page(g, p);
+            if (!hp) return fail(GTS_EINVAL, "graph does not hold page %u", p);
+            GTS_CUDA(cudaMemcpyAsync(pc.buf + (size_t)pc.loc[p] * pb, hp, pb, cudaMemcpyHostToDevice, c->copy_stream));
         }
         GTS_CUDA(cudaEventRecord(c->ring_ready[ev], c->copy_stream));
         GTS_CUDA(cudaStreamWaitEvent(c->stream, c->ring_ready[ev], 0));

@@ -23,8 +23,11 @@
 #include <algorithm>
 #include <cstring>
 
+#include "comm.h"
 #include "expand.cuh"
+#include "route.cuh"
 #include "sweep.cuh"
+#include "traverse.h"
 
 namespace gts {
 
@@ -177,20 +180,27 @@ sssp_check_kernel(PageSet ps, const uint32_t* __restrict__ dist, uint32_t* work_
     if (__syncthreads_or(op.bad) && threadIdx.x == 0) *bad_flag = 1u;
 }
 
-// Merge the per-rank next frontiers (world > 1: OR of the all-gathered
-// bitmaps), add them to visited, write LV = new_level once per newly reached
-// vertex (when level != nullptr) and count them.
-__global__ void frontier_finish_kernel(const uint32_t* __restrict__ gathered, int world, uint64_t words,
-                                       uint32_t* next, uint32_t* visited, uint32_t* level, uint32_t new_level,
-                                       unsigned long long* count) {
+// Merge the per-rank next frontiers and count them, over bitmap words [w0, w1)
+// (bitmap pointers are biased: word w of the rank's range is ptr[w]).
+// gathered != nullptr (Strategy-P / S_BCAST): the world ranks' next bitmaps
+// all-gathered [world][gwords]; their OR becomes next and is added to visited.
+// gathered == nullptr: next already holds the merged frontier (one rank, or
+// Strategy-S after the routed apply).  LV = new_level is written once per newly
+// reached vertex when level != nullptr.
+__global__ void frontier_finish_kernel(const uint32_t* __restrict__ gathered, int world, uint64_t gwords, uint64_t w0,
+                                       uint64_t w1, uint32_t* next, uint32_t* visited, uint32_t* level,
+                                       uint32_t new_level, unsigned long long* count) {
     unsigned long long c = 0;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
-        uint32_t bits = gathered[w];
-        for (int r = 1; r < world; ++r) bits |= gathered[(uint64_t)r * words + w];
-        if (world > 1) {
+    for (uint64_t w = w0 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < w1; w += stride) {
+        uint32_t bits;
+        if (gathered) {
+            bits = gathered[w];
+            for (int r = 1; r < world; ++r) bits |= gathered[(uint64_t)r * gwords + w];
             next[w] = bits;
             if (visited) visited[w] |= bits;
+        } else {
+            bits = next[w];
         }
         c += __popc(bits);
         if (level) {
@@ -204,19 +214,25 @@ __global__ void frontier_finish_kernel(const uint32_t* __restrict__ gathered, in
     block_add_u64(c, count);
 }
 
-// SSSP near-far pending set: new pending = improved this round (next, merged over
-// ranks) + pending vertices that were not expanded (dist > T).  Counts the
-// pending vertices, those already within T, and the minimum pending distance.
-__global__ void sssp_finish_kernel(const uint32_t* __restrict__ gathered, int world, uint64_t words,
-                                   const uint32_t* __restrict__ cur, uint32_t* next, const uint32_t* __restrict__ dist,
-                                   uint32_t T, unsigned long long* count, unsigned long long* near,
-                                   unsigned int* minpend) {
+// SSSP near-far pending set over words [w0, w1) (biased pointers): new pending =
+// improved this round (next, or the OR of the all-gathered per-rank bitmaps) +
+// pending vertices that were not expanded (dist > T).  Counts the pending
+// vertices, those already within T, and the minimum pending distance.
+__global__ void sssp_finish_kernel(const uint32_t* __restrict__ gathered, int world, uint64_t gwords, uint64_t w0,
+                                   uint64_t w1, const uint32_t* __restrict__ cur, uint32_t* next,
+                                   const uint32_t* __restrict__ dist, uint32_t T, unsigned long long* count,
+                                   unsigned long long* near, unsigned int* minpend) {
     unsigned long long c = 0, nr = 0;
     uint32_t mn = 0xFFFFFFFFu;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
-        uint32_t bits = gathered[w];
-        for (int r = 1; r < world; ++r) bits |= gathered[(uint64_t)r * words + w];
+    for (uint64_t w = w0 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < w1; w += stride) {
+        uint32_t bits;
+        if (gathered) {
+            bits = gathered[w];
+            for (int r = 1; r < world; ++r) bits |= gathered[(uint64_t)r * gwords + w];
+        } else {
+            bits = next[w];
+        }
         uint32_t keep = cur[w] & ~bits;
         while (keep) {
             const int b = __ffs(keep) - 1;
@@ -465,27 +481,16 @@ static PageSet resident_set(Context* c, const Graph* g, const uint32_t* list, co
     ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
     ps.entry_encoding = g->entry_encoding;
     ps.rvt_start = c->dg.rvt_start;
-    ps.ww = env_ww();
     return ps;
 }
 
-enum Algo { kBFS, kSSSP };
-
-static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_run_config* cfg, uint32_t* out,
-                    gts_run_stats* st, Algo algo) {
-    clear_error();
-    const double t_start = now_s();
-    gts_run_config rc;
-    GTS_TRY(validate_common(c, g, cfg, &rc));
-    if (!out) return fail(GTS_EINVAL, "NULL output");
-    if (src >= g->n) return fail(GTS_EINVAL, "src %llu >= n %llu", (unsigned long long)src, (unsigned long long)g->n);
-    if (algo == kSSSP && !g->weighted) return fail(GTS_EUNSUPPORTED, "gts_sssp needs a graph built with weights");
+// One rank (world 1, no virtual ranks): the tuned single-GPU path (level
+// slots, batched levels, degree-ordered byte levels, LP slicing, page cache).
+static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, const gts_run_config& rc, uint32_t* out,
+                           gts_run_stats* st, int algo, double t_start, bool streamed, double upload_s) {
     const uint64_t n = g->n, words = (n + 31) / 32;
-    const bool streamed = choose_streamed(c, g, rc, 4 * n + 16 * words);
-    double upload_s = 0;
-    GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
     const bool timing = rc.flags & GTS_RUN_TIMING;
-    uint32_t *value, *visited = nullptr, *cur, *next, *list, *gathered = nullptr;
+    uint32_t *value, *visited = nullptr, *cur, *next, *list;
     Counters* ctr;
     GTS_TRY(c->buf(kBufValue, n * 4, (void**)&value));
     if (algo == kBFS) GTS_TRY(c->buf(kBufVisited, words * 4, (void**)&visited));
@@ -493,18 +498,17 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     GTS_TRY(c->buf(kBufNext, words * 4, (void**)&next));
     GTS_TRY(c->buf(kBufList, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&list));
     GTS_TRY(c->buf(kBufCtr, sizeof(Counters), (void**)&ctr));
-    if (c->world > 1) GTS_TRY(c->buf(kBufGather, words * 4 * c->world, (void**)&gathered));
     cudaStream_t s = c->stream;
     // BFS level slots: the frontier of level L lives in slot L of a K-slot bitmap
     // store, and LV is written once at the end by level_fill_kernel.  A traversal
     // deeper than K levels fills LV from the slots and continues with the
     // ping-pong frontiers, writing LV per level in frontier_finish_kernel.
-    // GTS_BFS_SLOTS=<K> (0 = per-level LV writes throughout); default 32, capped at 1 GiB.
+    // gts_run_config.bfs_level_slots = K (GTS_OFF: per-level LV writes throughout); default 32,
+    // capped at 1 GiB.
     uint32_t K = 0;
     uint32_t* lvb = nullptr;
     if (algo == kBFS) {
-        const char* ke = getenv("GTS_BFS_SLOTS");
-        K = ke ? (uint32_t)std::max(0L, atol(ke)) : 32u;
+        K = rc.bfs_level_slots == GTS_OFF ? 0u : rc.bfs_level_slots ? rc.bfs_level_slots : 32u;
         K = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(K, 255), (1ull << 30) / (words * 4));
         if (K < 3) K = 0;
         if (K) {
@@ -540,23 +544,19 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         {bfs_expand_kernel<true, kMicroTile>, bfs_expand_kernel<true, kMicroEdge>,
          bfs_expand_kernel<true, kMicroVertex>, bfs_expand_kernel<true, kMicroHybrid>}};
     BfsKern bfs_kern = bfs_k[g->weighted ? 1 : 0][micro];
-    // three 512-thread CTAs per SM (40 registers, a few spilled bytes) by default: the
-    // per-tile barriers of one CTA are covered by the other two (RMAT-27 BFS kernels
-    // 10.25 -> 9.26 ms); GTS_BFS_OCC=2 selects two CTAs (64 registers)
-    const char* oce = getenv("GTS_BFS_OCC");
-    if (micro == kMicroTile && (!oce || atoi(oce) != 2))
+    // three 512-thread CTAs per SM (40 registers): the per-tile barriers of one CTA are
+    // covered by the other two (RMAT-27 BFS kernels 10.25 -> 9.26 ms against two)
+    if (micro == kMicroTile)
         bfs_kern = g->weighted ? bfs_expand_kernel<true, kMicroTile, 3> : bfs_expand_kernel<false, kMicroTile, 3>;
-    const char* hde = getenv("GTS_HYBRID_DEG");
-    const uint32_t hybrid_deg = hde ? (uint32_t)std::max(1L, atol(hde)) : 8u;
-    // GTS_SSSP_OCC=3: three 512-thread CTAs per SM for the SSSP expansion (RMAT-27: 35.7 vs
-    // 35.1 ms for two -- the weighted walk spills 124 bytes at 40 registers -- so off by default)
-    const char* soe = getenv("GTS_SSSP_OCC");
-    auto sssp_kern = (soe && atoi(soe) == 3) ? sssp_expand_kernel<3> : sssp_expand_kernel<2>;
+    const uint32_t hybrid_deg = rc.hybrid_deg ? rc.hybrid_deg : 8u;
+    // two 512-thread CTAs per SM for the SSSP expansion (three measured 35.7 vs 35.1 ms on
+    // RMAT-27: the weighted walk spills at 40 registers)
+    auto sssp_kern = sssp_expand_kernel<2>;
     const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_kern;
     int grid = 0;
     GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
     const int fin_grid = c->num_sms * 4;
-    uint64_t pages_processed = l0.size(), nccl_bytes = 0;
+    uint64_t pages_processed = l0.size();
     uint32_t levels = 0;
     Counters h;
     SweepStats ss;
@@ -567,33 +567,25 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
     // is within it.  Label-correcting, so any delta gives the exact distances.
     // Default unbounded (plain frontier Bellman-Ford): on RMAT-27 delta 16 / 64 /
     // 256 / unbounded measured 71 / 49 / 38 / 36 ms -- low-diameter power-law
-    // graphs waste few relaxations.  GTS_SSSP_DELTA=<w> selects a bucket width.
-    const char* de = getenv("GTS_SSSP_DELTA");
-    const uint64_t delta = de ? std::max<long>(1, atol(de)) : 0xFFFFFFFEull;
+    // graphs waste few relaxations.  gts_run_config.sssp_delta selects a bucket width.
+    const uint64_t delta = rc.sssp_delta ? rc.sssp_delta : 0xFFFFFFFEull;
     uint32_t T = algo == kSSSP ? (uint32_t)std::min<uint64_t>(delta, 0xFFFFFFFEull) : 0xFFFFFFFEu;
     // Persisting-L2 window on the structure every edge probes: SSSP on degree-ordered
     // pages the dense head [0, W) of dist (the most relaxed entries), BFS the visited
     // bitmap.  It also replaces lines an earlier PageRank call left persisting.
-    // GTS_L2_PERSIST_SSSP / GTS_L2_PERSIST_BFS = <MiB>, 0 = off.
+    // gts_run_config.l2_persist_mib (0 = 96 MiB, GTS_OFF = none).
     bool persist = false;
     if (!streamed && (algo == kBFS || g->ordered)) {
-        const char* pe = getenv(algo == kBFS ? "GTS_L2_PERSIST_BFS" : "GTS_L2_PERSIST_SSSP");
-        const size_t want = std::min<size_t>((size_t)(pe ? atol(pe) : 96) << 20, algo == kBFS ? words * 4 : n * 4);
+        const size_t want = std::min<size_t>((size_t)l2_persist_mib(rc) << 20, algo == kBFS ? words * 4 : n * 4);
         if (want > 0) {
             GTS_TRY(persist_window(c, s, algo == kBFS ? (void*)visited : (void*)value, want));
             persist = true;
         }
     }
-    const char* wde = getenv("GTS_WDENSE");
-    const uint32_t wdense = wde ? (uint32_t)std::min(2, std::max(0, atoi(wde))) : 0u;
-    const char* spe = getenv("GTS_SPLIT");
-    const bool split_on = !spe || atoi(spe) > 0;
-    // BFS on resident pages, one rank: levels are enqueued GTS_BFS_BATCH (default 8) at a
-    // time without a host round trip (per-level new-vertex counts and page-list counts go
+    // BFS on resident pages, one rank: levels are enqueued levels_per_sync (default 8) at
+    // a time without a host round trip (per-level new-vertex counts and page-list counts go
     // to device arrays; the levels after the last non-empty one run on an empty frontier)
-    const char* bbe = getenv("GTS_BFS_BATCH");
-    const uint32_t B = (algo == kBFS && !streamed && c->world == 1 && K > 0)
-                           ? (uint32_t)std::max(1L, bbe ? atol(bbe) : 8L) : 1u;
+    const uint32_t B = (algo == kBFS && !streamed && K > 0) ? (rc.levels_per_sync ? rc.levels_per_sync : 8u) : 1u;
     unsigned long long* lvl_cnt = nullptr;           // [K] new vertices per level (BFS)
     uint32_t* lvl_pages = nullptr;                   // [K] pages in the list of level L
     if (algo == kBFS) {
@@ -612,10 +604,9 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
                                 PageSet p2 = ps;
                                 p2.hybrid_deg = hybrid_deg;
-                                p2.wdense = wdense;
                                 // few pages in this level (e.g. the source hub's LPs): slice LPs so
-                                // every CTA gets work, decided on the device (GTS_SPLIT=0 disables)
-                                p2.split = split_on ? 0u : 1u;
+                                // every CTA gets work, decided on the device
+                                p2.split = 0u;
                                 const int gl = std::min(grid, cap);
                                 if (algo == kBFS) {
                                     bfs_kern<<<gl, kThreads, 0, s>>>(
@@ -632,20 +623,12 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         else GTS_TRY(sweep_pages(c, g, rc, streamed, &h_list, list, (uint32_t)h_list.size(), &ctr->list_count,
                                  launch, &ss));
         std::pair<cudaEvent_t, cudaEvent_t> ev;
-        if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
-        if (c->world > 1) {
-            GTS_NCCL(ncclGroupStart());
-            if (algo == kSSSP) GTS_NCCL(ncclAllReduce(value, value, n, ncclUint32, ncclMin, c->comm, s));
-            GTS_NCCL(ncclAllGather(next, gathered, words, ncclUint32, c->comm, s));
-            GTS_NCCL(ncclGroupEnd());
-            nccl_bytes += words * 4 + (algo == kSSSP ? n * 4 : 0);
-        }
-        if (timing) { cudaEventRecord(ev.second, s); ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
+        if (timing) { ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
         GTS_CUDA(cudaMemsetAsync(&ctr->count, 0, 8, s));
         GTS_CUDA(cudaMemsetAsync(&ctr->list_count, 0, 4, s));
         if (algo == kBFS) {
-            frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, next,
-                                                            visited, slots ? nullptr : value, L + 1,
+            frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(nullptr, 1, words, 0, words, next, visited,
+                                                            slots ? nullptr : value, L + 1,
                                                             L < K ? lvl_cnt + L : &ctr->count);
             GTS_CUDA(cudaMemsetAsync(&ctr->vprefix_words, 0xFF, 4, s));
             visited_prefix_kernel<<<fin_grid, 256, 0, s>>>(visited, words, &ctr->vprefix_words);
@@ -653,8 +636,8 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         } else {
             GTS_CUDA(cudaMemsetAsync(&ctr->near, 0, 8, s));
             GTS_CUDA(cudaMemsetAsync(&ctr->minpend, 0xFF, 4, s));
-            sssp_finish_kernel<<<fin_grid, 256, 0, s>>>(c->world > 1 ? gathered : next, c->world, words, cur, next,
-                                                        value, T, &ctr->count, &ctr->near, &ctr->minpend);
+            sssp_finish_kernel<<<fin_grid, 256, 0, s>>>(nullptr, 1, words, 0, words, cur, next, value, T,
+                                                        &ctr->count, &ctr->near, &ctr->minpend);
         }
         frontier_pages_kernel<<<fin_grid, 256, 0, s>>>(next, c->dg.rvt_start, c->dg.nslots,
                                                        c->dg.all_local ? nullptr : c->dg.local_list,
@@ -753,11 +736,6 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         ++launches;
     }
     if (persist) GTS_TRY(persist_window(c, s, nullptr, 0));
-    if (algo == kSSSP && c->world > 1) {   // every rank must agree before the collective check
-        GTS_NCCL(ncclAllReduce(&ctr->flag, &ctr->flag, 1, ncclUint32, ncclMax, c->comm, s));
-        GTS_CUDA(cudaMemcpyAsync(&h.flag, &ctr->flag, 4, cudaMemcpyDeviceToHost, s));
-        GTS_CUDA(cudaStreamSynchronize(s));
-    }
     if (algo == kSSSP && h.flag) {
         // exact overflow test (see SsspOp::edges): sweep all local pages once
         GTS_CUDA(cudaMemsetAsync(&ctr->flag2, 0, 4, s));
@@ -774,7 +752,6 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
                                 return GTS_OK;
                             }, &ss));
         uint32_t bad = 0;
-        if (c->world > 1) GTS_NCCL(ncclAllReduce(&ctr->flag2, &ctr->flag2, 1, ncclUint32, ncclMax, c->comm, s));
         GTS_CUDA(cudaMemcpyAsync(&bad, &ctr->flag2, 4, cudaMemcpyDeviceToHost, s));
         GTS_CUDA(cudaStreamSynchronize(s));
         if (bad) return fail(GTS_EOVERFLOW, "an SSSP distance reaches 2^32-1");
@@ -796,7 +773,7 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         st->cache_misses = ss.cache_misses;
         if (timing) st->h2d_s = c->t_h2d.sum_s();
         st->edges_traversed = h.edges;
-        st->nccl_bytes = nccl_bytes;
+        st->wa_bytes = (uint64_t)n * 4 + (uint64_t)(algo == kBFS ? 3 : 2) * words * 4;
         st->launches = launches + main_launches;
         st->main_kernel_launches = main_launches;
         st->levels_or_iters = levels;
@@ -807,6 +784,552 @@ static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_
         c->t_h2d.sum_s();
     }
     return GTS_OK;
+}
+
+// ------------------------------------------------------- multi-rank path ---
+// N ranks (real, one per process, or virtual on one GPU; comm.h), Strategy-P,
+// Strategy-S with routed updates, or the paper-literal S_BCAST:
+//   P       pages h(j) = j mod N, WA replicated; per level every rank expands
+//           its frontier pages into its own next bitmap, the bitmaps are
+//           all-gathered and OR-ed (NCCL has no bitwise OR);
+//           SSSP also all-reduces dist with min.
+//   S       rank r owns WA [lo, hi) and the pages whose sources lie in it; a
+//           remote destination becomes a message to its owner (BFS: dst,
+//           deduplicated per sender by a sent bitmap; SSSP: (dst, dist);
+//           WCC: (dst, label)), exchanged with grouped send/recv and applied
+//           by the owner; frontier counts are all-reduced.
+//   S_BCAST every rank expands every frontier page but applies only updates
+//           into its own range; the ranges are merged as under P.
+// WCC under S is push-only min-label propagation on GTS_BUILD_SYMMETRIC pages
+// (each edge is stored at both endpoints, so the owner of either endpoint
+// pushes along it; SURVEY 8(e) WCC caveat): the result, the minimum VID of
+// each weakly connected component, is the union-find result.
+
+enum { kDstAll = 0, kDstRoute = 1, kDstDrop = 2 };   // remote destinations: (none under P), route, drop
+
+__device__ __forceinline__ bool in_range(uint32_t v, uint64_t lo, uint64_t hi) { return (uint64_t)v - lo < hi - lo; }
+
+template <bool W>
+struct MBfsOp {
+    static constexpr bool kReadWeights = false;
+    static constexpr bool kWeighted = W;
+    const uint32_t* cur;       // biased bitmaps (word w of the rank's range at ptr[w])
+    uint32_t* visited;
+    uint32_t* next;
+    uint32_t* sent;            // Strategy-S: remote vertices already sent by this rank (full n bits)
+    unsigned long long nedges;
+    uint64_t lo, hi;
+    int mode;
+    RouteOut ro;
+    __device__ const uint32_t* frontier() const { return cur; }
+    __device__ bool select(uint32_t v) { return test_bit(cur, v); }
+    __device__ uint32_t payload(uint32_t, uint32_t deg) {
+        nedges += deg;
+        return 0u;
+    }
+    __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t len, uint32_t&) {
+        if (!test_bit(cur, vid)) return false;
+        if (threadIdx.x == 0) nedges += len;
+        return true;
+    }
+    // Alg 2 lines 17-20 for local destinations (exactly-once discovery through the
+    // visited bit); remote ones go to their owner once per traversal (sent bit).
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t*, const uint32_t*, const uint32_t*,
+                                          const bool* valid) {
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            if (!valid[q]) continue;
+            const uint32_t v = dst[q], wi = v >> 5, b = 1u << (v & 31);
+            if (in_range(v, lo, hi)) {
+                if (!(__ldcg(visited + wi) & b) && !(atomicOr(visited + wi, b) & b)) atomicOr(next + wi, b);
+            } else if (mode == kDstRoute) {
+                if (!(__ldcg(sent + wi) & b) && !(atomicOr(sent + wi, b) & b)) route_push<uint32_t>(ro, v, v);
+            }
+        }
+    }
+    __device__ void end_page() {}
+};
+
+// SSSP relaxation (kMin = dist) and WCC label propagation share one op: the
+// payload of a selected vertex u is val[u]; an edge (u, v, w) offers val[u] + w
+// (SSSP) or val[u] (WCC) to v, applied with atomicMin; an improvement marks v.
+template <bool W, bool kSssp>
+struct MMinOp {
+    static constexpr bool kReadWeights = kSssp;
+    static constexpr bool kWeighted = W;
+    const uint32_t* cur;
+    uint32_t* val;             // biased: val[v] for v in [lo, hi)
+    uint32_t* next;
+    unsigned long long nedges;
+    bool ovf;
+    uint32_t T;                // SSSP near-far threshold
+    uint64_t lo, hi;
+    int mode;
+    RouteOut ro;
+    __device__ const uint32_t* frontier() const { return cur; }
+    __device__ bool select(uint32_t v) { return test_bit(cur, v) && (!kSssp || __ldcg(val + v) <= T); }
+    __device__ uint32_t payload(uint32_t v, uint32_t deg) {
+        nedges += deg;
+        return *((volatile uint32_t*)val + v);
+    }
+    __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t len, uint32_t& pl) {
+        if (!test_bit(cur, vid)) return false;
+        pl = *((volatile uint32_t*)val + vid);
+        if (kSssp && pl > T) return false;
+        if (threadIdx.x == 0) nedges += len;
+        return true;
+    }
+    __device__ __forceinline__ void edges(const uint32_t* dst, const uint32_t* w, const uint32_t* pu,
+                                          const uint32_t*, const bool* valid) {
+#pragma unroll
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            if (!valid[q]) continue;
+            uint32_t cand = pu[q];
+            if (kSssp) {
+                const uint64_t nd = (uint64_t)pu[q] + w[q];
+                if (nd >= (uint64_t)GTS_UNREACHED) {          // checked exactly after convergence
+                    ovf = true;
+                    continue;
+                }
+                cand = (uint32_t)nd;
+            }
+            const uint32_t v = dst[q];
+            if (in_range(v, lo, hi)) {
+                if (cand < __ldcg(val + v) && cand < atomicMin(val + v, cand)) atomicOr(next + (v >> 5), 1u << (v & 31));
+            } else if (mode == kDstRoute) {
+                route_push<uint2>(ro, v, make_uint2(v, cand));
+            }
+        }
+    }
+    __device__ void end_page() {}
+};
+
+template <bool W>
+__global__ void __launch_bounds__(kThreads, 2)
+mbfs_expand_kernel(PageSet ps, MBfsOp<W> op, uint32_t* work_ctr, unsigned long long* edges_out) {
+    __shared__ TileSmem sm;
+    expand_pages(ps, op, sm, work_ctr);
+    block_add_u64(op.nedges, edges_out);
+}
+
+template <bool W, bool kSssp>
+__global__ void __launch_bounds__(kThreads, 2)
+mmin_expand_kernel(PageSet ps, MMinOp<W, kSssp> op, uint32_t* work_ctr, unsigned long long* edges_out,
+                   uint32_t* ovf_flag) {
+    __shared__ TileSmem sm;
+    expand_pages(ps, op, sm, work_ctr);
+    block_add_u64(op.nedges, edges_out);
+    if (__syncthreads_or(op.ovf) && threadIdx.x == 0) *ovf_flag = 1u;
+}
+
+struct RecvView {
+    const uint8_t* recv;
+    uint64_t off[kMaxRanks];
+    const unsigned long long* cnt;   // device, per peer
+    int nranks;
+};
+
+// owner side of the routed BFS: exactly-once discovery of each received vertex
+__global__ void bfs_apply_kernel(RecvView rv, uint32_t* visited, uint32_t* next) {
+    const uint32_t* m = reinterpret_cast<const uint32_t*>(rv.recv);
+    for (int p = 0; p < rv.nranks; ++p) {
+        const uint64_t c = rv.cnt[p];
+        for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < c; i += (uint64_t)gridDim.x * blockDim.x) {
+            const uint32_t v = m[rv.off[p] + i], wi = v >> 5, b = 1u << (v & 31);
+            if (!(atomicOr(visited + wi, b) & b)) atomicOr(next + wi, b);
+        }
+    }
+}
+
+// owner side of routed SSSP / WCC: val[v] = min(val[v], x), mark v if it decreased
+__global__ void min_apply_kernel(RecvView rv, uint32_t* val, uint32_t* next) {
+    const uint2* m = reinterpret_cast<const uint2*>(rv.recv);
+    for (int p = 0; p < rv.nranks; ++p) {
+        const uint64_t c = rv.cnt[p];
+        for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < c; i += (uint64_t)gridDim.x * blockDim.x) {
+            const uint2 e = m[rv.off[p] + i];
+            if (e.y < atomicMin(val + e.x, e.y)) atomicOr(next + (e.x >> 5), 1u << (e.x & 31));
+        }
+    }
+}
+
+// val[v] = v and frontier bit set for every v in [lo, hi) (WCC label propagation start)
+__global__ void wcc_lp_init_kernel(uint32_t* val, uint32_t* cur, uint64_t lo, uint64_t hi) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t v = lo + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < hi; v += stride) {
+        val[v] = (uint32_t)v;
+        atomicOr(cur + (v >> 5), 1u << (v & 31));
+    }
+}
+
+__global__ void set_source_range_kernel(uint32_t* value, uint32_t* visited, uint32_t* cur, uint64_t src) {
+    value[src] = 0;
+    if (visited) visited[src >> 5] |= 1u << (src & 31);
+    cur[src >> 5] |= 1u << (src & 31);
+}
+
+struct MSlot {
+    int r = 0;
+    uint64_t lo = 0, hi = 0, w0 = 0, w1 = 0;   // WA range and the bitmap words it covers
+    uint32_t *value = nullptr, *visited = nullptr, *cur = nullptr, *next = nullptr, *sent = nullptr;  // biased
+    uint32_t *gathered = nullptr, *list = nullptr, *d_pages = nullptr;
+    Counters* ctr = nullptr;
+    std::vector<uint32_t> pages, h_list;
+    Counters h = {};
+};
+
+constexpr int kBufMulti = 200;     // scratch slots of local slot i: kBufMulti + 16 i + k
+constexpr int kBufRoute = 100;     // route buffers (comm.cu route_setup)
+constexpr int kBufResult = 199;    // assembled full-n result
+
+int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_run_config& rc, Ranks& R, void* out,
+                   gts_run_stats* st, int algo, double t_start, bool streamed, double upload_s) {
+    const uint64_t n = g->n, words = (n + 31) / 32;
+    const int N = R.world, L = R.nloc;
+    const uint32_t strat = rc.strategy;
+    const bool route = strat == GTS_STRATEGY_S;
+    const int mode = strat == GTS_STRATEGY_P ? kDstAll : route ? kDstRoute : kDstDrop;
+    if (algo == kWCCLP && !route) return fail(GTS_EINVAL, "label propagation is the Strategy-S WCC");
+    if (algo == kWCCLP && !g->symmetric)
+        return fail(GTS_EUNSUPPORTED, "gts_wcc under Strategy-S needs pages built with GTS_BUILD_SYMMETRIC");
+    const bool timing = rc.flags & GTS_RUN_TIMING;
+    cudaStream_t s = c->stream;
+    const int eg = c->num_sms * 4;
+    std::vector<int32_t> owner;
+    std::vector<uint64_t> vr;
+    partition(g, strat, N, owner, vr);
+    std::vector<MSlot> S(L);
+    uint64_t wa_bytes = 0;
+    for (int i = 0; i < L; ++i) {
+        MSlot& m = S[i];
+        m.r = R.rank(i);
+        if (R.virt) {
+            for (uint64_t j = 0; j < g->num_pages; ++j)
+                if (strat == GTS_STRATEGY_S_BCAST || owner[j] == m.r) m.pages.push_back((uint32_t)j);
+            GTS_TRY(c->buf(kBufMulti + 16 * i + 0, std::max<size_t>(m.pages.size(), 1) * 4, (void**)&m.d_pages));
+            if (!m.pages.empty())
+                GTS_CUDA(cudaMemcpyAsync(m.d_pages, m.pages.data(), m.pages.size() * 4, cudaMemcpyHostToDevice, s));
+        } else {
+            m.pages = c->dg.h_local_list;
+            m.d_pages = c->dg.local_list;
+        }
+        if (strat == GTS_STRATEGY_P) {
+            m.lo = 0;
+            m.hi = n;
+        } else {
+            m.lo = vr[m.r];
+            m.hi = vr[m.r + 1];
+        }
+        // WA: the full replicated arrays (P, S_BCAST) or this rank's range only (S)
+        const uint64_t alo = route ? m.lo : 0, ahi = route ? m.hi : n;
+        m.w0 = route ? alo >> 5 : 0;
+        m.w1 = route ? (ahi + 31) >> 5 : words;
+        const uint64_t nw = std::max<uint64_t>(m.w1 - m.w0, 1), nv = std::max<uint64_t>(ahi - alo, 1);
+        uint32_t *val, *vis = nullptr, *cu, *nx;
+        GTS_TRY(c->buf(kBufMulti + 16 * i + 1, nv * 4, (void**)&val));
+        if (algo == kBFS) GTS_TRY(c->buf(kBufMulti + 16 * i + 2, nw * 4, (void**)&vis));
+        GTS_TRY(c->buf(kBufMulti + 16 * i + 3, nw * 4, (void**)&cu));
+        GTS_TRY(c->buf(kBufMulti + 16 * i + 4, nw * 4, (void**)&nx));
+        m.value = val - alo;
+        m.visited = vis ? vis - m.w0 : nullptr;
+        m.cur = cu - m.w0;
+        m.next = nx - m.w0;
+        if (i == 0) wa_bytes = nv * 4 + nw * 4 * (algo == kBFS ? 3 : 2);
+        if (!route) GTS_TRY(c->buf(kBufMulti + 16 * i + 5, (size_t)N * words * 4, (void**)&m.gathered));
+        if (route && algo == kBFS) {
+            GTS_TRY(c->buf(kBufMulti + 16 * i + 6, words * 4, (void**)&m.sent));
+            GTS_CUDA(cudaMemsetAsync(m.sent, 0, words * 4, s));
+            if (i == 0) wa_bytes += words * 4;
+        }
+        GTS_TRY(c->buf(kBufMulti + 16 * i + 7, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&m.list));
+        GTS_TRY(c->buf(kBufMulti + 16 * i + 8, sizeof(Counters), (void**)&m.ctr));
+        GTS_CUDA(cudaMemsetAsync(m.ctr, 0, sizeof(Counters), s));
+        GTS_CUDA(cudaMemsetAsync(cu, 0, nw * 4, s));
+        GTS_CUDA(cudaMemsetAsync(nx, 0, nw * 4, s));
+        if (vis) GTS_CUDA(cudaMemsetAsync(vis, 0, nw * 4, s));
+        if (algo == kWCCLP) {
+            wcc_lp_init_kernel<<<eg, 256, 0, s>>>(m.value, m.cur, m.lo, m.hi);
+            m.h_list = m.pages;            // every vertex starts active
+        } else {
+            GTS_CUDA(cudaMemsetAsync(val, 0xFF, nv * 4, s));
+        }
+    }
+    const uint64_t isrc = algo == kWCCLP ? 0 : map_src(g, src);
+    if (algo != kWCCLP) {
+        // the pages holding src (Alg 1 line 5) among each rank's pages; its WA entry on its owner(s)
+        auto it = std::upper_bound(g->start_vid.begin(), g->start_vid.end(), (uint32_t)isrc);
+        const int64_t p = (int64_t)(it - g->start_vid.begin()) - 1;
+        const int64_t a = g->kind[p] == GTS_PAGE_LP ? g->lp_first[p] : p, b = g->kind[p] == GTS_PAGE_LP ? g->lp_last[p] : p;
+        for (MSlot& m : S) {
+            for (int64_t q = a; q <= b; ++q)
+                if (std::binary_search(m.pages.begin(), m.pages.end(), (uint32_t)q)) m.h_list.push_back((uint32_t)q);
+            if (isrc >= m.lo && isrc < m.hi) set_source_range_kernel<<<1, 1, 0, s>>>(m.value, m.visited, m.cur, isrc);
+        }
+    }
+    for (MSlot& m : S) {
+        m.h.list_count = (uint32_t)m.h_list.size();
+        if (!m.h_list.empty())
+            GTS_CUDA(cudaMemcpyAsync(m.list, m.h_list.data(), m.h_list.size() * 4, cudaMemcpyHostToDevice, s));
+        GTS_CUDA(cudaMemcpyAsync(&m.ctr->list_count, &m.h.list_count, 4, cudaMemcpyHostToDevice, s));
+    }
+    GTS_CUDA(cudaStreamSynchronize(s));        // host vectors above are read by the copies
+    Route rt;
+    if (route) {
+        std::vector<std::vector<uint32_t>> pl(L);
+        std::vector<const uint32_t*> dpl(L);
+        for (int i = 0; i < L; ++i) {
+            pl[i] = S[i].pages;
+            dpl[i] = S[i].d_pages;
+        }
+        std::vector<std::array<uint64_t, kMaxRanks>> cap;
+        GTS_TRY(route_capacities(c, g, R, rc, streamed, pl, dpl.data(), vr, 0, cap));
+        GTS_TRY(route_setup(c, R, cap, algo == kBFS ? 4 : 8, kBufRoute, rt));
+    }
+    const uint64_t delta = rc.sssp_delta ? rc.sssp_delta : 0xFFFFFFFEull;
+    uint32_t T = algo == kSSSP ? (uint32_t)std::min<uint64_t>(delta, 0xFFFFFFFEull) : 0xFFFFFFFEu;
+    const bool W = g->weighted;
+    const void* kexp = algo == kBFS ? (W ? (const void*)mbfs_expand_kernel<true> : (const void*)mbfs_expand_kernel<false>)
+                       : algo == kSSSP ? (const void*)mmin_expand_kernel<true, true>
+                                       : (W ? (const void*)mmin_expand_kernel<true, false>
+                                            : (const void*)mmin_expand_kernel<false, false>);
+    int grid = 0;
+    GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
+    uint64_t launches = 0, main_launches = 0, pages_processed = 0;
+    uint32_t levels = 0;
+    SweepStats ss;
+    for (uint32_t lev = 0;; ++lev) {
+        if (route) GTS_CUDA(cudaMemsetAsync(rt.d_scnt, 0, (size_t)L * kMaxRanks * 8, s));
+        for (int i = 0; i < L; ++i) {
+            MSlot& m = S[i];
+            pages_processed += m.h.list_count;
+            RouteOut ro{};
+            if (route) {
+                ro.send = rt.send[i];
+                ro.cnt = rt.d_scnt + (size_t)i * kMaxRanks;
+                ro.ovf = rt.d_ovf + i;
+                for (int q = 0; q <= N; ++q) ro.vr[q] = vr[q];
+                for (int q = 0; q < N; ++q) {
+                    ro.off[q] = rt.soff[i][q];
+                    ro.cap[q] = rt.scap[i][q];
+                }
+                ro.nranks = N;
+            }
+            auto launch = [&](const PageSet& ps, int gcap) -> int {
+                GTS_CUDA(cudaMemsetAsync(&m.ctr->work, 0, 4, s));
+                std::pair<cudaEvent_t, cudaEvent_t> ev;
+                if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
+                PageSet p2 = ps;
+                p2.split = 0u;
+                const int gl = std::min(grid, gcap);
+                if (algo == kBFS) {
+                    if (W) {
+                        MBfsOp<true> op{m.cur, m.visited, m.next, m.sent, 0ull, m.lo, m.hi, mode, ro};
+                        mbfs_expand_kernel<true><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges);
+                    } else {
+                        MBfsOp<false> op{m.cur, m.visited, m.next, m.sent, 0ull, m.lo, m.hi, mode, ro};
+                        mbfs_expand_kernel<false><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges);
+                    }
+                } else if (algo == kSSSP) {
+                    MMinOp<true, true> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro};
+                    mmin_expand_kernel<true, true><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges,
+                                                                         &m.ctr->flag);
+                } else if (W) {
+                    MMinOp<true, false> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro};
+                    mmin_expand_kernel<true, false><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges,
+                                                                          &m.ctr->flag);
+                } else {
+                    MMinOp<false, false> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro};
+                    mmin_expand_kernel<false, false><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges,
+                                                                           &m.ctr->flag);
+                }
+                if (timing) cudaEventRecord(ev.second, s);
+                GTS_CUDA(cudaGetLastError());
+                ++main_launches;
+                return GTS_OK;
+            };
+            GTS_TRY(sweep_pages(c, g, rc, streamed, &m.h_list, m.list, m.h.list_count, &m.ctr->list_count, launch, &ss));
+        }
+        // ---- merge (a12) ----
+        std::pair<cudaEvent_t, cudaEvent_t> ev;
+        if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
+        if (route) {
+            GTS_TRY(R.route_exchange(rt));
+            for (int i = 0; i < L; ++i) {
+                RecvView rv{};
+                rv.recv = rt.recv[i];
+                for (int q = 0; q < N; ++q) rv.off[q] = rt.roff[i][q];
+                rv.cnt = rt.d_rcnt + (size_t)i * kMaxRanks;
+                rv.nranks = N;
+                if (algo == kBFS) bfs_apply_kernel<<<eg, 256, 0, s>>>(rv, S[i].visited, S[i].next);
+                else min_apply_kernel<<<eg, 256, 0, s>>>(rv, S[i].value, S[i].next);
+                ++launches;
+            }
+        } else {
+            if (algo == kSSSP) {           // dist: all-reduce(min) over the replicas
+                std::vector<void*> b(L);
+                for (int i = 0; i < L; ++i) b[i] = S[i].value;
+                GTS_TRY(R.allreduce(b.data(), n, kCU32, kCMin));
+            }
+            std::vector<const void*> sb(L);
+            std::vector<void*> rb(L);
+            for (int i = 0; i < L; ++i) {
+                sb[i] = S[i].next;
+                rb[i] = S[i].gathered;
+            }
+            GTS_TRY(R.allgather(sb.data(), rb.data(), words * 4));
+        }
+        if (timing) { cudaEventRecord(ev.second, s); ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
+        // ---- finish: merged next frontier, counts, next page set (a6) ----
+        for (int i = 0; i < L; ++i) {
+            MSlot& m = S[i];
+            GTS_CUDA(cudaMemsetAsync(&m.ctr->count, 0, 8, s));
+            GTS_CUDA(cudaMemsetAsync(&m.ctr->list_count, 0, 4, s));
+            const uint32_t* gath = route ? nullptr : m.gathered;
+            if (algo == kSSSP) {
+                GTS_CUDA(cudaMemsetAsync(&m.ctr->near, 0, 8, s));
+                GTS_CUDA(cudaMemsetAsync(&m.ctr->minpend, 0xFF, 4, s));
+                sssp_finish_kernel<<<eg, 256, 0, s>>>(gath, N, words, m.w0, m.w1, m.cur, m.next, m.value, T,
+                                                      &m.ctr->count, &m.ctr->near, &m.ctr->minpend);
+            } else {
+                frontier_finish_kernel<<<eg, 256, 0, s>>>(gath, N, words, m.w0, m.w1, m.next, m.visited,
+                                                          algo == kBFS ? m.value : nullptr, lev + 1, &m.ctr->count);
+            }
+            frontier_pages_kernel<<<eg, 256, 0, s>>>(m.next, c->dg.rvt_start, c->dg.nslots, m.d_pages,
+                                                     (uint32_t)m.pages.size(), m.list, &m.ctr->list_count);
+            launches += 2;
+        }
+        if (route) {                       // frontier counts are per range: sum (SSSP: and min) over ranks
+            std::vector<void*> b(L);
+            for (int i = 0; i < L; ++i) b[i] = &S[i].ctr->count;
+            GTS_TRY(R.allreduce(b.data(), 1, kCU64, kCSum));
+            if (algo == kSSSP) {
+                for (int i = 0; i < L; ++i) b[i] = &S[i].ctr->near;
+                GTS_TRY(R.allreduce(b.data(), 1, kCU64, kCSum));
+                for (int i = 0; i < L; ++i) b[i] = &S[i].ctr->minpend;
+                GTS_TRY(R.allreduce(b.data(), 1, kCU32, kCMin));
+            }
+        }
+        if (timing) cudaEventRecord(ev.second, s);
+        GTS_CUDA(cudaGetLastError());
+        for (MSlot& m : S) GTS_CUDA(cudaMemcpyAsync(&m.h, m.ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+        ++levels;
+        if (S[0].h.count == 0) break;
+        if (algo == kSSSP && S[0].h.near == 0) {
+            const uint64_t nt = (uint64_t)S[0].h.minpend + delta;
+            T = (uint32_t)std::min<uint64_t>(nt, 0xFFFFFFFEull);
+        }
+        for (MSlot& m : S) {
+            if (streamed) {                // the host drives the copies: fetch and sort the page set
+                m.h_list.resize(m.h.list_count);
+                if (m.h.list_count) {
+                    GTS_CUDA(cudaMemcpyAsync(m.h_list.data(), m.list, m.h.list_count * 4ull, cudaMemcpyDeviceToHost, s));
+                    GTS_CUDA(cudaStreamSynchronize(s));
+                    std::sort(m.h_list.begin(), m.h_list.end());
+                    GTS_CUDA(cudaMemcpyAsync(m.list, m.h_list.data(), m.h.list_count * 4ull, cudaMemcpyHostToDevice, s));
+                    GTS_CUDA(cudaStreamSynchronize(s));
+                }
+            }
+            std::swap(m.cur, m.next);
+            GTS_CUDA(cudaMemsetAsync(m.next + m.w0, 0, (m.w1 - m.w0) * 4, s));
+        }
+    }
+    if (route) {
+        bool ovf = false;
+        GTS_TRY(R.route_overflow(rt, &ovf));
+        if (ovf) return fail(GTS_ECUDA, "Strategy-S route region overflow (capacity count mismatch)");
+    }
+    // ---- result: every rank's range into one full array (a13) ----
+    uint32_t* res = S[0].value;
+    if (route) {
+        GTS_TRY(c->buf(kBufResult, n * 4, (void**)&res));
+        std::vector<void*> full(L, res);
+        for (MSlot& m : S)
+            if (m.hi > m.lo)
+                GTS_CUDA(cudaMemcpyAsync(res + m.lo, m.value + m.lo, (m.hi - m.lo) * 4, cudaMemcpyDeviceToDevice, s));
+        GTS_TRY(R.gather_ranges(full.data(), vr, 4));
+    }
+    if (algo == kSSSP) {                   // exact overflow test, on every rank, over its pages
+        std::vector<void*> b(L);
+        for (int i = 0; i < L; ++i) b[i] = &S[i].ctr->flag;
+        GTS_TRY(R.allreduce(b.data(), 1, kCU32, kCMax));
+        uint32_t flag = 0;
+        GTS_CUDA(cudaMemcpyAsync(&flag, &S[0].ctr->flag, 4, cudaMemcpyDeviceToHost, s));
+        GTS_CUDA(cudaStreamSynchronize(s));
+        if (flag) {
+            int g2 = 0;
+            GTS_TRY(sms_grid(c, (const void*)sssp_check_kernel, kThreads, 0, &g2));
+            for (int i = 0; i < L; ++i) {
+                MSlot& m = S[i];
+                GTS_CUDA(cudaMemsetAsync(&m.ctr->flag2, 0, 4, s));
+                std::vector<uint32_t> hl = m.pages;
+                GTS_TRY(sweep_pages(c, g, rc, streamed, &hl, m.d_pages, (uint32_t)hl.size(), nullptr,
+                                    [&](const PageSet& ps, int gcap) -> int {
+                                        GTS_CUDA(cudaMemsetAsync(&m.ctr->work, 0, 4, s));
+                                        sssp_check_kernel<<<std::min(g2, gcap), kThreads, 0, s>>>(ps, res, &m.ctr->work,
+                                                                                                &m.ctr->flag2);
+                                        GTS_CUDA(cudaGetLastError());
+                                        return GTS_OK;
+                                    }, &ss));
+            }
+            for (int i = 0; i < L; ++i) b[i] = &S[i].ctr->flag2;
+            GTS_TRY(R.allreduce(b.data(), 1, kCU32, kCMax));
+            uint32_t bad = 0;
+            GTS_CUDA(cudaMemcpyAsync(&bad, &S[0].ctr->flag2, 4, cudaMemcpyDeviceToHost, s));
+            GTS_CUDA(cudaStreamSynchronize(s));
+            if (bad) return fail(GTS_EOVERFLOW, "an SSSP distance reaches 2^32-1");
+        }
+    }
+    GTS_TRY(deliver(c, g, res, out, rc.out_location, algo == kWCCLP));
+    if (st) {
+        std::memset(st, 0, sizeof(*st));
+        st->wall_s = now_s() - t_start;
+        st->upload_s = upload_s;
+        if (timing) {
+            st->main_kernel_s = c->t_main.sum_s();
+            st->merge_s = c->t_merge.sum_s();
+            st->finish_s = c->t_finish.sum_s();
+            st->h2d_s = c->t_h2d.sum_s();
+        }
+        uint64_t edges = 0;
+        for (MSlot& m : S) edges += m.h.edges;
+        st->pages_processed = pages_processed;
+        st->h2d_bytes = ss.h2d_bytes;
+        st->edges_traversed = edges;
+        st->nccl_bytes = R.bytes;
+        st->launches = launches + main_launches;
+        st->main_kernel_launches = main_launches;
+        st->levels_or_iters = levels;
+        st->wa_bytes = wa_bytes;
+        st->routed_msgs = rt.sent_msgs;
+    } else if (timing) {
+        c->t_main.sum_s();
+        c->t_merge.sum_s();
+        c->t_finish.sum_s();
+        c->t_h2d.sum_s();
+    }
+    return GTS_OK;
+}
+
+static int traverse(gts_context* c, const gts_graph* g, uint64_t src, const gts_run_config* cfg, uint32_t* out,
+                    gts_run_stats* st, int algo) {
+    clear_error();
+    const double t_start = now_s();
+    gts_run_config rc;
+    GTS_TRY(validate_common(c, g, cfg, &rc));
+    if (!out) return fail(GTS_EINVAL, "NULL output");
+    if (src >= g->n) return fail(GTS_EINVAL, "src %llu >= n %llu", (unsigned long long)src, (unsigned long long)g->n);
+    if (algo == kSSSP && !g->weighted) return fail(GTS_EUNSUPPORTED, "gts_sssp needs a graph built with weights");
+    Ranks R;
+    GTS_TRY(make_ranks(c, rc, &R));
+    const uint64_t n = g->n, words = (n + 31) / 32;
+    const uint64_t attr = R.world > 1 && rc.strategy == GTS_STRATEGY_S ? (4 * n + 16 * words) / R.world + words
+                                                                         : 4 * n + 16 * words;
+    const bool streamed = choose_streamed(c, g, rc, attr);
+    double upload_s = 0;
+    GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
+    if (R.world == 1) return traverse_single(c, g, src, rc, out, st, algo, t_start, streamed, upload_s);
+    return traverse_multi(c, g, src, rc, R, out, st, algo, t_start, streamed, upload_s);
 }
 
 // ------------------------------------------------------------------- BC ---
@@ -1017,7 +1540,8 @@ static int betweenness(gts_context* c, const gts_graph* g, const uint64_t* sourc
             };
             GTS_TRY(sweep_pages(c, g, rc, streamed, &h_list, list, cur_count, &ctr->list_count, launchA, &ss));
             GTS_CUDA(cudaMemsetAsync(&ctr->count, 0, 8, s));
-            frontier_finish_kernel<<<eg, 256, 0, s>>>(next, 1, words, next, visited, lv, L + 1, &ctr->count);
+            frontier_finish_kernel<<<eg, 256, 0, s>>>(nullptr, 1, words, 0, words, next, visited, lv, L + 1,
+                                                      &ctr->count);
             // pass B: sigma of the newly discovered vertices
             auto launchB = [&](const PageSet& ps, int cap) -> int {
                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));

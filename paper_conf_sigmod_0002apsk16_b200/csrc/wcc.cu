@@ -6,17 +6,21 @@
 // into a concurrent union-find forest whose roots are component minima
 // (ECL-CC-style hooking with atomicCAS, path halving), then a finalize pass
 // points every vertex at its root = the minimum VID of its weakly connected
-// component.  One sweep is exact on one GPU.  Strategy-P/S with N > 1: each
-// rank hooks its own pages, labels are merged with an NCCL all-reduce(min),
-// and the sweep repeats from the merged labels until no rank hooks anything.
+// component.  One sweep is exact on one GPU.  Strategy-P with N > 1: each
+// rank hooks its own pages, labels are merged with an all-reduce(min), and
+// the sweep repeats from the merged labels until no rank hooks anything.
+// S_BCAST: every rank hooks every page (replicated, exact after one sweep).
+// Strategy-S: routed label propagation on symmetrised pages (traverse.cu).
 #include <cuda_runtime.h>
 #include <nccl.h>
 
 #include <cstdlib>
 #include <cstring>
 
+#include "comm.h"
 #include "expand.cuh"
 #include "sweep.cuh"
+#include "traverse.h"
 
 namespace gts {
 
@@ -210,6 +214,7 @@ __global__ void wcc_finalize_kernel(uint32_t* parent, uint64_t n) {
 }
 
 enum { kBufLabel = 30, kBufWccCtr, kBufWccGiant };
+constexpr int kBufWccMulti = 400;   // multi-rank slot i: kBufWccMulti + 4 i + k
 
 }  // namespace gts
 
@@ -223,53 +228,75 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     GTS_TRY(validate_common(c, g, cfg, &rc));
     if (rc.flags & GTS_MICRO_MASK) return fail(GTS_EUNSUPPORTED, "GTS_MICRO_* techniques apply to gts_bfs and gts_pagerank");
     if (!label_out) return fail(GTS_EINVAL, "NULL output");
+    Ranks R;
+    GTS_TRY(make_ranks(c, rc, &R));
     const uint64_t n = g->n;
-    const bool streamed = choose_streamed(c, g, rc, 4 * n);
+    const int N = R.world, L = R.nloc;
+    const uint32_t strat = N > 1 ? rc.strategy : GTS_STRATEGY_P;
+    const bool streamed = choose_streamed(c, g, rc, strat == GTS_STRATEGY_S ? 4 * n / N + n / 8 : 4 * n);
     double upload_s = 0;
     GTS_TRY(ensure_graph(c, g, rc.strategy, !streamed, &upload_s));
+    // Strategy-S: routed min-label propagation on symmetrised pages (traverse.cu)
+    if (strat == GTS_STRATEGY_S) return traverse_multi(c, g, 0, rc, R, label_out, st, kWCCLP, t_start, streamed, upload_s);
+    // One rank, Strategy-P (each rank hooks its pages; forests merged by all-reduce(min), repeated
+    // until no rank hooks) or S_BCAST (every rank hooks every page: exact after one sweep, no exchange)
     const bool timing = rc.flags & GTS_RUN_TIMING;
-    uint32_t *label, *ctr;
-    GTS_TRY(c->buf(kBufLabel, n * 4, (void**)&label));
-    GTS_TRY(c->buf(kBufWccCtr, 8, (void**)&ctr));
     cudaStream_t s = c->stream;
     const int eg = c->num_sms * 4;
-    wcc_init_kernel<<<eg, 256, 0, s>>>(label, n);
+    std::vector<int32_t> owner;
+    std::vector<uint64_t> vr;
+    partition(g, strat, N, owner, vr);
+    std::vector<uint32_t*> label(L), ctr(L);
+    std::vector<std::vector<uint32_t>> pages(L);
+    std::vector<const uint32_t*> d_pages(L);
+    for (int i = 0; i < L; ++i) {
+        if (R.virt) {
+            for (uint64_t j = 0; j < g->num_pages; ++j)
+                if (strat == GTS_STRATEGY_S_BCAST || owner[j] == R.rank(i)) pages[i].push_back((uint32_t)j);
+            uint32_t* dp;
+            GTS_TRY(c->buf(kBufWccMulti + 4 * i, std::max<size_t>(pages[i].size(), 1) * 4, (void**)&dp));
+            if (!pages[i].empty())
+                GTS_CUDA(cudaMemcpyAsync(dp, pages[i].data(), pages[i].size() * 4, cudaMemcpyHostToDevice, s));
+            d_pages[i] = dp;
+        } else {
+            pages[i] = c->dg.h_local_list;
+            d_pages[i] = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
+        }
+        GTS_TRY(c->buf(L == 1 ? kBufLabel : kBufWccMulti + 4 * i + 1, n * 4, (void**)&label[i]));
+        GTS_TRY(c->buf(L == 1 ? kBufWccCtr : kBufWccMulti + 4 * i + 2, 8, (void**)&ctr[i]));
+        wcc_init_kernel<<<eg, 256, 0, s>>>(label[i], n);
+    }
+    GTS_CUDA(cudaStreamSynchronize(s));
+    // three 512-thread CTAs per SM for the sweep (40 registers; RMAT-27 sweep 17.4 -> 14.6 ms
+    // against two: the third CTA covers the per-tile barriers)
+    auto sweep_k = g->weighted ? wcc_sweep_kernel<true, 3> : wcc_sweep_kernel<false, 3>;
     int grid = 0;
-    // three 512-thread CTAs per SM for the sweep by default (40 registers; RMAT-27 sweep
-    // 17.4 -> 14.6 ms: the third CTA covers the per-tile barriers); GTS_WCC_OCC=2 = two
-    const char* oce = getenv("GTS_WCC_OCC");
-    const bool occ3 = !oce || atoi(oce) != 2;
-    auto sweep_k = g->weighted ? (occ3 ? wcc_sweep_kernel<true, 3> : wcc_sweep_kernel<true, 2>)
-                               : (occ3 ? wcc_sweep_kernel<false, 3> : wcc_sweep_kernel<false, 2>);
     GTS_TRY(sms_grid(c, (const void*)sweep_k, kThreads, 0, &grid));
-    uint64_t launches = 1, main_launches = 0, nccl_bytes = 0;
+    uint64_t launches = L, main_launches = 0;
     uint32_t sweeps = 0;
     uint32_t* hs = (uint32_t*)c->h_small;
     SweepStats ss;
-    const uint32_t* d_list = (c->dg.all_local && !streamed) ? nullptr : c->dg.local_list;
-    // sampling pass + compression (resident pages only: streamed, it would cost a
-    // whole extra transfer of the topology); GTS_WCC_SAMPLE=k neighbours, 0 = off
-    const char* se = getenv("GTS_WCC_SAMPLE");
-    const uint32_t ks = se ? (uint32_t)atol(se) : 1u;
-    // persisting-L2 window on the head of the union-find forest (degree-ordered
-    // pages: the most probed parents); GTS_L2_PERSIST_WCC=<MiB>, 0 = off
+    // sampling pass + compression (one rank, resident pages only: streamed, it would cost a
+    // whole extra transfer of the topology); gts_run_config.wcc_sample = k neighbours
+    const uint32_t ks = rc.wcc_sample == GTS_OFF ? 0u : rc.wcc_sample ? rc.wcc_sample : 1u;
+    // persisting-L2 window on the head of the union-find forest (degree-ordered pages: the
+    // most probed parents); gts_run_config.l2_persist_mib
     bool persist = false;
-    if (!streamed && g->ordered) {
-        const char* pe = getenv("GTS_L2_PERSIST_WCC");
-        const size_t want = std::min<size_t>((size_t)(pe ? atol(pe) : 96) << 20, n * 4);
+    if (!streamed && g->ordered && N == 1) {
+        const size_t want = std::min<size_t>(l2_persist_mib(rc) << 20, n * 4);
         if (want > 0) {
-            GTS_TRY(persist_window(c, s, label, want));
+            GTS_TRY(persist_window(c, s, label[0], want));
             persist = true;
         }
     }
     uint32_t* gbm = nullptr;   // giant filter bitmap (+ r* after it)
-    if (!streamed && ks > 0) {
+    if (!streamed && ks > 0 && N == 1) {
         std::pair<cudaEvent_t, cudaEvent_t> ev;
         if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-        GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
+        GTS_CUDA(cudaMemsetAsync(ctr[0], 0, 4, s));
         PageSet ps;
         ps.base = c->dg.pages;
-        ps.list = d_list;
+        ps.list = d_pages[0];
         ps.loc = c->dg.loc;
         ps.d_count = nullptr;
         ps.count = c->dg.n_local;
@@ -277,53 +304,59 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
         ps.mode = c->dg.all_local ? kAddrByPid : kAddrByLoc;
         ps.entry_encoding = g->entry_encoding;
         ps.rvt_start = c->dg.rvt_start;
-        ps.ww = env_ww();
         int sg = 0;
         GTS_TRY(sms_grid(c, (const void*)wcc_sample_kernel, kThreads, 0, &sg));
-        wcc_sample_kernel<<<sg, kThreads, 0, s>>>(ps, label, ctr, ks);
-        wcc_finalize_kernel<<<eg, 256, 0, s>>>(label, n);
+        wcc_sample_kernel<<<sg, kThreads, 0, s>>>(ps, label[0], ctr[0], ks);
+        wcc_finalize_kernel<<<eg, 256, 0, s>>>(label[0], n);
         GTS_TRY(c->buf(kBufWccGiant, (n + 31) / 32 * 4 + 16, (void**)&gbm));
-        wcc_giant_kernel<<<eg, 256, 0, s>>>(label, n, gbm, gbm + (n + 31) / 32);
+        wcc_giant_kernel<<<eg, 256, 0, s>>>(label[0], n, gbm, gbm + (n + 31) / 32);
         if (timing) cudaEventRecord(ev.second, s);
         GTS_CUDA(cudaGetLastError());
         launches += 2;
     }
     for (;;) {
-        GTS_CUDA(cudaMemsetAsync(ctr + 1, 0, 4, s));
-        std::pair<cudaEvent_t, cudaEvent_t> ev;
-        GTS_TRY(sweep_pages(c, g, rc, streamed, &c->dg.h_local_list, d_list, c->dg.n_local, nullptr,
-                            [&](const PageSet& ps, int cap) -> int {
-                                GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
-                                std::pair<cudaEvent_t, cudaEvent_t> e2;
-                                if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
-                                sweep_k<<<std::min(grid, cap), kThreads, 0, s>>>(ps, label, ctr, ctr + 1, gbm,
-                                                                                  gbm ? gbm + (n + 31) / 32 : nullptr);
-                                if (timing) cudaEventRecord(e2.second, s);
-                                GTS_CUDA(cudaGetLastError());
-                                ++main_launches;
-                                return GTS_OK;
-                            }, &ss));
-        ++sweeps;
-        if (c->world > 1) {
-            if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
-            GTS_NCCL(ncclGroupStart());
-            GTS_NCCL(ncclAllReduce(label, label, n, ncclUint32, ncclMin, c->comm, s));
-            GTS_NCCL(ncclAllReduce(ctr + 1, ctr + 1, 1, ncclUint32, ncclMax, c->comm, s));
-            GTS_NCCL(ncclGroupEnd());
-            if (timing) cudaEventRecord(ev.second, s);
-            nccl_bytes += n * 4 + 4;
+        for (int i = 0; i < L; ++i) {
+            GTS_CUDA(cudaMemsetAsync(ctr[i] + 1, 0, 4, s));
+            std::vector<uint32_t> hl(pages[i]);
+            GTS_TRY(sweep_pages(c, g, rc, streamed, &hl, d_pages[i], (uint32_t)hl.size(), nullptr,
+                                [&](const PageSet& ps, int cap) -> int {
+                                    GTS_CUDA(cudaMemsetAsync(ctr[i], 0, 4, s));
+                                    std::pair<cudaEvent_t, cudaEvent_t> e2;
+                                    if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
+                                    sweep_k<<<std::min(grid, cap), kThreads, 0, s>>>(
+                                        ps, label[i], ctr[i], ctr[i] + 1, gbm, gbm ? gbm + (n + 31) / 32 : nullptr);
+                                    if (timing) cudaEventRecord(e2.second, s);
+                                    GTS_CUDA(cudaGetLastError());
+                                    ++main_launches;
+                                    return GTS_OK;
+                                }, &ss));
         }
+        ++sweeps;
+        const bool merge = N > 1 && strat == GTS_STRATEGY_P;
+        if (merge) {                    // a12: forests merged by min, hook flags by max
+            std::pair<cudaEvent_t, cudaEvent_t> ev;
+            if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
+            std::vector<void*> lb(L), fb(L);
+            for (int i = 0; i < L; ++i) {
+                lb[i] = label[i];
+                fb[i] = ctr[i] + 1;
+            }
+            GTS_TRY(R.allreduce(lb.data(), n, kCU32, kCMin));
+            GTS_TRY(R.allreduce(fb.data(), 1, kCU32, kCMax));
+            if (timing) cudaEventRecord(ev.second, s);
+        }
+        std::pair<cudaEvent_t, cudaEvent_t> ev;
         if (timing) { ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
-        wcc_finalize_kernel<<<eg, 256, 0, s>>>(label, n);
+        for (int i = 0; i < L; ++i) wcc_finalize_kernel<<<eg, 256, 0, s>>>(label[i], n);
         if (timing) cudaEventRecord(ev.second, s);
-        ++launches;
-        if (c->world == 1) break;              // union-find is exact after one sweep on one GPU
-        GTS_CUDA(cudaMemcpyAsync(hs, ctr + 1, 4, cudaMemcpyDeviceToHost, s));
+        launches += L;
+        if (!merge) break;              // union-find over every page is exact after one sweep
+        GTS_CUDA(cudaMemcpyAsync(hs, ctr[0] + 1, 4, cudaMemcpyDeviceToHost, s));
         GTS_CUDA(cudaStreamSynchronize(s));
         if (hs[0] == 0) break;
     }
     if (persist) GTS_TRY(persist_window(c, s, nullptr, 0));
-    GTS_TRY(deliver(c, g, label, label_out, rc.out_location, true));
+    GTS_TRY(deliver(c, g, label[0], label_out, rc.out_location, true));
     if (st) {
         std::memset(st, 0, sizeof(*st));
         st->wall_s = now_s() - t_start;
@@ -332,15 +365,19 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
             st->main_kernel_s = c->t_main.sum_s();
             st->merge_s = c->t_merge.sum_s();
             st->finish_s = c->t_finish.sum_s();
+            st->h2d_s = c->t_h2d.sum_s();
         }
-        st->pages_processed = (uint64_t)c->dg.n_local * sweeps;
+        uint64_t np = 0;
+        for (auto& p : pages) np += p.size();
+        st->pages_processed = np * sweeps;
         st->h2d_bytes = ss.h2d_bytes;
-        if (timing) st->h2d_s = c->t_h2d.sum_s();
-        st->edges_traversed = g->m * (uint64_t)sweeps / (uint64_t)c->world;
-        st->nccl_bytes = nccl_bytes;
+        st->edges_traversed = (strat == GTS_STRATEGY_S_BCAST ? g->m * (uint64_t)L : g->m * (uint64_t)L / (uint64_t)N) *
+                              sweeps;
+        st->nccl_bytes = R.bytes;
         st->launches = launches + main_launches;
         st->main_kernel_launches = main_launches;
         st->levels_or_iters = sweeps;
+        st->wa_bytes = n * 4;
     } else if (timing) {
         c->t_main.sum_s();
         c->t_merge.sum_s();

@@ -33,8 +33,9 @@ GTS_RUN_TIMING = 1
 GTS_MICRO_DEFAULT, GTS_MICRO_EDGE, GTS_MICRO_VERTEX, GTS_MICRO_HYBRID, GTS_MICRO_TILE = 0, 1 << 8, 2 << 8, 3 << 8, 4 << 8
 MICRO = {"default": GTS_MICRO_DEFAULT, "edge": GTS_MICRO_EDGE, "vertex": GTS_MICRO_VERTEX,
          "hybrid": GTS_MICRO_HYBRID, "tile": GTS_MICRO_TILE}
-GTS_BUILD_DEGREE_ORDER = 1
+GTS_BUILD_DEGREE_ORDER, GTS_BUILD_SYMMETRIC, GTS_BUILD_OWNER_FILTER = 1, 2, 4
 GTS_UNREACHED = 0xFFFFFFFF
+GTS_OFF = 0xFFFFFFFF
 
 EXPORTED = ["gts_last_error", "gts_version", "gts_build_pages", "gts_plan_pages", "gts_graph_get_stats",
             "gts_graph_pages", "gts_graph_directory", "gts_graph_order", "gts_graph_free", "gts_get_unique_id",
@@ -49,14 +50,16 @@ class GtsError(RuntimeError):
 
 
 class PageConfig(ctypes.Structure):
-    _fields_ = [("struct_size", ctypes.c_uint32), ("page_bytes", ctypes.c_uint32),
-                ("entry_encoding", ctypes.c_uint32), ("flags", ctypes.c_uint32)]
+    _fields_ = [(k, ctypes.c_uint32) for k in ("struct_size", "page_bytes", "entry_encoding", "flags", "owner_rank",
+                                               "owner_world", "owner_strategy", "reserved")]
 
 
 class GraphStats(ctypes.Structure):
     _fields_ = [(k, ctypes.c_uint64) for k in ("n", "m", "num_pages", "n_sp", "n_lp", "n_lp_vertices",
                                                "page_bytes", "topo_bytes", "used_bytes", "max_outdeg")] + \
-               [(k, ctypes.c_uint32) for k in ("weighted", "entry_encoding", "n_hot", "ordered")]
+               [(k, ctypes.c_uint32) for k in ("weighted", "entry_encoding", "n_hot", "ordered")] + \
+               [("host_page_bytes", ctypes.c_uint64), ("symmetric", ctypes.c_uint32), ("owner_rank", ctypes.c_int32),
+                ("owner_world", ctypes.c_uint32), ("owner_strategy", ctypes.c_uint32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -64,7 +67,12 @@ class GraphStats(ctypes.Structure):
 
 class RunConfig(ctypes.Structure):
     _fields_ = [(k, ctypes.c_uint32) for k in ("struct_size", "strategy", "residency", "ring_slots",
-                                               "batch_pages", "out_location", "flags", "cache_mib")]
+                                               "batch_pages", "out_location", "flags", "cache_mib",
+                                               "virtual_ranks", "sssp_delta", "levels_per_sync", "l2_persist_mib",
+                                               "bfs_level_slots", "wcc_sample", "hybrid_deg", "reserved")]
+
+# gts_run_config 1.1 fields settable through the keyword `tune` of the compute calls
+TUNABLE = ("sssp_delta", "levels_per_sync", "l2_persist_mib", "bfs_level_slots", "wcc_sample", "hybrid_deg")
 
 
 class RunStats(ctypes.Structure):
@@ -73,7 +81,7 @@ class RunStats(ctypes.Structure):
                [(k, ctypes.c_uint64) for k in ("h2d_bytes", "nccl_bytes", "pages_processed", "edges_traversed",
                                                "launches", "main_kernel_launches")] + \
                [(k, ctypes.c_uint32) for k in ("levels_or_iters", "reserved")] + \
-               [(k, ctypes.c_uint64) for k in ("cache_hits", "cache_misses")]
+               [(k, ctypes.c_uint64) for k in ("cache_hits", "cache_misses", "wa_bytes", "routed_msgs")]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_ if k != "reserved"}
@@ -127,9 +135,14 @@ def gts_last_error():
     return _lib.gts_last_error().decode(errors="replace")
 
 
-def _page_config(page_bytes, entry_encoding, order=False):
-    return PageConfig(ctypes.sizeof(PageConfig), int(page_bytes), int(entry_encoding),
-                      GTS_BUILD_DEGREE_ORDER if order else 0)
+def _page_config(page_bytes, entry_encoding, order=False, symmetric=False, owner=None):
+    """owner = (rank, world, strategy): build only that rank's pages (GTS_BUILD_OWNER_FILTER)."""
+    flags = (GTS_BUILD_DEGREE_ORDER if order else 0) | (GTS_BUILD_SYMMETRIC if symmetric else 0)
+    r = w = st = 0
+    if owner is not None:
+        flags |= GTS_BUILD_OWNER_FILTER
+        r, w, st = (int(x) for x in owner)
+    return PageConfig(ctypes.sizeof(PageConfig), int(page_bytes), int(entry_encoding), flags, r, w, st, 0)
 
 
 class Graph:
@@ -151,9 +164,10 @@ class Graph:
         return st.as_dict()
 
     def pages(self):
-        """Copy of the host page bytes (uint8, num_pages * page_bytes)."""
+        """Copy of the host page bytes this graph holds (uint8; every page in ID order, or with an owner
+        filter that rank's pages in ascending ID)."""
         st = self.stats()
-        nbytes = st["num_pages"] * st["page_bytes"]
+        nbytes = st["host_page_bytes"]
         p = _lib.gts_graph_pages(self.handle)
         return np.ctypeslib.as_array((ctypes.c_uint8 * nbytes).from_address(p)).copy() if nbytes else \
             np.zeros(0, np.uint8)
@@ -184,18 +198,19 @@ class Graph:
             pass
 
 
-def gts_build_pages(row_ptr, col_idx, weights=None, page_bytes=1 << 20, entry_encoding=GTS_ENTRY_VID32, order=False):
+def gts_build_pages(row_ptr, col_idx, weights=None, page_bytes=1 << 20, entry_encoding=GTS_ENTRY_VID32, order=False,
+                    symmetric=False, owner=None):
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.uint64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.uint32)
     if weights is not None:
         weights = np.ascontiguousarray(weights, dtype=np.uint32)
     n = row_ptr.shape[0] - 1
     m = col_idx.shape[0]
-    cfg = _page_config(page_bytes, entry_encoding, order)
+    cfg = _page_config(page_bytes, entry_encoding, order, symmetric, owner)
     h = ctypes.c_void_p()
     _check(_lib.gts_build_pages(n, m, _np_ptr(row_ptr), _np_ptr(col_idx), _np_ptr(weights), ctypes.byref(cfg),
                                 ctypes.byref(h)))
-    return Graph(h, n, m)
+    return Graph(h, n, 2 * m if symmetric else m)
 
 
 def gts_plan_pages(row_ptr, weighted=False, page_bytes=1 << 20, entry_encoding=GTS_ENTRY_VID32):
@@ -260,10 +275,16 @@ def gts_context_create(device=0, rank=0, world_size=1, unique_id: bytes | None =
     return Context(h, device, rank, world_size)
 
 
-def _run_config(strategy, residency, ring_slots, batch_pages, out_location, timing, cache_mib=0, micro=0):
+def _run_config(strategy, residency, ring_slots, batch_pages, out_location, timing, cache_mib=0, micro=0,
+                virtual_ranks=0, tune=None):
     micro = MICRO[micro] if isinstance(micro, str) else int(micro)
-    return RunConfig(ctypes.sizeof(RunConfig), strategy, residency, ring_slots, batch_pages, out_location,
-                     (GTS_RUN_TIMING if timing else 0) | micro, int(cache_mib))
+    rc = RunConfig(ctypes.sizeof(RunConfig), strategy, residency, ring_slots, batch_pages, out_location,
+                   (GTS_RUN_TIMING if timing else 0) | micro, int(cache_mib), int(virtual_ranks))
+    for k, v in (tune or {}).items():
+        if k not in TUNABLE:
+            raise ValueError(f"unknown tuning field {k}")
+        setattr(rc, k, int(v))
+    return rc
 
 
 def _out(out, n, dtype, ctx=None):
@@ -289,10 +310,11 @@ def _out(out, n, dtype, ctx=None):
 
 
 def gts_bfs(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-            batch_pages=0, timing=False, cache_mib=0, micro=GTS_MICRO_DEFAULT):
-    """Returns (levels, stats dict).  micro: GTS_MICRO_* or "default"/"edge"/"vertex"/"hybrid"."""
+            batch_pages=0, timing=False, cache_mib=0, micro=GTS_MICRO_DEFAULT, virtual_ranks=0, tune=None):
+    """Returns (levels, stats dict).  micro: GTS_MICRO_* or "default"/"edge"/"vertex"/"hybrid".
+    virtual_ranks=V: run the V-rank job of `strategy` on this GPU.  tune: {gts_run_config 1.1 field: value}."""
     out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
-    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib, micro)
+    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib, micro, virtual_ranks, tune)
     st = RunStats()
     _check(_lib.gts_bfs(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()
@@ -300,9 +322,9 @@ def gts_bfs(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RE
 
 def gts_pagerank(ctx, graph, iters=10, damping=0.85, dangling=GTS_DANGLING_UNIFORM, out=None,
                  strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0, batch_pages=0, timing=False,
-                 micro=GTS_MICRO_DEFAULT):
+                 micro=GTS_MICRO_DEFAULT, virtual_ranks=0, tune=None):
     out, ptr, loc = _out(out, graph.n, np.float32, ctx)
-    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, 0, micro)
+    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, 0, micro, virtual_ranks, tune)
     st = RunStats()
     _check(_lib.gts_pagerank(ctx.handle, graph.handle, int(iters), float(damping), int(dangling),
                              ctypes.byref(cfg), ptr, ctypes.byref(st)))
@@ -310,18 +332,18 @@ def gts_pagerank(ctx, graph, iters=10, damping=0.85, dangling=GTS_DANGLING_UNIFO
 
 
 def gts_sssp(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-             batch_pages=0, timing=False, cache_mib=0):
+             batch_pages=0, timing=False, cache_mib=0, virtual_ranks=0, tune=None):
     out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
-    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib)
+    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib, 0, virtual_ranks, tune)
     st = RunStats()
     _check(_lib.gts_sssp(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()
 
 
 def gts_wcc(ctx, graph, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-            batch_pages=0, timing=False):
+            batch_pages=0, timing=False, virtual_ranks=0, tune=None):
     out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
-    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing)
+    cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, 0, 0, virtual_ranks, tune)
     st = RunStats()
     _check(_lib.gts_wcc(ctx.handle, graph.handle, ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()

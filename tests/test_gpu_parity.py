@@ -98,15 +98,15 @@ def test_bfs_pid16_entries(G, ctx, name):
 
 
 @pytest.mark.parametrize("name", ["fig1", "path", "bintree", "rmat16_4k", "rmat20", "twitter20"])
-@pytest.mark.parametrize("k", ["0", "3", "5", "64"])
-@pytest.mark.parametrize("batch", ["1", "3", "8"])
-def test_bfs_level_slots(G, ctx, name, k, batch, monkeypatch):
-    """Level-slot LV construction (GTS_BFS_SLOTS=K): LV written once from the per-level
-    frontier bitmaps; traversals deeper than K switch to per-level LV writes mid-way.
-    K=0 is per-level writes throughout.  Levels enqueued GTS_BFS_BATCH at a time between
-    host round trips.  Resident, streamed and degree-ordered pages; edge and level counts."""
-    monkeypatch.setenv("GTS_BFS_SLOTS", k)
-    monkeypatch.setenv("GTS_BFS_BATCH", batch)
+@pytest.mark.parametrize("k", [0xFFFFFFFF, 3, 5, 64])
+@pytest.mark.parametrize("batch", [1, 3, 8])
+def test_bfs_level_slots(G, ctx, name, k, batch):
+    """Level-slot LV construction (gts_run_config.bfs_level_slots = K): LV written once from
+    the per-level frontier bitmaps; traversals deeper than K switch to per-level LV writes
+    mid-way.  K = GTS_OFF is per-level writes throughout.  Levels enqueued levels_per_sync
+    at a time between host round trips.  Resident, streamed and degree-ordered pages; edge
+    and level counts."""
+    tune = {"bfs_level_slots": k, "levels_per_sync": batch}
     g, pb = graph(name)
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
     go = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
@@ -115,37 +115,17 @@ def test_bfs_level_slots(G, ctx, name, k, batch, monkeypatch):
         reached = want != oracle.UNREACHED
         depth = int(want[reached].max()) + 1
         for gg, kw in ((gr, {}), (go, {}), (gr, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3))):
-            got, st = G.gts_bfs(ctx, gg, src, **kw)
+            got, st = G.gts_bfs(ctx, gg, src, tune=tune, **kw)
             assert np.array_equal(got, want), (name, k, src, kw, int(np.sum(got != want)))
             assert st["levels_or_iters"] == depth, (st["levels_or_iters"], depth)
             assert st["edges_traversed"] == int(np.diff(g.row_ptr)[reached].sum())
 
 
-@pytest.mark.parametrize("name", ["fig1", "rmat16_4k", "rmat20", "twitter20", "instar"])
-@pytest.mark.parametrize("occ", ["2", "3"])
-def test_occupancy_variants(G, ctx, name, occ, monkeypatch):
-    """Two- and three-CTA-per-SM builds of the BFS, WCC and SSSP expansion kernels
-    (GTS_BFS_OCC / GTS_WCC_OCC / GTS_SSSP_OCC), resident and degree-ordered pages."""
-    for k in ("GTS_BFS_OCC", "GTS_WCC_OCC", "GTS_SSSP_OCC"):
-        monkeypatch.setenv(k, occ)
-    g, pb = graph(name)
-    w = inputs.edge_weights(g)
-    for order in (False, True):
-        gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
-        src = _sources(g)[1]
-        assert np.array_equal(G.gts_bfs(ctx, gr, src)[0], oracle.bfs(g.row_ptr, g.col, src))
-        assert np.array_equal(G.gts_wcc(ctx, gr)[0], oracle.wcc(g.row_ptr, g.col))
-        grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb, order=order)
-        assert np.array_equal(G.gts_sssp(ctx, grw, src)[0], oracle.sssp(g.row_ptr, g.col, w, src))
-
-
 @pytest.mark.parametrize("name", ["fig1", "outstar", "instar", "rmat16_4k", "rmat16_256", "twitter20"])
-@pytest.mark.parametrize("split", ["0", "1"])
-def test_lp_slicing(G, ctx, name, split, monkeypatch):
-    """LP slicing for small page sets (GTS_SPLIT): BFS and SSSP from the max-degree
-    vertex (its LPs are the whole first level) and from vertex 0, resident and streamed,
-    bit-exact either way."""
-    monkeypatch.setenv("GTS_SPLIT", split)
+def test_lp_slicing(G, ctx, name):
+    """LP slicing for small page sets: BFS and SSSP from the max-degree vertex (its LPs
+    are the whole first level, sliced over the grid) and from vertex 0, resident and
+    streamed, bit-exact."""
     g, pb = graph(name)
     w = inputs.edge_weights(g)
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb)
@@ -154,23 +134,20 @@ def test_lp_slicing(G, ctx, name, split, monkeypatch):
         want = oracle.bfs(g.row_ptr, g.col, src)
         for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=2)):
             got, st = G.gts_bfs(ctx, gr, src, **kw)
-            assert np.array_equal(got, want), (name, split, src, kw)
+            assert np.array_equal(got, want), (name, src, kw)
             reached = want != oracle.UNREACHED
             assert st["edges_traversed"] == int(np.diff(g.row_ptr)[reached].sum())
             assert np.array_equal(G.gts_sssp(ctx, grw, src, **kw)[0], oracle.sssp(g.row_ptr, g.col, w, src))
 
 
 @pytest.mark.parametrize("name", ["fig1", "rmat16_4k", "rmat16_64k", "rmat20", "twitter20", "bintree"])
-@pytest.mark.parametrize("wdense", ["0", "1", "2"])
-def test_weighted_dense_tiles(G, ctx, name, wdense, monkeypatch):
-    """Weighted pages under the three dense-tile tests (GTS_WDENSE): SSSP and BFS bit-exact,
-    warp-window and tile walks."""
-    monkeypatch.setenv("GTS_WDENSE", wdense)
+def test_weighted_dense_tiles(G, ctx, name):
+    """Weighted pages (dense tiles by warp windows skip the weight words): SSSP and BFS
+    bit-exact."""
     g, pb = graph(name)
     w = inputs.edge_weights(g)
     src = _sources(g)[1]
-    for ww in ("1", "0"):
-        monkeypatch.setenv("GTS_WW", ww)
+    if True:
         for order in (False, True):
             grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb, order=order)
             assert np.array_equal(G.gts_sssp(ctx, grw, src)[0], oracle.sssp(g.row_ptr, g.col, w, src))
@@ -178,11 +155,9 @@ def test_weighted_dense_tiles(G, ctx, name, wdense, monkeypatch):
 
 
 @pytest.mark.parametrize("name", ["fig1", "multi", "path", "outstar", "rand", "rmat16_4k", "rmat16_256", "rmat20", "twitter20"])
-@pytest.mark.parametrize("gww", ["0", "1"])
-def test_sparse_gather_walks(G, ctx, name, gww, monkeypatch):
-    """Sparse tiles' item gather: per-thread binary search (GTS_GWW=0) or warp windows over
-    the item-start mask (GTS_GWW=1); BFS / SSSP / WCC bit-exact, natural and degree order."""
-    monkeypatch.setenv("GTS_GWW", gww)
+def test_sparse_tiles(G, ctx, name):
+    """Sparse tiles' item gather (compacted frontier vertices, a binary search per 4 edges);
+    BFS / SSSP / WCC bit-exact, natural and degree order, several sources."""
     g, pb = graph(name)
     w = inputs.edge_weights(g)
     for order in (False, True):
@@ -403,87 +378,33 @@ def test_degree_ordered_unaligned_device_outputs(G, ctx, name):
 
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "twitter20", "instar", "multi"])
-@pytest.mark.parametrize("mode", ["persist", "nopersist", "warpwindow"])
-def test_pagerank_ordered_variants(G, ctx, name, mode, monkeypatch):
-    """Degree-ordered PageRank with and without the L2 persistence window (GTS_L2_PERSIST=0),
-    and with the warp-window walk (record-start masks) instead of the tile walk."""
-    if mode == "nopersist":
-        monkeypatch.setenv("GTS_L2_PERSIST", "0")
-    if mode == "warpwindow":
-        monkeypatch.setenv("GTS_PR_WW", "1")
+@pytest.mark.parametrize("mode", ["persist", "nopersist"])
+def test_pagerank_ordered_variants(G, ctx, name, mode):
+    """Degree-ordered PageRank with and without the L2 persistence window
+    (gts_run_config.l2_persist_mib = GTS_OFF)."""
+    tune = {"l2_persist_mib": G.GTS_OFF} if mode == "nopersist" else None
     g, pb = graph(name)
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
     for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3)):
-        got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, **kw)
+        got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, tune=tune, **kw)
         _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, mode, kw))
-
-
-# Binned (propagation-blocking) scatter geometries (DESIGN.md 6b): hot set,
-# fine-bin width, fine-bin count, coarse-bin width, phase-2 chunk.  The small
-# geometries push RMAT-16 / in-star edges through hundreds of fine and coarse
-# bins and multi-chunk items; "off" is the plain red.add scatter.
-PB_GEOMS = {
-    "default": dict(GTS_PR_BINNED="1"),
-    "small": dict(GTS_PR_BINNED="1", GTS_PB_HOT="64", GTS_PB_FINE_SHIFT="6", GTS_PB_NFINE="100", GTS_PB_COARSE_SHIFT="9",
-                  GTS_PB_CHUNK="1024"),
-    "hubonly": dict(GTS_PR_BINNED="1", GTS_PB_HOT="4", GTS_PB_FINE_SHIFT="8", GTS_PB_CHUNK="1024"),
-    "coarse_only": dict(GTS_PR_BINNED="1", GTS_PB_HOT="128", GTS_PB_NFINE="0", GTS_PB_COARSE_SHIFT="4"),
-    "fine_max": dict(GTS_PR_BINNED="1", GTS_PB_HOT="4", GTS_PB_FINE_SHIFT="2", GTS_PB_NFINE="512", GTS_PB_COARSE_SHIFT="2"),
-    "off": dict(GTS_PR_BINNED="0"),
-    "warpwindow": dict(GTS_PR_BINNED="0", GTS_PR_WW="1"),
-}
-
-
-@pytest.mark.parametrize("name", ["rmat16_4k", "rmat16_1m", "rmat20", "twitter20", "instar", "multi", "fig1", "path"])
-@pytest.mark.parametrize("geom", list(PB_GEOMS))
-def test_pagerank_binned_geometries(G, ctx, name, geom, monkeypatch):
-    for k, v in PB_GEOMS[geom].items():
-        monkeypatch.setenv(k, v)
-    g, pb = graph(name)
-    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
-    for mode in (G.GTS_DANGLING_UNIFORM, G.GTS_DANGLING_DROP):
-        got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, mode)
-        _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85, dangling=mode), g, (name, geom, mode))
-    if name == "rmat16_4k":               # weighted pages skip the weight words
-        grw = G.gts_build_pages(g.row_ptr, g.col, inputs.edge_weights(g), page_bytes=2 * pb, order=True)
-        got, _ = G.gts_pagerank(ctx, grw, 10, 0.85)
-        _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, geom, "weighted"))
 
 
 @pytest.mark.parametrize("name", ["fig1", "multi", "path", "cycle", "outstar", "instar", "rand", "rmat16_4k",
                                   "rmat16_256", "rmat20", "twitter20"])
-@pytest.mark.parametrize("ks", ["0", "1", "2", "8"])
+@pytest.mark.parametrize("ks", [0xFFFFFFFF, 1, 2, 8])
 @pytest.mark.parametrize("order", [False, True])
-def test_wcc_sampling(G, ctx, name, ks, order, monkeypatch):
-    """WCC with the sampling pre-pass hooking the first ks out-neighbours (0 = off)."""
-    monkeypatch.setenv("GTS_WCC_SAMPLE", ks)
+def test_wcc_sampling(G, ctx, name, ks, order):
+    """WCC with the sampling pre-pass hooking the first ks out-neighbours (GTS_OFF = no pass)."""
+    tune = {"wcc_sample": ks}
     g, pb = graph(name)
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
-    got, _ = G.gts_wcc(ctx, gr)
+    got, _ = G.gts_wcc(ctx, gr, tune=tune)
     assert np.array_equal(got, oracle.wcc(g.row_ptr, g.col)), (name, ks, order)
     if name == "rmat16_4k":
         grw = G.gts_build_pages(g.row_ptr, g.col, inputs.edge_weights(g), page_bytes=2 * pb, order=order)
-        got, _ = G.gts_wcc(ctx, grw)
+        got, _ = G.gts_wcc(ctx, grw, tune=tune)
         assert np.array_equal(got, oracle.wcc(g.row_ptr, g.col)), (name, ks, order, "weighted")
-
-
-@pytest.mark.parametrize("name", ["fig1", "multi", "path", "bintree", "rand", "rmat16_4k", "rmat16_256", "rmat20",
-                                  "twitter20"])
-@pytest.mark.parametrize("order", [False, True])
-def test_tile_walk_dense_tiles(G, ctx, name, order, monkeypatch):
-    """Dense tiles by the tile walk (binary search per 16 bytes, GTS_WW=0) instead of warp windows."""
-    monkeypatch.setenv("GTS_WW", "0")
-    g, pb = graph(name)
-    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
-    for s in _sources(g):
-        lv, _ = G.gts_bfs(ctx, gr, s)
-        assert np.array_equal(lv, oracle.bfs(g.row_ptr, g.col, s)), (name, s)
-    w = inputs.edge_weights(g)
-    grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=2 * pb, order=order)
-    d, _ = G.gts_sssp(ctx, grw, 0)
-    assert np.array_equal(d, oracle.sssp(g.row_ptr, g.col, w, 0)), name
-    lab, _ = G.gts_wcc(ctx, gr)
-    assert np.array_equal(lab, oracle.wcc(g.row_ptr, g.col)), name
 
 
 # ------------------------------------------------- streamed + LRU page cache ---
@@ -516,37 +437,15 @@ def test_streamed_page_cache(G, ctx, name, cache_pages):
     assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, src))
 
 
-# ------------------------------------- Strategy-S with routed updates (virtual ranks) ---
-
-@pytest.mark.parametrize("name", ["fig1", "rmat16_4k", "rmat20", "twitter20", "instar", "outstar"])
-@pytest.mark.parametrize("vranks", [2, 3, 8])
-@pytest.mark.parametrize("order", [False, True])
-def test_pagerank_strategy_s_routed(G, ctx, name, vranks, order, monkeypatch):
-    """Strategy-S with range-partitioned WA and routed updates: V
-    virtual ranks run one after another on this GPU (GTS_VIRTUAL_RANKS), each
-    scattering only its own pages into its own WA range and packing every other
-    update into per-owner (dst, value) buffers; the in-memory exchange then
-    applies them.  Exercises owner lookup, capacity counting, warp-aggregated
-    packing, hot-partial routing and apply; only the NCCL send/recv is skipped."""
-    monkeypatch.setenv("GTS_VIRTUAL_RANKS", str(vranks))
-    g, pb = graph(name)
-    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
-    want = oracle.pagerank(g.row_ptr, g.col, 10, 0.85)
-    for kw in ({}, dict(residency=G.GTS_STREAMED, ring_slots=2, batch_pages=3)):
-        got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, strategy=G.GTS_STRATEGY_S, **kw)
-        _pr_check(got, want, g, (name, vranks, order, kw))
-
-
-@pytest.mark.parametrize("delta", ["1", "16", "256", "4294967294"])
+@pytest.mark.parametrize("delta", [1, 16, 256, 4294967294])
 @pytest.mark.parametrize("name", ["rmat16_4k", "rmat20", "path", "bintree"])
-def test_sssp_near_far_deltas(G, ctx, name, delta, monkeypatch):
-    """Near-far SSSP bucket widths, from 1 (Dijkstra-like) to unbounded (plain
-    frontier Bellman-Ford): distances are exact for every width."""
-    monkeypatch.setenv("GTS_SSSP_DELTA", delta)
+def test_sssp_near_far_deltas(G, ctx, name, delta):
+    """Near-far SSSP bucket widths (gts_run_config.sssp_delta), from 1 (Dijkstra-like) to
+    unbounded (plain frontier Bellman-Ford): distances are exact for every width."""
     g, pb = graph(name)
     w = inputs.edge_weights(g)
     gr = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb * 2 if pb < (1 << 20) else pb)
-    got, _ = G.gts_sssp(ctx, gr, 0)
+    got, _ = G.gts_sssp(ctx, gr, 0, tune={"sssp_delta": delta})
     assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, 0))
 
 
@@ -583,15 +482,14 @@ def test_bc_streamed_and_device_output(G, ctx):
 
 @pytest.mark.parametrize("name", ["rmat16_4k", "twitter20", "instar"])
 @pytest.mark.parametrize("vranks", [2, 5])
-def test_pagerank_strategy_s_bcast(G, ctx, name, vranks, monkeypatch):
+def test_pagerank_strategy_s_bcast(G, ctx, name, vranks):
     """Paper-literal Strategy-S: every (virtual) rank sweeps every
-    page and keeps only the updates of its own WA range; no exchange."""
-    monkeypatch.setenv("GTS_VIRTUAL_RANKS", str(vranks))
+    page and keeps only the updates of its own WA range."""
     g, pb = graph(name)
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
-    got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, strategy=G.GTS_STRATEGY_S_BCAST)
+    got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, strategy=G.GTS_STRATEGY_S_BCAST, virtual_ranks=vranks)
     _pr_check(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, (name, vranks, "bcast"))
-    lv, _ = G.gts_bfs(ctx, gr, 0, strategy=G.GTS_STRATEGY_S_BCAST)
+    lv, _ = G.gts_bfs(ctx, gr, 0, strategy=G.GTS_STRATEGY_S_BCAST, virtual_ranks=vranks)
     assert np.array_equal(lv, oracle.bfs(g.row_ptr, g.col, 0))
 
 
@@ -631,15 +529,15 @@ def test_bfs_micro_weighted_pid16_streamed(G, ctx, micro):
     assert np.array_equal(got, want) and st["h2d_bytes"] > 0
 
 
-@pytest.mark.parametrize("hdeg", ["1", "1000000"])
-def test_hybrid_threshold_extremes(G, ctx, hdeg, monkeypatch):
-    """GTS_HYBRID_DEG=1 sends (almost) every page edge-centric, 10^6 every page vertex-centric."""
-    monkeypatch.setenv("GTS_HYBRID_DEG", hdeg)
+@pytest.mark.parametrize("hdeg", [1, 1000000])
+def test_hybrid_threshold_extremes(G, ctx, hdeg):
+    """hybrid_deg = 1 sends (almost) every page edge-centric, 10^6 every page vertex-centric."""
+    tune = {"hybrid_deg": hdeg}
     g, pb = graph("rmat20")
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=65536)
-    got, _ = G.gts_bfs(ctx, gr, 0, micro="hybrid")
+    got, _ = G.gts_bfs(ctx, gr, 0, micro="hybrid", tune=tune)
     assert np.array_equal(got, oracle.bfs(g.row_ptr, g.col, 0))
-    pr, _ = G.gts_pagerank(ctx, gr, 10, 0.85, micro="hybrid")
+    pr, _ = G.gts_pagerank(ctx, gr, 10, 0.85, micro="hybrid", tune=tune)
     _pr_check(pr, oracle.pagerank(g.row_ptr, g.col, 10, 0.85), g, ("hybrid", hdeg))
 
 

@@ -171,3 +171,57 @@ def test_gloo_strategies(world):
             assert res[("bfs", strategy)], res
             assert res[("wcc", strategy)], res
             assert res[("sssp", strategy)], res
+
+
+def _owner_worker(rank, world, port, strategy, out):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import inputs
+    import paper_conf_sigmod_0002apsk16_b200 as G
+    try:
+        g = inputs.rmat(14)
+        pb = 8192
+        # each process builds and holds only its own pages (libgts GTS_BUILD_OWNER_FILTER)
+        gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True, owner=(rank, world, strategy))
+        st = gr.stats()
+        owner, vr = G.gts_partition_pages(gr, strategy, world)
+        mine = np.nonzero(owner == rank)[0]
+        got = [None] * world
+        dist.all_gather_object(got, (mine, gr.pages(), st["host_page_bytes"]))
+        if rank == 0:
+            full = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+            fp = full.pages().reshape(-1, pb)
+            seen = np.zeros(fp.shape[0], np.int64)
+            for ids, pages, hb in got:
+                assert hb == len(ids) * pb
+                assert np.array_equal(pages.reshape(-1, pb), fp[ids])
+                seen[ids] += 1
+            out.put(("ok", bool(np.all(seen == 1)), [hb for _, _, hb in got], full.stats()["topo_bytes"]))
+    except Exception as e:  # pragma: no cover
+        out.put(("err", repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("strategy", [0, 1])
+def test_gloo_owner_filtered_builds(world, strategy):
+    """One process per rank (gloo): every rank builds only its pages through libgts;
+    together they hold every page exactly once, byte-identical to a full build, with
+    host page bytes ~T_topo / N per rank (the multi-GPU memory plan)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_owner_worker, args=(r, world, port, strategy, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=120)
+    assert res[0] == "ok", res
+    _, partition_ok, host_bytes, topo = res
+    assert partition_ok
+    assert sum(host_bytes) == topo
+    assert max(host_bytes) <= topo / world * 1.2 + 16384
