@@ -22,6 +22,7 @@
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <algorithm>
 #include <cstdlib>
 #include <cstring>
 
@@ -199,24 +200,35 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             }
         } else {
             const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
-            for (uint32_t t0 = 0; t0 < nslots; t0 += T) {
+            // Software pipeline over the page's tiles: the slot offsets and x values of
+            // tile t+1 are loaded into registers while tile t's records stream, so a tile
+            // exposes one DRAM latency (its records) instead of three in a row (offsets,
+            // then x, then records) -- on low-degree pages a tile's records are only a few
+            // KB, so these latencies, not bytes, set the walk's time.
+            uint32_t r_off = 0, r_nxt = 0;
+            float r_x = 0.f;
+            auto prefetch = [&](uint32_t t0) {
                 const uint32_t nv = min((uint32_t)T, nslots - t0);
                 if ((uint32_t)tid < nv) {
                     const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
-                    sm.off[tid] = ld_stream_u32(slot + 4, pol) >> 2;
-                    if ((uint32_t)tid == nv - 1) {                 // end of the tile's last record
-                        if (t0 + nv < nslots) {
-                            sm.off[nv] = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
-                        } else {
-                            const uint32_t o = ld_stream_u32(slot + 4, pol);
-                            sm.off[nv] = (o >> 2) + 1 + (ld32(data + o) << wshift);
-                        }
-                    }
+                    r_off = ld_stream_u32(slot + 4, pol);
+                    r_x = ld_stream_f32(x + start + t0 + tid, pol);
+                    if ((uint32_t)tid == nv - 1)      // end of the tile's last record: the next slot's offset
+                        r_nxt = t0 + nv < nslots ? ld_stream_u32(slot - kSlotBytes + 4, pol) : 0xFFFFFFFFu;
+                }
+            };
+            prefetch(0);
+            for (uint32_t t0 = 0; t0 < nslots; t0 += T) {
+                const uint32_t nv = min((uint32_t)T, nslots - t0);
+                const float xv = r_x;
+                if ((uint32_t)tid < nv) {
+                    sm.off[tid] = r_off >> 2;
+                    if ((uint32_t)tid == nv - 1)      // the page's last record ends after its own length
+                        sm.off[nv] = r_nxt != 0xFFFFFFFFu ? r_nxt >> 2 : (r_off >> 2) + 1 + (ld32(data + r_off) << wshift);
                 }
                 __syncthreads();
                 if ((uint32_t)tid < nv) {
                     const uint32_t deg = (sm.off[tid + 1] - sm.off[tid] - 1) >> wshift;
-                    const float xv = ld_stream_f32(x + start + t0 + tid, pol);
                     float c = 0.f;
                     // dangling mass (R3); a routed rank counts only its own WA range (under
                     // S_BCAST every rank sees every page)
@@ -225,6 +237,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                     else c = d * xv / (float)deg;
                     sm.c[tid] = c;
                 }
+                if (t0 + T < nslots) prefetch(t0 + T);
                 __syncthreads();
                 const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
                 const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
@@ -355,23 +368,25 @@ __global__ void pr_finish_kernel(float* x, float* acc, uint64_t n, uint64_t lo, 
     const float base = (float)((1.0 - d) / (double)n + (uniform ? d * D / (double)n : 0.0));
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     const uint64_t t0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    // float4 body where x + v and acc + v share their 16-byte phase (a biased pointer of a
+    // Strategy-S range need not be 16-byte aligned at a multiple of 4); scalar head and tail
+    const uintptr_t px = (uintptr_t)(x + lo), pa = (uintptr_t)(acc + lo);
+    const uint64_t len = hi - lo;
+    const uint64_t head = ((px ^ pa) & 15u) ? len : std::min<uint64_t>(len, ((16u - (px & 15u)) & 15u) / 4u);
+    const uint64_t nvec = (len - head) / 4;
+    float4* x4 = reinterpret_cast<float4*>(x + lo + head);
+    float4* acc4 = reinterpret_cast<float4*>(acc + lo + head);
     const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
-    uint64_t a4 = (lo + 3) / 4, b4 = hi / 4;            // aligned float4 span inside [lo, hi)
-    if (b4 < a4) b4 = a4;
-    float4* x4 = reinterpret_cast<float4*>(x);
-    float4* acc4 = reinterpret_cast<float4*>(acc);
-    for (uint64_t i = a4 + t0; i < b4; i += stride) {
+    for (uint64_t i = t0; i < nvec; i += stride) {
         const float4 a = acc4[i];
         x4[i] = make_float4(base + a.x, base + a.y, base + a.z, base + a.w);
         acc4[i] = z;
     }
-    if (t0 < 8) {                                       // unaligned head [lo, 4*a4) and tail [4*b4, hi)
-        const uint64_t i = t0 < 4 ? lo + t0 : 4 * b4 + (t0 - 4);
-        const bool ok = t0 < 4 ? (i < 4 * a4 && i < hi) : (i < hi && i >= 4 * a4);
-        if (ok) {
-            x[i] = base + acc[i];
-            acc[i] = 0.f;
-        }
+    const uint64_t tail0 = head + 4 * nvec;
+    for (uint64_t k = t0; k < head + (len - tail0); k += stride) {     // head [0, head) and tail [tail0, len)
+        const uint64_t i = lo + (k < head ? k : tail0 + (k - head));
+        x[i] = base + acc[i];
+        acc[i] = 0.f;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) *dang_reset = 0.0;
 }
