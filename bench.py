@@ -158,6 +158,9 @@ class ClockSampler:
 # --------------------------------------------------------------------- reference arm ---
 
 def run_reference(args, rank):
+    """The reference arm (this tier has no installable reference): the oracle, as it stands,
+    on every host core (OpenMP build, level-synchronous BFS -- the metric's algorithm) on a
+    bounded RMAT-24 sample of the workload, one BFS per step (rank 0 only)."""
     if rank != 0:
         return
     import inputs
@@ -169,13 +172,14 @@ def run_reference(args, rank):
     deg = np.diff(g.row_ptr).astype(np.int64)
     for i in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        lv = oracle.bfs(g.row_ptr, g.col, 0)
+        lv = oracle.bfs_levelsync(g.row_ptr, g.col, 0, omp=True)
         dt = time.perf_counter() - t0
         if i >= args.warmup:
             times.append(dt)
         edges = int(deg[lv != oracle.UNREACHED].sum())
     t = float(np.sum(times))
     gteps = edges * len(times) / t / 1e9
+    threads = oracle.num_threads(omp=True)
     line = {"impl": "reference", "metric": METRIC, "value": gteps, "unit": "GTEPS", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / len(times),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
@@ -183,16 +187,45 @@ def run_reference(args, rank):
             "config": {"workload": f"rmat{args.scale}_bfs_pr_sssp_wcc", "scale": args.scale, "src": 0,
                        "sample": f"reference arm: oracle BFS (the metric's algorithm) on the RMAT-{scale} sample",
                        "sample_scale": scale},
-            "cpu_baseline": {"value": gteps, "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                             "sample": f"oracle BFS from vertex 0 on RMAT-{scale} (same generator as RMAT-{args.scale},"
-                                       f" 1/{2 ** (args.scale - scale)} of its edges), single thread, per step"},
+            "cpu_baseline": {"value": gteps, "unit": "GTEPS", "cores": threads, "kind": "oracle", "host": host_info(),
+                             "sample": f"oracle level-synchronous BFS (OpenMP build, {threads} threads) from vertex 0 "
+                                       f"on RMAT-{scale} (same generator as RMAT-{args.scale}, "
+                                       f"1/{2 ** (args.scale - scale)} of its edges), per step"},
             "e2e": {"value": gteps, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 # ----------------------------------------------------------------------------- GPU arm ---
 
-def cpu_baseline(args):
+def host_info():
+    """nproc and the lscpu model / sockets / cores of the host the oracle runs on."""
+    info = {"nproc": os.cpu_count()}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            k, _, v = ln.partition(":")
+            k = k.strip()
+            if k in ("Model name", "Socket(s)", "Core(s) per socket", "Thread(s) per core"):
+                info[k] = v.strip()
+    except Exception:  # pragma: no cover
+        pass
+    return info
+
+
+def oracle_bfs_all_cores(g, src):
+    """The oracle's level-synchronous BFS (OpenMP build, every host core) on the bench
+    graph itself: the all-core CPU baseline and the level array B_BFS is computed from."""
+    import oracle
+    t0 = time.perf_counter()
+    lv = oracle.bfs_levelsync(g.row_ptr, g.col, src, omp=True)
+    return lv, time.perf_counter() - t0
+
+
+def cpu_baseline(args, have_full=None, full_t=None, full_edges=None):
+    """the oracle as it stands on the GPU box's host cores -- (1) every core
+    (OpenMP build) on the bench workload itself (BFS, the metric's algorithm), (2) one core
+    (plain build) on an RMAT-24 sample, and the PageRank iteration time of the OpenMP build
+    on that sample (t(2 iterations) - t(1 iteration): the transpose is excluded)."""
     import inputs
     import oracle
     scale = args.ref_scale
@@ -203,12 +236,66 @@ def cpu_baseline(args):
     t_bfs = time.perf_counter() - t0
     edges = int(deg[lv != oracle.UNREACHED].sum())
     t0 = time.perf_counter()
-    oracle.pagerank(g.row_ptr, g.col, 1, 0.85)
-    t_pr = time.perf_counter() - t0
-    return {"value": edges / t_bfs / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
-            "sample": f"oracle BFS from vertex 0 on RMAT-{scale} (same generator, 1/{2 ** (args.scale - scale)} of the "
-                      f"RMAT-{args.scale} edges), single thread; plus 1 oracle PageRank iteration (incl. its transpose)",
-            "bfs_s": t_bfs, "pagerank_s_per_iter": t_pr, "sample_m": g.m}
+    oracle.pagerank(g.row_ptr, g.col, 1, 0.85, omp=True)
+    t1 = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    oracle.pagerank(g.row_ptr, g.col, 2, 0.85, omp=True)
+    t2 = time.perf_counter() - t0
+    threads = oracle.num_threads(omp=True)
+    out = {"unit": "GTEPS", "kind": "oracle", "host": host_info(),
+           "one_core": {"value": edges / t_bfs / 1e9, "cores": 1, "bfs_s": t_bfs,
+                        "sample": f"oracle FIFO-queue BFS from vertex 0 on RMAT-{scale} (same generator, "
+                                  f"1/{2 ** (args.scale - scale)} of the RMAT-{args.scale} edges), plain build"},
+           "pagerank_s_per_iter_sample": max(t2 - t1, 0.0), "pagerank_sample": f"RMAT-{scale}, OpenMP build, "
+           f"{threads} threads, t(2 iterations) - t(1 iteration)"}
+    if have_full:
+        out.update({"value": full_edges / full_t / 1e9, "cores": threads, "bfs_s": full_t,
+                    "sample": f"oracle level-synchronous BFS (OpenMP build, {threads} threads = every host core) "
+                              f"on the bench graph itself, from the bench source, once"})
+    else:
+        out.update({"value": out["one_core"]["value"], "cores": 1, "sample": out["one_core"]["sample"]})
+    return out
+
+
+def bfs_algorithmic_bytes(lv_caller, row_ptr, gr):
+    """B_BFS of SURVEY 8(d), from the oracle's level array and the page directory:
+    sum over levels of the frontier-bitmap bits of each active page (nslots / 8 bytes;
+    LP continuation pages, 1 bit each, are not counted) + per reached vertex its slot
+    offset, ADJLIST_SZ and adjacency (4 + 4 + 4 deg; the slot's VID is implied by its
+    position) + a 4-byte visited test per traversed edge + a 4-byte LV write per reached
+    vertex.  Independent of the GPU's timing."""
+    import oracle
+    reached = lv_caller != oracle.UNREACHED
+    deg = np.diff(row_ptr).astype(np.int64)
+    edges = int(deg[reached].sum())
+    nr = int(reached.sum())
+    d = gr.directory()
+    internal = gr.order()
+    ids = internal[reached].astype(np.int64)
+    page = np.searchsorted(d["start_vid"].astype(np.int64), ids, side="right") - 1
+    lev = lv_caller[reached].astype(np.int64)
+    key = np.unique(lev * (1 << 32) + page)
+    frontier_bits = float(d["nslots"][key & 0xFFFFFFFF].astype(np.int64).sum()) / 8.0
+    b = frontier_bits + 12.0 * nr + 4.0 * edges + 4.0 * edges + 4.0 * nr
+    return b, {"frontier_bitmap": frontier_bits, "slot_len_adj": 12.0 * nr + 4.0 * edges,
+               "visited_tests": 4.0 * edges, "lv_writes": 4.0 * nr, "edges": edges, "reached": nr,
+               "active_page_levels": int(key.size)}
+
+
+def h2d_peak_gbs(nbytes=256 << 20, reps=10):
+    """Pinned host -> device copy bandwidth in this process (cudaMemcpyAsync via torch), best of reps."""
+    import torch
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    best = 0.0
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        d.copy_(h, non_blocking=True)
+        e1.record()
+        torch.cuda.synchronize()
+        best = max(best, nbytes / (e0.elapsed_time(e1) * 1e-3) / 1e9)
+    return best
 
 
 def make_graph(args, rank, world, dist):
@@ -254,6 +341,7 @@ def main():
     ap.add_argument("--page-bytes", type=int, default=1 << 20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-streamed", action="store_true", help="skip the streamed-topology leg (a3)")
     ap.add_argument("--algos", default="bfs,pr,sssp,wcc")
     ap.add_argument("--order", dest="order", action="store_true", default=True,
                     help="build pages with GTS_BUILD_DEGREE_ORDER (default)")
@@ -291,6 +379,12 @@ def main():
     src = 0 if args.workload == "rmat" else int(np.argmax(np.diff(g.row_ptr)))
     wname = f"rmat{args.scale}" if args.workload == "rmat" else "twitter_shaped"
     log(f"[rank {rank}] {wname} generated n={n} m={m} in {time.time() - t0:.1f}s")
+    # the oracle on every host core, on this very graph: the all-core CPU baseline and the
+    # level array the algorithmic BFS bytes (roofline_bfs) are computed from
+    lv_oracle = t_oracle = None
+    if rank == 0 and not args.no_cpu_baseline and "bfs" in algos:
+        lv_oracle, t_oracle = oracle_bfs_all_cores(g, src)
+        log(f"[rank 0] oracle BFS on all host cores: {t_oracle:.2f}s")
     t0 = time.time()
     gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=args.page_bytes, order=args.order)
     grw = None
@@ -300,6 +394,11 @@ def main():
         del w
     gst = gr.stats()
     log(f"[rank {rank}] pages built in {time.time() - t0:.1f}s: {gst}")
+    B_bfs = bfs_parts = edges_oracle = None
+    if lv_oracle is not None:
+        B_bfs, bfs_parts = bfs_algorithmic_bytes(lv_oracle, g.row_ptr, gr)
+        edges_oracle = bfs_parts["edges"]
+        del lv_oracle
     del g
     drop_shared_graph(args, rank, world, dist)
 
@@ -433,6 +532,16 @@ def main():
                               "frac": red / avg / 1e9 / tj.get("l2_red_ceiling_gops", 1.0),
                               "ceiling_source": tj.get("_l2_red_source")}
 
+    roof_bfs = None
+    if B_bfs is not None and out["bfs"]["main_s"] > 0:
+        t_call = out["bfs"]["main_s"] / K          # the BFS kernels of one call (all levels)
+        roof_bfs = {"bound": "hbm", "kernel": "bfs_expand_kernel (+ finish / page-set kernels)",
+                    "achieved": B_bfs / t_call / 1e9, "peak": peak, "unit": "GB/s", "frac": B_bfs / t_call / 1e9 / peak,
+                    "algorithmic_bytes_per_call": B_bfs, "parts": bfs_parts, "kernel_s_per_call": t_call,
+                    "peak_source": peak_src,
+                    "what": "B_BFS of SURVEY 8(d) from the oracle's levels and the page directory / the BFS "
+                            "kernels' CUDA-event time per call"}
+
     # end-to-end through the public API with host buffers (pages re-uploaded from pinned host memory)
     e2e = None
     if not args.no_e2e and "bfs" in algos:
@@ -456,10 +565,36 @@ def main():
                        "D2H of the level array, wall clock, median",
                "pagerank_s_per_iter": float(np.median(tp_)) / 10}
 
+    # streamed topology (a3): pages from pinned host memory through the ring, after the timed region
+    streamed = None
+    if not args.no_streamed and world == 1 and "pr" in algos and "bfs" in algos:
+        peak_h2d = h2d_peak_gbs()
+        ctx.evict(gr)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        _, sp = G.gts_pagerank(ctx, gr, 2, 0.85, out=pr, residency=G.GTS_STREAMED, timing=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        t_pr = e0.elapsed_time(e1) * 1e-3 / 2
+        e0.record(stream)
+        _, sb = G.gts_bfs(ctx, gr, src, out=lv, residency=G.GTS_STREAMED, timing=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        t_bfs = e0.elapsed_time(e1) * 1e-3
+        link_pr = sp["h2d_bytes"] / 2 / t_pr / 1e9
+        link_bfs = sb["h2d_bytes"] / t_bfs / 1e9
+        streamed = {"pagerank_s_per_iter": t_pr, "bfs_gteps": sb["edges_traversed"] / t_bfs / 1e9, "bfs_s": t_bfs,
+                    "h2d_bytes_per_pr_iter": sp["h2d_bytes"] / 2, "h2d_bytes_bfs": sb["h2d_bytes"],
+                    "link_gbs_pr": link_pr, "link_gbs_bfs": link_bfs, "h2d_peak_gbs": peak_h2d,
+                    "link_frac": link_pr / peak_h2d, "link_frac_bfs": link_bfs / peak_h2d,
+                    "what": "GTS_STREAMED (forced): topology pages copied from pinned host memory into a 4 x 64 MiB "
+                            "device ring per iteration / level, kernels overlapped; RA/WA resident; CUDA events "
+                            "on the call stream; peak = pinned H2D of 256 MiB in this process, best of 10"}
+
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:
         try:
-            cpu = cpu_baseline(args)
+            cpu = cpu_baseline(args, t_oracle is not None, t_oracle, edges_oracle)
         except Exception as e:  # pragma: no cover
             cpu = {"error": str(e)}
 
@@ -488,7 +623,8 @@ def main():
                 "kernel_s_per_step": {a: out[a]["main_s"] / K for a in algos},
                 "call_ms_each_step": {a: [round(1e3 * t, 3) for t, _ in rec[a]] for a in algos},
                 "merge_s_per_step": {a: out[a]["merge_s"] / K for a in algos},
-                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "roofline": roof, "roofline_bfs": roof_bfs, "streamed": streamed,
+                "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": int(sum(out[a]["launches"] for a in algos))}
         print(json.dumps(line), flush=True)
     ctx.free()

@@ -1063,7 +1063,10 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
         for (MSlot& m : S) {
             for (int64_t q = a; q <= b; ++q)
                 if (std::binary_search(m.pages.begin(), m.pages.end(), (uint32_t)q)) m.h_list.push_back((uint32_t)q);
-            if (isrc >= m.lo && isrc < m.hi) set_source_range_kernel<<<1, 1, 0, s>>>(m.value, m.visited, m.cur, isrc);
+            // the source's LV / dist and frontier bit: on its owner under S, in every replica
+            // otherwise (P and S_BCAST keep the frontier and WA replicated)
+            if (!route || (isrc >= m.lo && isrc < m.hi))
+                set_source_range_kernel<<<1, 1, 0, s>>>(m.value, m.visited, m.cur, isrc);
         }
     }
     for (MSlot& m : S) {

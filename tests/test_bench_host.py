@@ -60,3 +60,24 @@ def test_reference_arm_line():
     line = json.loads(r.stdout.strip().splitlines()[-1])
     assert line["impl"] == "reference" and line["value"] > 0 and line["unit"] == "GTEPS"
     assert line["cpu_baseline"]["kind"] == "oracle" and line["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_bfs_algorithmic_bytes_hand_graph():
+    """B_BFS of SURVEY 8(d) on a hand graph: 0->1, 0->2, 1->2, vertex 3 isolated, one SP
+    page of 4 slots.  Levels 0 and 1 each activate that page (4 bits = 0.5 B each);
+    3 reached vertices x 12 B (slot offset + ADJLIST_SZ + LV... see bench.py) and 3
+    traversed edges x (4 B adjacency + 4 B visited test); 3 LV writes x 4 B."""
+    sys.path.insert(0, ROOT)
+    import bench
+    import inputs
+    import oracle
+    import paper_conf_sigmod_0002apsk16_b200 as G
+    g = inputs.from_edges(4, [(0, 1), (0, 2), (1, 2)])
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=256)
+    lv = oracle.bfs(g.row_ptr, g.col, 0)
+    b, parts = bench.bfs_algorithmic_bytes(lv, g.row_ptr, gr)
+    assert parts["edges"] == 3 and parts["reached"] == 3 and parts["active_page_levels"] == 2
+    assert b == 0.5 + 0.5 + 12 * 3 + 4 * 3 + 4 * 3 + 4 * 3
+    # degree-ordered pages give the same bytes (the directory is in internal IDs)
+    go = G.gts_build_pages(g.row_ptr, g.col, page_bytes=256, order=True)
+    assert bench.bfs_algorithmic_bytes(lv, g.row_ptr, go)[0] == b

@@ -15,7 +15,8 @@ mkdir -p $O
 what=${1:-tests}; shift || true
 case "$what" in
   tests)
-    timeout 3000 python -m pytest tests -m gpu ${@:--x -q} > $O/tests.log 2>&1; echo "pytest rc=$?"; tail -5 $O/tests.log ;;
+    [ $# -eq 0 ] && set -- -x -q
+    timeout 3000 python -m pytest -m gpu "$@" > $O/tests.log 2>&1; echo "pytest rc=$?"; tail -5 $O/tests.log ;;
   bench)
     timeout 1500 python bench.py "$@" > $O/bench.json 2> $O/bench.log; echo "bench rc=$?"; tail -c 3000 $O/bench.json ;;
   launches)
