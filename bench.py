@@ -342,6 +342,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-streamed", action="store_true", help="skip the streamed-topology leg (a3)")
+    ap.add_argument("--strategy", default="P", choices=["P", "S", "S_BCAST"],
+                    help="multi-GPU strategy for N > 1 (SURVEY 8(e)); P = the default scaling run")
     ap.add_argument("--algos", default="bfs,pr,sssp,wcc")
     ap.add_argument("--order", dest="order", action="store_true", default=True,
                     help="build pages with GTS_BUILD_DEGREE_ORDER (default)")
@@ -386,11 +388,19 @@ def main():
         lv_oracle, t_oracle = oracle_bfs_all_cores(g, src)
         log(f"[rank 0] oracle BFS on all host cores: {t_oracle:.2f}s")
     t0 = time.time()
-    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=args.page_bytes, order=args.order)
+    strat = {"P": G.GTS_STRATEGY_P, "S": G.GTS_STRATEGY_S, "S_BCAST": G.GTS_STRATEGY_S_BCAST}[args.strategy]
+    # N > 1: every rank builds and pins only the pages it processes (GTS_BUILD_OWNER_FILTER),
+    # so host page bytes per rank are ~T_topo / N
+    own = (rank, world, strat) if world > 1 else None
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=args.page_bytes, order=args.order, owner=own)
+    grs = None
+    if "wcc" in algos and world > 1 and strat == G.GTS_STRATEGY_S:   # routed WCC: symmetrised pages
+        grs = G.gts_build_pages(g.row_ptr, g.col, page_bytes=args.page_bytes, order=args.order, owner=own,
+                                symmetric=True)
     grw = None
     if "sssp" in algos:
         w = inputs.edge_weights(g)
-        grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=args.page_bytes, order=args.order)
+        grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=args.page_bytes, order=args.order, owner=own)
         del w
     gst = gr.stats()
     log(f"[rank {rank}] pages built in {time.time() - t0:.1f}s: {gst}")
@@ -424,15 +434,15 @@ def main():
             e1 = torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             if a == "bfs":
-                _, st = G.gts_bfs(ctx, gr, src, out=lv, timing=True)
+                _, st = G.gts_bfs(ctx, gr, src, out=lv, timing=True, strategy=strat)
             elif a == "pr":
                 if sampler is not None:
                     sampler.kick()
-                _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=pr, timing=True)
+                _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=pr, timing=True, strategy=strat)
             elif a == "sssp":
-                _, st = G.gts_sssp(ctx, grw, src, out=ds, timing=True)
+                _, st = G.gts_sssp(ctx, grw, src, out=ds, timing=True, strategy=strat)
             else:
-                _, st = G.gts_wcc(ctx, gr, out=lab, timing=True)
+                _, st = G.gts_wcc(ctx, grs if grs is not None else gr, out=lab, timing=True, strategy=strat)
             e1.record(stream)
             evs[a] = (e0, e1)
             res[a] = st
@@ -552,12 +562,12 @@ def main():
             ctx.evict(gr)
             barrier()
             t0 = time.perf_counter()
-            _, st = G.gts_bfs(ctx, gr, src, out=hl)
+            _, st = G.gts_bfs(ctx, gr, src, out=hl, strategy=strat)
             tb.append(maxred(time.perf_counter() - t0))
             ctx.evict(gr)
             barrier()
             t0 = time.perf_counter()
-            G.gts_pagerank(ctx, gr, 10, 0.85, out=hp)
+            G.gts_pagerank(ctx, gr, 10, 0.85, out=hp, strategy=strat)
             tp_.append(maxred(time.perf_counter() - t0))
         e2e = {"value": out["bfs"]["edges"] / K / float(np.median(tb)) / 1e9, "unit": "GTEPS",
                "h2d_bytes_per_step": int(gst["topo_bytes"] / world), "d2h_bytes_per_step": 4 * n,
@@ -609,8 +619,9 @@ def main():
                            "page_bytes": args.page_bytes, "num_pages": gst["num_pages"], "n_lp": gst["n_lp"],
                            "vertex_order": "in-degree (GTS_BUILD_DEGREE_ORDER)" if args.order else "VID",
                            "topo_bytes": gst["topo_bytes"], "residency": "resident",
-                           "strategy": "P" if world > 1 else "single",
-                           "parallelism": f"strategy-P x{world}",
+                           "strategy": args.strategy if world > 1 else "single",
+                           "parallelism": f"strategy-{args.strategy} x{world}",
+                           "host_page_bytes_per_rank": gst["host_page_bytes"],
                            "l2": "inputs larger than L2 (topology %.1f GB vs 126 MB L2), no flush" %
                                  (gst["topo_bytes"] / 1e9),
                            "step": "+".join(algos)},

@@ -127,9 +127,12 @@ constexpr size_t pr_dyn_smem() {
 // dense hot-set sizes: 512-thread CTAs (2 per SM) hold kHotDense floats each;
 // 1024-thread CTAs (1 per SM) hold kHotDenseBig
 constexpr uint32_t kHotDenseBig = 53248;
+// vertices per thread in a scatter tile (1024-thread CTAs: 2048-vertex tiles)
+constexpr int kPrVpt = 2;
 
-__device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const uint32_t* rvt) {
-    return enc == GTS_ENTRY_VID32 ? e : __ldg(rvt + (e >> 16)) + (e & 0xFFFFu);
+template <bool kVid32>
+__device__ __forceinline__ uint32_t pr_decode(uint32_t e, const uint32_t* rvt) {
+    return kVid32 ? e : __ldg(rvt + (e >> 16)) + (e & 0xFFFFu);
 }
 
 // K_PR_SP / K_PR_LP (Alg 4/5) for a persistent CTA of T threads.  The record
@@ -137,11 +140,11 @@ __device__ __forceinline__ uint32_t pr_decode(uint32_t e, uint32_t enc, const ui
 // (records are packed in VID order from offset 0), streamed with 16-byte
 // evict_first loads, kPrUnroll in flight per thread; the owner of each 4-word
 // group is found by a binary search over the tile's record offsets.
-template <bool kWeighted, int kMode, int T, int kMinBlocks, uint32_t H>
+template <bool kWeighted, int kMode, int T, int kMinBlocks, uint32_t H, int VPT, bool kVid>
 __global__ void __launch_bounds__(T, kMinBlocks)
 pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__ hot_keys,
                   float d, double* dang_out, uint32_t* work_ctr, uint32_t n_hot, const RouteParams rp) {
-    __shared__ PrSmem<T> sm;
+    __shared__ PrSmem<T * VPT> sm;
     extern __shared__ uint4 dyn_smem[];
     uint32_t* hkeys = reinterpret_cast<uint32_t*>(dyn_smem);
     float* hacc = kMode == kHash ? reinterpret_cast<float*>(hkeys + kHotSlots) : reinterpret_cast<float*>(dyn_smem);
@@ -157,7 +160,6 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
     __syncthreads();
     const uint64_t pol = policy_evict_first();
     const uint32_t count = ps.count;
-    const uint32_t enc = ps.entry_encoding;
     constexpr uint32_t wshift = kWeighted ? 1 : 0;
     PrEmitter<kMode, H> em{acc, hkeys, hacc, &rp, 0u, 0.f, false};
     double dang = 0.0;
@@ -194,51 +196,70 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
 #pragma unroll
                     for (int k = 0; k < 4; ++k) {
                         const uint32_t w = 4 * q + k;
-                        if (w >= 1 && w < wend) em.edge(pr_decode(word_of(v[u], k), enc, ps.rvt_start), c);
+                        if (w >= 1 && w < wend) em.edge(pr_decode<kVid>(word_of(v[u], k), ps.rvt_start), c);
                     }
                 }
             }
         } else {
             const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
-            // Software pipeline over the page's tiles: the slot offsets and x values of
-            // tile t+1 are loaded into registers while tile t's records stream, so a tile
-            // exposes one DRAM latency (its records) instead of three in a row (offsets,
-            // then x, then records) -- on low-degree pages a tile's records are only a few
-            // KB, so these latencies, not bytes, set the walk's time.
-            uint32_t r_off = 0, r_nxt = 0;
-            float r_x = 0.f;
+            // Tiles of TV = VPT * T consecutive vertices.  Software pipeline over the page's
+            // tiles: the slot offsets and x values of tile t+1 are loaded into registers
+            // while tile t's records stream, so a tile exposes one DRAM latency (its
+            // records) instead of three in a row (offsets, then x, then records) -- on
+            // low-degree pages a tile's records are only a few KB, so latencies, not
+            // bytes, set the walk's time.
+            constexpr uint32_t TV = (uint32_t)T * VPT;
+            uint32_t r_off[VPT], r_nxt = 0;
+            float r_x[VPT];
             auto prefetch = [&](uint32_t t0) {
-                const uint32_t nv = min((uint32_t)T, nslots - t0);
-                if ((uint32_t)tid < nv) {
-                    const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
-                    r_off = ld_stream_u32(slot + 4, pol);
-                    r_x = ld_stream_f32(x + start + t0 + tid, pol);
-                    if ((uint32_t)tid == nv - 1)      // end of the tile's last record: the next slot's offset
-                        r_nxt = t0 + nv < nslots ? ld_stream_u32(slot - kSlotBytes + 4, pol) : 0xFFFFFFFFu;
+                const uint32_t nv = min(TV, nslots - t0);
+#pragma unroll
+                for (int k = 0; k < VPT; ++k) {
+                    const uint32_t i = (uint32_t)tid + (uint32_t)k * T;
+                    if (i < nv) {
+                        const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + i + 1);
+                        r_off[k] = ld_stream_u32(slot + 4, pol);
+                        r_x[k] = ld_stream_f32(x + start + t0 + i, pol);
+                        if (i == nv - 1)              // end of the tile's last record: the next slot's offset
+                            r_nxt = t0 + nv < nslots ? ld_stream_u32(slot - kSlotBytes + 4, pol) : 0xFFFFFFFFu;
+                    }
                 }
             };
             prefetch(0);
-            for (uint32_t t0 = 0; t0 < nslots; t0 += T) {
-                const uint32_t nv = min((uint32_t)T, nslots - t0);
-                const float xv = r_x;
-                if ((uint32_t)tid < nv) {
-                    sm.off[tid] = r_off >> 2;
-                    if ((uint32_t)tid == nv - 1)      // the page's last record ends after its own length
-                        sm.off[nv] = r_nxt != 0xFFFFFFFFu ? r_nxt >> 2 : (r_off >> 2) + 1 + (ld32(data + r_off) << wshift);
+            for (uint32_t t0 = 0; t0 < nslots; t0 += TV) {
+                const uint32_t nv = min(TV, nslots - t0);
+#pragma unroll
+                for (int k = 0; k < VPT; ++k) {
+                    const uint32_t i = (uint32_t)tid + (uint32_t)k * T;
+                    if (i < nv) {
+                        sm.off[i] = r_off[k] >> 2;
+                        if (i == nv - 1)              // the page's last record ends after its own length
+                            sm.off[nv] = r_nxt != 0xFFFFFFFFu ? r_nxt >> 2
+                                                              : (r_off[k] >> 2) + 1 + (ld32(data + r_off[k]) << wshift);
+                    }
                 }
                 __syncthreads();
-                if ((uint32_t)tid < nv) {
-                    const uint32_t deg = (sm.off[tid + 1] - sm.off[tid] - 1) >> wshift;
-                    float c = 0.f;
-                    // dangling mass (R3); a routed rank counts only its own WA range (under
-                    // S_BCAST every rank sees every page)
-                    if (deg == 0 && (kMode != kRoute || (uint64_t)(start + t0 + tid) - rp.lo < rp.hi - rp.lo))
-                        dang += (double)xv;
-                    else c = d * xv / (float)deg;
-                    sm.c[tid] = c;
+#pragma unroll
+                for (int k = 0; k < VPT; ++k) {
+                    const uint32_t i = (uint32_t)tid + (uint32_t)k * T;
+                    if (i < nv) {
+                        const uint32_t deg = (sm.off[i + 1] - sm.off[i] - 1) >> wshift;
+                        float c = 0.f;
+                        // dangling mass (R3); a routed rank counts only its own WA range (under
+                        // S_BCAST every rank sees every page)
+                        if (deg == 0 && (kMode != kRoute || (uint64_t)(start + t0 + i) - rp.lo < rp.hi - rp.lo))
+                            dang += (double)r_x[k];
+                        else c = d * r_x[k] / (float)deg;
+                        sm.c[i] = c;
+                    }
                 }
-                if (t0 + T < nslots) prefetch(t0 + T);
+                if (t0 + TV < nslots) prefetch(t0 + TV);
                 __syncthreads();
+                // the tile's record region, 16-byte evict_first loads, kPrUnroll in flight per
+                // thread (coalesced: lane-consecutive groups); the owner of each 16-byte group by
+                // a binary search over the tile's offsets, then record by record.  (Giving each
+                // thread 4 consecutive groups -- one search per 16 words -- measured slower on
+                // RMAT-27: 14.4 vs 11.5 ms, the uncoalesced loads cost more than the searches.)
                 const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
                 const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
                 for (uint32_t qb = qbeg + tid; qb < qend; qb += T * kPrUnroll) {
@@ -270,7 +291,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                             }
                             const uint32_t rel = w - cur;     // 0 = ADJLIST_SZ word; > deg = weight words
                             if (rel == 0 || rel > ((nxt - cur - 1) >> wshift)) continue;
-                            em.edge(pr_decode(word_of(v[u], k), enc, ps.rvt_start), sm.c[j]);
+                            em.edge(pr_decode<kVid>(word_of(v[u], k), ps.rvt_start), sm.c[j]);
                         }
                     }
                 }
@@ -474,24 +495,36 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         dyn = 0;
         threads = kThreads;
         n_hot = 0;
-    } else if (mode == kHash) {
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kHash, kThreads, 2, 0>
-                           : (const void*)pr_scatter_kernel<false, kHash, kThreads, 2, 0>;
-        dyn = pr_dyn_smem<kHash, 0>();
-        threads = kThreads;
-        n_hot = 0;
-    } else if (mode == kRoute) {
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kRoute, 1024, 1, kHotDenseBig>
-                           : (const void*)pr_scatter_kernel<false, kRoute, 1024, 1, kHotDenseBig>;
-        dyn = pr_dyn_smem<kRoute, kHotDenseBig>();
-        threads = 1024;
-        n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
     } else {
-        kern = g->weighted ? (const void*)pr_scatter_kernel<true, kDense, 1024, 1, kHotDenseBig>
-                           : (const void*)pr_scatter_kernel<false, kDense, 1024, 1, kHotDenseBig>;
-        dyn = pr_dyn_smem<kDense, kHotDenseBig>();
-        threads = 1024;
-        n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
+        // template instance: <weighted, mode, threads, CTAs/SM, hot set, vertices per thread, VID32 entries>
+        const bool vid = g->entry_encoding == GTS_ENTRY_VID32;
+        const char* dv = getenv("GTS_DEV_VPT");     // (temporary A/B of the tile size)
+        const int vpt = dv ? atoi(dv) : kPrVpt;
+#define GTS_PRK(W, M, TT, MB, HH, V) (vid ? (const void*)pr_scatter_kernel<W, M, TT, MB, HH, V, true> \
+                                          : (const void*)pr_scatter_kernel<W, M, TT, MB, HH, V, false>)
+        if (mode == kHash) {
+            kern = g->weighted ? GTS_PRK(true, kHash, kThreads, 2, 0, 1) : GTS_PRK(false, kHash, kThreads, 2, 0, 1);
+            dyn = pr_dyn_smem<kHash, 0>();
+            threads = kThreads;
+            n_hot = 0;
+        } else if (mode == kRoute) {
+            kern = g->weighted ? GTS_PRK(true, kRoute, 1024, 1, kHotDenseBig, kPrVpt)
+                               : GTS_PRK(false, kRoute, 1024, 1, kHotDenseBig, kPrVpt);
+            dyn = pr_dyn_smem<kRoute, kHotDenseBig>();
+            threads = 1024;
+            n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
+        } else {
+            if (vpt == 1)
+                kern = g->weighted ? GTS_PRK(true, kDense, 1024, 1, kHotDenseBig, 1)
+                                   : GTS_PRK(false, kDense, 1024, 1, kHotDenseBig, 1);
+            else
+                kern = g->weighted ? GTS_PRK(true, kDense, 1024, 1, kHotDenseBig, 2)
+                                   : GTS_PRK(false, kDense, 1024, 1, kHotDenseBig, 2);
+            dyn = pr_dyn_smem<kDense, kHotDenseBig>();
+            threads = 1024;
+            n_hot = (uint32_t)std::min<uint64_t>(n, kHotDenseBig);
+        }
+#undef GTS_PRK
     }
     GTS_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
     int grid = 0;

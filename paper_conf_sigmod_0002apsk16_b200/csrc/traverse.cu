@@ -585,7 +585,18 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     // BFS on resident pages, one rank: levels are enqueued levels_per_sync (default 8) at
     // a time without a host round trip (per-level new-vertex counts and page-list counts go
     // to device arrays; the levels after the last non-empty one run on an empty frontier)
-    const uint32_t B = (algo == kBFS && !streamed && K > 0) ? (rc.levels_per_sync ? rc.levels_per_sync : 8u) : 1u;
+    // SSSP with an unbounded bucket (the default: T never moves) batches its rounds the same way,
+    // each round's pending count and page-list count going to a 64-entry ring
+    const bool sssp_batch = algo == kSSSP && !streamed && !cached && rc.sssp_delta == 0;
+    const uint32_t B = ((algo == kBFS && K > 0) || sssp_batch) && !streamed
+                           ? std::min<uint32_t>(rc.levels_per_sync ? rc.levels_per_sync : 8u, 32u) : 1u;
+    constexpr uint32_t kRing = 64;
+    unsigned long long* ring_cnt = nullptr;          // SSSP batched rounds: [kRing] pending counts
+    uint32_t* ring_pages = nullptr;                  // [kRing] pages in the next round's list
+    if (sssp_batch) {
+        GTS_TRY(c->buf(kBufLvCnt, (size_t)kRing * 12, (void**)&ring_cnt));
+        ring_pages = reinterpret_cast<uint32_t*>(ring_cnt + kRing);
+    }
     unsigned long long* lvl_cnt = nullptr;           // [K] new vertices per level (BFS)
     uint32_t* lvl_pages = nullptr;                   // [K] pages in the list of level L
     if (algo == kBFS) {
@@ -636,8 +647,13 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
         } else {
             GTS_CUDA(cudaMemsetAsync(&ctr->near, 0, 8, s));
             GTS_CUDA(cudaMemsetAsync(&ctr->minpend, 0xFF, 4, s));
+            unsigned long long* cnt = &ctr->count;
+            if (sssp_batch) {
+                cnt = ring_cnt + (L % kRing);
+                GTS_CUDA(cudaMemsetAsync(cnt, 0, 8, s));
+            }
             sssp_finish_kernel<<<fin_grid, 256, 0, s>>>(nullptr, 1, words, 0, words, cur, next, value, T,
-                                                        &ctr->count, &ctr->near, &ctr->minpend);
+                                                        cnt, &ctr->near, &ctr->minpend);
         }
         frontier_pages_kernel<<<fin_grid, 256, 0, s>>>(next, c->dg.rvt_start, c->dg.nslots,
                                                        c->dg.all_local ? nullptr : c->dg.local_list,
@@ -648,10 +664,12 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
         GTS_CUDA(cudaGetLastError());
         if (algo == kBFS && L < K)                    // pages of level L+1's list (lvl_pages has K+1 entries)
             GTS_CUDA(cudaMemcpyAsync(lvl_pages + L + 1, &ctr->list_count, 4, cudaMemcpyDeviceToDevice, s));
+        if (sssp_batch)
+            GTS_CUDA(cudaMemcpyAsync(ring_pages + (L % kRing), &ctr->list_count, 4, cudaMemcpyDeviceToDevice, s));
         ++levels;
-        // host round trip: every level (SSSP, streamed, multi-rank), else every B levels and
+        // host round trip: every level (near-far SSSP, streamed), else every B levels and
         // before the level slots run out
-        const bool sync = B == 1 || (L + 1) % B == 0 || !(slots && L + 3 < K);
+        const bool sync = B == 1 || (L + 1) % B == 0 || (algo == kBFS && !(slots && L + 3 < K));
         if (!sync) {
             if (slots && L + 2 < K) {
                 cur = next;
@@ -659,8 +677,21 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
                 GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
                 continue;
             }
+            if (sssp_batch) {
+                std::swap(cur, next);
+                GTS_CUDA(cudaMemsetAsync(next, 0, words * 4, s));
+                continue;
+            }
         }
         GTS_CUDA(cudaMemcpyAsync(&h, ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
+        std::vector<unsigned long long> r_cnt;
+        std::vector<uint32_t> r_pages;
+        if (sssp_batch) {
+            r_cnt.resize(kRing);
+            r_pages.resize(kRing);
+            GTS_CUDA(cudaMemcpyAsync(r_cnt.data(), ring_cnt, kRing * 8, cudaMemcpyDeviceToHost, s));
+            GTS_CUDA(cudaMemcpyAsync(r_pages.data(), ring_pages, kRing * 4, cudaMemcpyDeviceToHost, s));
+        }
         if (algo == kBFS && L < K) {
             h_cnt.resize(L + 1);
             h_pages.resize(L + 2);
@@ -685,8 +716,22 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
             h.list_count = h_pages[L + 1];
             if (done) break;
         }
+        if (sssp_batch) {                         // rounds synced..L of the batch
+            bool done = false;
+            for (uint32_t l = synced; l <= L; ++l) {
+                if (r_cnt[l % kRing] == 0) {         // round l left nothing pending: SSSP ends there
+                    levels = l + 1;
+                    done = true;
+                    break;
+                }
+                if (l < L) pages_processed += r_pages[l % kRing];
+            }
+            synced = L + 1;
+            h.count = done ? 0 : r_cnt[L % kRing];
+            h.list_count = r_pages[L % kRing];
+        }
         if (h.count == 0) break;
-        if (algo == kSSSP && h.near == 0) {      // nothing pending within T: open the next bucket
+        if (algo == kSSSP && !sssp_batch && h.near == 0) {   // nothing pending within T: open the next bucket
             const uint64_t nt = (uint64_t)h.minpend + delta;
             T = (uint32_t)std::min<uint64_t>(nt, 0xFFFFFFFEull);
         }
