@@ -32,21 +32,26 @@
  *     slot_i   at page_bytes - 8 - 8(i+1): u32 VID, u32 OFF
  *              VID = START_VID + i (VIDs consecutive within a page)
  *     rec_i    at OFF (records are packed in VID order from offset 0):
- *              u32 ADJLIST_SZ, u32 ADJLIST[ADJLIST_SZ] (, u32 W[ADJLIST_SZ] if
- *              the graph is weighted)
+ *              u32 ADJLIST_SZ, u32 ADJLIST[ADJLIST_SZ]              (unweighted)
+ *              u32 ADJLIST_SZ, u32 0, (u32 ADJ, u32 W)[ADJLIST_SZ]  (weighted: every
+ *              record 8-byte aligned, an edge's neighbour and weight adjacent, so
+ *              one 8-byte load reads both; the weights are not in the paper's
+ *              format, R11)
  *   LP (large page: one chunk of the adjacency list of one high-degree
  *       vertex, Fig 1c):
  *     footer   (last 16 B)        : u32 total_deg, u32 chunk_idx,
  *                                   u32 nslots (= 1), u32 kind (= GTS_PAGE_LP)
  *     slot_0   at page_bytes - 16 - 8 : u32 VID, u32 OFF (= 0)
- *     rec_0    at 0               : u32 chunk_len, u32 ADJLIST[chunk_len] (, W)
+ *     rec_0    at 0               : u32 chunk_len, u32 ADJLIST[chunk_len]
+ *                                   (weighted: u32 chunk_len, u32 0, (ADJ, W)[chunk_len])
  *   ADJLIST entries: GTS_ENTRY_VID32 (default) stores the neighbour VID;
  *   GTS_ENTRY_PID16_SLOT16 stores the paper's physical record ID
  *   (ADJ_PID << 16 | ADJ_OFF), whose VID is RVT[ADJ_PID].START_VID + ADJ_OFF
  *   (App A).  Both carry the same information (R-PID in DESIGN.md).
  *   Unused bytes are zero.  SP and LP pages share one page-ID space in VID
- *   order; a vertex is an LP vertex iff 4 + 4*deg*(1+weighted) + 8 does not
- *   fit an empty SP (R15); greedy packing in VID order (R15).
+ *   order; a vertex is an LP vertex iff its record (4 + 4 deg, weighted 8 + 8 deg)
+ *   + its 8-byte slot does not fit an empty SP (R15); greedy packing in VID
+ *   order (R15).
  */
 #ifndef GTS_H
 #define GTS_H

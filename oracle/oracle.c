@@ -283,7 +283,8 @@ int oracle_wcc(uint64_t n, const uint64_t* row_ptr, const uint32_t* col, uint32_
  *   footer (last 8 bytes):  u32 nslots, u32 kind (0 = SP, 1 = LP)
  *   LP adds before it:       u32 total_deg, u32 chunk_idx
  *   slot k (k = 0,1,..):     at page_end - footer - 8(k+1): u32 vid, u32 off
- *   record at off:           u32 sz, u32 adj[sz] (, u32 w[sz] if weighted)
+ *   record at off:           u32 sz, u32 adj[sz]            (unweighted)
+ *                            u32 sz, u32 0, (u32 adj, u32 w)[sz]  (weighted)
  * Entry encoding 0 = VID32; 1 = PID16_SLOT16 (ADJ_PID << 16 | ADJ_OFF), decoded
  * as RVT[ADJ_PID].START_VID + ADJ_OFF (App A) where START_VID of a page
  * is the VID of its slot 0.
@@ -326,8 +327,9 @@ int64_t oracle_decode_pages(const uint8_t* pages, uint64_t num_pages, uint64_t p
             const uint8_t* s = end - footer - 8 * (uint64_t)(k + 1);
             uint32_t vid = rd32(s), off = rd32(s + 4);
             uint32_t sz = rd32(pg + off);
+            uint64_t first = weighted ? 8 : 4, stride = weighted ? 8 : 4;   /* entries after the header */
             for (uint32_t i = 0; i < sz; ++i) {
-                uint32_t e = rd32(pg + off + 4 + 4 * (uint64_t)i);
+                uint32_t e = rd32(pg + off + first + stride * (uint64_t)i);
                 uint32_t v;
                 if (entry_encoding == 1) {
                     uint32_t pid = e >> 16, slot = e & 0xFFFFu;
@@ -337,7 +339,7 @@ int64_t oracle_decode_pages(const uint8_t* pages, uint64_t num_pages, uint64_t p
                     v = e;
                 }
                 col[deg[vid]] = v;
-                if (weighted && w) w[deg[vid]] = rd32(pg + off + 4 + 4 * (uint64_t)sz + 4 * (uint64_t)i);
+                if (weighted && w) w[deg[vid]] = rd32(pg + off + first + stride * (uint64_t)i + 4);
                 deg[vid]++;
             }
         }

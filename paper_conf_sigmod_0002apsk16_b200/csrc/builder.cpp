@@ -62,9 +62,10 @@ static bool valid_page_bytes(uint32_t pb) {
 
 int plan_pages(uint64_t n, const uint64_t* row_ptr, bool weighted, uint32_t page_bytes,
                uint32_t entry_encoding, std::vector<PagePlanEntry>& plan, gts_graph_stats* st) {
-    const uint64_t words_per_edge = weighted ? 2 : 1;
+    // record bytes: 4 + 4 deg (unweighted) or 8 + 8 deg (weighted: header sz, 0; (adj, w) pairs)
+    const uint64_t words_per_edge = rec_edge_words(weighted), hdr_bytes = 4 * rec_hdr_words(weighted);
     const uint64_t sp_cap_bytes = page_bytes - kSpFooter;                    // records + slots
-    const uint64_t lp_cap = (page_bytes - kLpFooter - kSlotBytes - 4) / (4 * words_per_edge);
+    const uint64_t lp_cap = (page_bytes - kLpFooter - kSlotBytes - hdr_bytes) / (4 * words_per_edge);
     const uint64_t max_slots = entry_encoding == GTS_ENTRY_PID16_SLOT16 ? 65536 : UINT32_MAX;
     if (lp_cap == 0) return fail(GTS_EINVAL, "page_bytes %u too small for one LP entry", page_bytes);
     plan.clear();
@@ -84,7 +85,7 @@ int plan_pages(uint64_t n, const uint64_t* row_ptr, bool weighted, uint32_t page
         uint64_t deg = row_ptr[v + 1] - row_ptr[v];
         if (deg > maxdeg) maxdeg = deg;
         if (deg >= (1ull << 32)) return fail(GTS_EOVERFLOW, "vertex %llu has degree >= 2^32", (unsigned long long)v);
-        uint64_t need = 4 + 4 * words_per_edge * deg + kSlotBytes;
+        uint64_t need = hdr_bytes + 4 * words_per_edge * deg + kSlotBytes;
         if (need > sp_cap_bytes) {                                            // LP vertex
             close_sp();
             uint64_t chunks = (deg + lp_cap - 1) / lp_cap;
@@ -92,7 +93,7 @@ int plan_pages(uint64_t n, const uint64_t* row_ptr, bool weighted, uint32_t page
             for (uint64_t c = 0; c < chunks; ++c) {
                 uint64_t len = std::min(lp_cap, deg - c * lp_cap);
                 plan.push_back(PagePlanEntry{(uint32_t)v, 1, GTS_PAGE_LP, first, first + (int64_t)chunks - 1});
-                used_total += 4 + 4 * words_per_edge * len + kSlotBytes + kLpFooter;
+                used_total += hdr_bytes + 4 * words_per_edge * len + kSlotBytes + kLpFooter;
             }
             n_lp += chunks;
             ++n_lpv;
@@ -385,8 +386,8 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
             }
         }
     }
-    const uint64_t wpe = weighted ? 2 : 1;
-    const uint64_t lp_cap = (pb - kLpFooter - kSlotBytes - 4) / (4 * wpe);
+    const uint64_t wpe = rec_edge_words(weighted), hdrb = 4 * rec_hdr_words(weighted);
+    const uint64_t lp_cap = (pb - kLpFooter - kSlotBytes - hdrb) / (4 * wpe);
 
     #pragma omp parallel for schedule(dynamic, 4)
     for (int64_t hp = 0; hp < (int64_t)g->n_host_pages; ++hp) {
@@ -394,12 +395,13 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
         uint8_t* pg = g->pages + (size_t)hp * pb;
         std::memset(pg, 0, pb);
         const PagePlanEntry& e = plan[p];
+        // entries after the record header: adj[len], or (adj, w) pairs for weighted records
         auto put_entries = [&](uint8_t* dst, uint64_t k0, uint64_t len) {
             for (uint64_t i = 0; i < len; ++i) {
                 uint32_t v = col_idx[k0 + i];
-                wr32(dst + 4 * i, enc == GTS_ENTRY_PID16_SLOT16 ? phys[v] : v);
+                wr32(dst + 4 * wpe * i, enc == GTS_ENTRY_PID16_SLOT16 ? phys[v] : v);
+                if (weighted) wr32(dst + 8 * i + 4, weights[k0 + i]);
             }
-            if (weighted) std::memcpy(dst + 4 * len, weights + k0, 4 * len);
         };
         if (e.kind == GTS_PAGE_LP) {
             uint64_t v = e.start_vid;
@@ -407,7 +409,7 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
             uint64_t c = (uint64_t)(p - e.lp_first);
             uint64_t k0 = c * lp_cap, len = std::min(lp_cap, deg - k0);
             wr32(pg, (uint32_t)len);
-            put_entries(pg + 4, row_ptr[v] + k0, len);
+            put_entries(pg + hdrb, row_ptr[v] + k0, len);
             uint8_t* end = pg + pb;
             wr32(end - 4, GTS_PAGE_LP);
             wr32(end - 8, 1);
@@ -422,11 +424,11 @@ extern "C" int gts_build_pages(uint64_t n, uint64_t m, const uint64_t* row_ptr, 
                 uint64_t v = (uint64_t)e.start_vid + s;
                 uint64_t deg = row_ptr[v + 1] - row_ptr[v];
                 wr32(pg + off, (uint32_t)deg);
-                put_entries(pg + off + 4, row_ptr[v], deg);
+                put_entries(pg + off + hdrb, row_ptr[v], deg);
                 uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(s + 1);
                 wr32(slot, (uint32_t)v);
                 wr32(slot + 4, (uint32_t)off);
-                off += 4 + 4 * wpe * deg;
+                off += hdrb + 4 * wpe * deg;
             }
             wr32(end - 4, GTS_PAGE_SP);
             wr32(end - 8, e.nslots);

@@ -102,7 +102,7 @@ int make_ranks(Context* c, const gts_run_config& rc, Ranks* R) {
 int Ranks::allreduce(void* const* bufs, size_t count, CType t, COp op) {
     if (world == 1 || count == 0) return GTS_OK;
     cudaStream_t s = c->stream;
-    bytes += count * type_size(t);
+    bytes += count * type_size(t) * nloc;     // (bytes: summed over the ranks this process runs)
     if (!virt) {
         GTS_NCCL(ncclAllReduce(bufs[0], bufs[0], count, nccl_type(t), nccl_op(op), c->comm, s));
         return GTS_OK;
@@ -122,7 +122,7 @@ int Ranks::allreduce(void* const* bufs, size_t count, CType t, COp op) {
 
 int Ranks::allgather(const void* const* send, void* const* recv, size_t nbytes) {
     cudaStream_t s = c->stream;
-    bytes += nbytes;
+    bytes += nbytes * nloc;
     if (!virt) {
         if (world == 1) {
             if (recv[0] != send[0]) GTS_CUDA(cudaMemcpyAsync(recv[0], send[0], nbytes, cudaMemcpyDeviceToDevice, s));
@@ -152,6 +152,7 @@ int Ranks::gather_ranges(void* const* full, const std::vector<uint64_t>& vr, siz
         bytes += (vr[r0 + 1] - vr[r0]) * es;
         return GTS_OK;
     }
+    bytes += (vr[nloc] - vr[0]) * es;
     for (int i = 0; i < nloc; ++i)
         for (int q = 0; q < nloc; ++q)
             if (q != i && full[q] != full[i] && vr[q + 1] > vr[q])
@@ -182,6 +183,7 @@ int Ranks::reduce_to_owners(float* const* part, float* const* dst, const std::ve
         GTS_CUDA(cudaGetLastError());
         return GTS_OK;
     }
+    bytes += limit * 4 * nloc;
     PtrArr pp{}, pd{};
     Ranges rg{};
     for (int i = 0; i < nloc; ++i) {

@@ -137,7 +137,7 @@ __device__ __forceinline__ WinMask win_mask(const uint32_t* off, int j0, uint32_
 
 // Op interface:
 //   static constexpr bool kReadWeights;  -- the op needs edge weights
-//   static constexpr bool kWeighted;     -- the pages carry weights (record = sz, adj[sz], w[sz])
+//   static constexpr bool kWeighted;     -- the pages carry weights (record = sz, 0, (adj, w)[sz])
 //   const uint32_t* frontier()                           -- bitmap behind select(), or nullptr (all)
 //   bool select(uint32_t vid)                            -- SP vertex expanded?
 //   uint32_t payload(uint32_t vid, uint32_t deg)         -- per selected vertex
@@ -173,8 +173,14 @@ __device__ __forceinline__ void gather_items(const PageSet& ps, Op& op, TileSmem
             }
             const uint32_t local = e - sm.pre[j];
             const uint32_t* adj = words + sm.off[j];
-            dst[q] = valid[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
-            w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_l1_u32(adj + sm.deg[j] + local, pol) : 0u;
+            if (Op::kWeighted) {                // (neighbour, weight): one 8-byte load
+                const uint2 pr = valid[q] ? ld_stream_l1_v2(adj + 2 * local, pol) : make_uint2(0u, 0u);
+                dst[q] = pr.x;
+                w[q] = pr.y;
+            } else {
+                dst[q] = valid[q] ? ld_stream_l1_u32(adj + local, pol) : 0u;
+                w[q] = 0u;
+            }
             pl[q] = sm.payload[j];
             src[q] = sm.src[j];
         }
@@ -227,7 +233,7 @@ __device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, cons
             uint32_t p2, nf, ex2, total;
             tile_scan(item, item ? deg : 0u, p2, nf, ex2, total, sm);
             if (item) {
-                sm.off[p2] = off / 4 + 1;
+                sm.off[p2] = off / 4 + rec_hdr_words(Op::kWeighted);
                 sm.deg[p2] = deg;
                 sm.src[p2] = v;
                 sm.payload[p2] = pay;
@@ -260,8 +266,14 @@ __device__ __forceinline__ void micro_edges(const PageSet& ps, Op& op, const uin
     for (int q = 0; q < kEdgesPerThread; ++q) {
         const uint32_t k = k0 + q * stride;
         valid[q] = k < deg;
-        dst[q] = valid[q] ? ld_stream_u32(adj + k, pol) : 0u;
-        w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_u32(adj + deg + k, pol) : 0u;
+        if (Op::kWeighted) {
+            const uint2 pr = valid[q] ? ld_stream_v2(adj + 2 * k, pol) : make_uint2(0u, 0u);
+            dst[q] = pr.x;
+            w[q] = pr.y;
+        } else {
+            dst[q] = valid[q] ? ld_stream_u32(adj + k, pol) : 0u;
+            w[q] = 0u;
+        }
         pl[q] = pay;
         src[q] = v;
     }
@@ -275,12 +287,12 @@ __device__ void expand_sp_micro(const PageSet& ps, Op& op, const uint8_t* data, 
                                 uint32_t nslots, uint64_t pol) {
     const uint32_t* words = reinterpret_cast<const uint32_t*>(data);
     const uint32_t start = ld32(end - kSpFooter - kSlotBytes);
-    constexpr uint32_t wsh = Op::kWeighted ? 1 : 0;
+    constexpr uint32_t wsh = Op::kWeighted ? 1 : 0, hdr = rec_hdr_words(Op::kWeighted);
     bool vertex = kMicro == kMicroVertex;
     if (kMicro == kMicroHybrid) {              // page density from its last record's end
         const uint32_t lo = ld32(end - kSpFooter - kSlotBytes * (uint64_t)nslots + 4);
-        const uint32_t used = lo / 4 + 1 + (ld32(data + lo) << wsh);     // record words
-        const uint32_t nedges = (used - nslots) >> wsh;
+        const uint32_t used = lo / 4 + hdr + (ld32(data + lo) << wsh);     // record words
+        const uint32_t nedges = (used - hdr * nslots) >> wsh;
         vertex = nedges < ps.hybrid_deg * nslots;
     }
     if (vertex) {
@@ -290,7 +302,7 @@ __device__ void expand_sp_micro(const PageSet& ps, Op& op, const uint8_t* data, 
             const uint32_t off = ld_stream_u32(end - kSpFooter - kSlotBytes * (uint64_t)(u + 1) + 4, pol);
             const uint32_t deg = ld_stream_u32(data + off, pol);
             const uint32_t pay = op.payload(v, deg);
-            const uint32_t* adj = words + off / 4 + 1;
+            const uint32_t* adj = words + off / 4 + hdr;
             for (uint32_t k0 = 0; k0 < deg; k0 += kEdgesPerThread) micro_edges(ps, op, adj, deg, k0, 1, pay, v, pol);
         }
     } else {
@@ -302,7 +314,7 @@ __device__ void expand_sp_micro(const PageSet& ps, Op& op, const uint8_t* data, 
             const uint32_t deg = ld_stream_u32(data + off, pol);
             uint32_t pay = lane == 0 ? op.payload(v, deg) : 0u;
             pay = __shfl_sync(0xFFFFFFFFu, pay, 0);
-            const uint32_t* adj = words + off / 4 + 1;
+            const uint32_t* adj = words + off / 4 + hdr;
             for (uint32_t k0 = lane; k0 < deg; k0 += 32 * kEdgesPerThread) micro_edges(ps, op, adj, deg, k0, 32, pay, v, pol);
         }
     }
@@ -380,15 +392,12 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
                 j0 += ns;
                 continue;
             }
-            // Weighted records (sz, adj[sz], w[sz]): a word is an entry iff it lies in
-            // the first sz words after its owner's header.  The lane's words have owners
-            // jb + c; the record bounds of jb and jb + 1 (all but a few lanes) are loaded
-            // once per lane, others on demand.
+            // Weighted records (sz, 0, (adj, w) pairs), 8-byte aligned: a word is an entry iff
+            // it lies past its owner's 2-word header at an even distance from the record start,
+            // and its weight is the next word of the same 16-byte group (k = 0 or 2 only).
             const uint32_t bpos0 = (4 * lane) & 31;
             const uint32_t nb = (mword >> bpos0) & 0xFu;
             const int jb = j0 + (int)(before + __popc(mword & ((1u << bpos0) - 1u)));
-            const uint32_t oA = jb >= 0 ? sm.soff[jb] : 0u;   // jb = -1: only words before W0 have c = 0
-            const uint32_t oB = sm.soff[jb + 1], oC = sm.soff[jb + 2];
             uint32_t c = 0;
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
@@ -396,15 +405,9 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
                 const uint32_t st = (nb >> k) & 1u;
                 c += st;
                 const int j = jb + (int)c;
-                bool ok = !st && w >= W0 && w < W1;
-                uint32_t dj = 0;
-                if (ok) {                              // adjacency words only, not the weights after them
-                    const uint32_t o = c == 0 ? oA : c == 1 ? oB : sm.soff[j];
-                    const uint32_t oe = c == 0 ? oB : c == 1 ? oC : sm.soff[j + 1];
-                    dj = (oe - o - 1) >> wsh;
-                    ok = w - o <= dj && sm.sel[j];
-                }
-                wt[k] = (Op::kReadWeights && ok) ? ld_stream_l1_u32(words + w + dj, pol) : 0u;
+                // (record starts are even words, so w - start is even iff k is even)
+                const bool ok = !st && !(k & 1) && w >= W0 && w < W1 && w - sm.soff[j] >= 2 && sm.sel[j];
+                wt[k] = ok ? word_of(vv[u], k + 1) : 0u;
                 valid[k] = ok;
                 dst[k] = decode_entry_t<kVid32>(ps, word_of(vv[u], k));
                 pl[k] = ok ? sm.paytile[j] : 0u;
@@ -448,7 +451,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             const uint32_t klo = (uint32_t)((uint64_t)len * sub / S), khi = (uint32_t)((uint64_t)len * (sub + 1) / S);
             uint32_t payload = 0;
             if (khi > klo && op.select_lp(vid, total, khi - klo, payload)) {
-                const uint32_t* adj = words + 1;
+                const uint32_t* adj = words + rec_hdr_words(Op::kWeighted);
                 for (uint32_t k0 = klo + tid; k0 < khi; k0 += kThreads * kEdgesPerThread) {
                     uint32_t dst[kEdgesPerThread], w[kEdgesPerThread], pl[kEdgesPerThread], src[kEdgesPerThread];
                     bool valid[kEdgesPerThread];
@@ -456,8 +459,14 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     for (int q = 0; q < kEdgesPerThread; ++q) {
                         const uint32_t k = k0 + q * kThreads;
                         valid[q] = k < khi;
-                        dst[q] = valid[q] ? ld_stream_u32(adj + k, pol) : 0u;
-                        w[q] = (Op::kReadWeights && valid[q]) ? ld_stream_u32(adj + len + k, pol) : 0u;
+                        if (Op::kWeighted) {
+                            const uint2 pr = valid[q] ? ld_stream_v2(adj + 2 * k, pol) : make_uint2(0u, 0u);
+                            dst[q] = pr.x;
+                            w[q] = pr.y;
+                        } else {
+                            dst[q] = valid[q] ? ld_stream_u32(adj + k, pol) : 0u;
+                            w[q] = 0u;
+                        }
                         pl[q] = payload;
                         src[q] = vid;
                     }
@@ -516,12 +525,13 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     sm.soff[tid] = o >> 2;
                     if ((uint32_t)tid == nv - 1) {
                         if (t0 + nv < nslots) sm.soff[nv] = ld_stream_u32(slot - kSlotBytes + 4, pol) >> 2;
-                        else sm.soff[nv] = (o >> 2) + 1 + (ld32(data + o) << (Op::kWeighted ? 1 : 0));
+                        else sm.soff[nv] = (o >> 2) + rec_hdr_words(Op::kWeighted) + (ld32(data + o) << (Op::kWeighted ? 1 : 0));
                     }
                 }
                 if (!__syncthreads_or(sel)) continue;   // (also publishes soff)
                 uint32_t deg = 0;
-                if ((uint32_t)tid < nv) deg = (sm.soff[tid + 1] - sm.soff[tid] - 1) >> (Op::kWeighted ? 1 : 0);
+                if ((uint32_t)tid < nv)
+                    deg = (sm.soff[tid + 1] - sm.soff[tid] - rec_hdr_words(Op::kWeighted)) >> (Op::kWeighted ? 1 : 0);
                 const uint32_t pay = sel ? op.payload(v, deg) : 0u;
                 if ((uint32_t)tid < nv) {               // published by tile_scan's barriers
                     sm.sel[tid] = sel ? 1 : 0;
@@ -550,7 +560,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 }
                 // sparse tile: compacted selected vertices, edge-parallel gather
                 if (item) {
-                    sm.off[pos] = sm.soff[tid] + 1;
+                    sm.off[pos] = sm.soff[tid] + rec_hdr_words(Op::kWeighted);
                     sm.deg[pos] = deg;
                     sm.src[pos] = v;
                     sm.payload[pos] = pay;

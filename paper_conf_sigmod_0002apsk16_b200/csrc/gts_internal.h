@@ -26,6 +26,11 @@ constexpr uint32_t kSpFooter = 8;    // u32 nslots, u32 kind
 constexpr uint32_t kLpFooter = 16;   // u32 total_deg, u32 chunk_idx, u32 nslots, u32 kind
 constexpr uint32_t kSlotBytes = 8;   // u32 vid, u32 off
 constexpr uint32_t kDefaultPageBytes = 1u << 20;
+// Record words (include/gts.h "Page layout"): unweighted u32 sz, u32 adj[sz];
+// weighted u32 sz, u32 0, then sz (u32 adj, u32 w) pairs, 8-byte aligned, so an
+// edge's neighbour and weight are one 8-byte load.
+GTS_HD constexpr uint32_t rec_hdr_words(bool weighted) { return weighted ? 2u : 1u; }
+GTS_HD constexpr uint32_t rec_edge_words(bool weighted) { return weighted ? 2u : 1u; }
 
 // ---- hot-destination table (PageRank CTA pre-aggregation, DESIGN.md K-PR) ----
 // Bucketed two-choice hash table of VIDs; a key lives in bucket h1 if h1 had a

@@ -37,6 +37,13 @@ __device__ __forceinline__ uint32_t ld_stream_l1_u32(const void* p, uint64_t pol
     return r;
 }
 
+// L1-allocating 8-byte variant (weighted (neighbour, weight) pairs of a gathered record)
+__device__ __forceinline__ uint2 ld_stream_l1_v2(const void* p, uint64_t pol) {
+    uint2 r;
+    asm volatile("ld.global.nc.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));
+    return r;
+}
+
 __device__ __forceinline__ uint2 ld_stream_v2(const void* p, uint64_t pol) {
     uint2 r;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"

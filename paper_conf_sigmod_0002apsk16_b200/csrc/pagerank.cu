@@ -181,7 +181,9 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             const uint32_t total = ld32(end - 16);
             const uint32_t len = ld32(data);
             const float c = d * __ldg(x + vid) / (float)total;
-            const uint32_t wend = 1 + len, qend = (wend + 3) >> 2;
+            // entries: words [hdr, hdr + len) (unweighted) or the even words of [2, 2 + 2 len)
+            constexpr uint32_t hdr = rec_hdr_words(kWeighted);
+            const uint32_t wend = hdr + (len << wshift), qend = (wend + 3) >> 2;
             for (uint32_t qb = tid; qb < qend; qb += T * kPrUnroll) {
                 uint4 v[kPrUnroll];
 #pragma unroll
@@ -196,7 +198,8 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
 #pragma unroll
                     for (int k = 0; k < 4; ++k) {
                         const uint32_t w = 4 * q + k;
-                        if (w >= 1 && w < wend) em.edge(pr_decode<kVid>(word_of(v[u], k), ps.rvt_start), c);
+                        if (w >= hdr && w < wend && !(kWeighted && (k & 1)))
+                            em.edge(pr_decode<kVid>(word_of(v[u], k), ps.rvt_start), c);
                     }
                 }
             }
@@ -235,7 +238,8 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                         sm.off[i] = r_off[k] >> 2;
                         if (i == nv - 1)              // the page's last record ends after its own length
                             sm.off[nv] = r_nxt != 0xFFFFFFFFu ? r_nxt >> 2
-                                                              : (r_off[k] >> 2) + 1 + (ld32(data + r_off[k]) << wshift);
+                                                              : (r_off[k] >> 2) + rec_hdr_words(kWeighted) +
+                                                                    (ld32(data + r_off[k]) << wshift);
                     }
                 }
                 __syncthreads();
@@ -243,7 +247,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                 for (int k = 0; k < VPT; ++k) {
                     const uint32_t i = (uint32_t)tid + (uint32_t)k * T;
                     if (i < nv) {
-                        const uint32_t deg = (sm.off[i + 1] - sm.off[i] - 1) >> wshift;
+                        const uint32_t deg = (sm.off[i + 1] - sm.off[i] - rec_hdr_words(kWeighted)) >> wshift;
                         float c = 0.f;
                         // dangling mass (R3); a routed rank counts only its own WA range (under
                         // S_BCAST every rank sees every page)
@@ -289,8 +293,10 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                                 cur = nxt;
                                 nxt = sm.off[j + 1];
                             }
-                            const uint32_t rel = w - cur;     // 0 = ADJLIST_SZ word; > deg = weight words
-                            if (rel == 0 || rel > ((nxt - cur - 1) >> wshift)) continue;
+                            // entries: rel >= 1 (unweighted); weighted records (sz, 0, (adj, w) pairs):
+                            // the even rel >= 2 (records are 8-byte aligned)
+                            const uint32_t rel = w - cur;
+                            if (kWeighted ? (rel < 2 || (rel & 1)) : rel == 0) continue;
                             em.edge(pr_decode<kVid>(word_of(v[u], k), ps.rvt_start), sm.c[j]);
                         }
                     }

@@ -113,7 +113,8 @@ struct WccOp {
 // visits every edge (the result is exact); the sample only makes its edges
 // cheap (one gather instead of two finds).
 __global__ void __launch_bounds__(kThreads, 2)
-wcc_sample_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t ks) {
+wcc_sample_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t ks, int weighted) {
+    const uint32_t hdr = rec_hdr_words(weighted != 0), ew = rec_edge_words(weighted != 0);
     __shared__ uint32_t s_item;
     const int tid = threadIdx.x;
     const uint64_t pol = policy_evict_first();
@@ -134,7 +135,7 @@ wcc_sample_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t ks)
             const uint32_t chunk = ld32(end - 12);
             const uint32_t len = ld32(data);
             if (chunk == 0 && (uint32_t)tid < min(ks, len)) {
-                const uint32_t v = decode_entry(ps, ld_stream_u32(words + 1 + tid, pol));
+                const uint32_t v = decode_entry(ps, ld_stream_u32(words + hdr + ew * tid, pol));
                 if (v != vid) uf_hook(parent, vid, v);
             }
         } else {
@@ -145,7 +146,7 @@ wcc_sample_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t ks)
                 const uint32_t deg = ld_stream_u32(words + off, pol);
                 const uint32_t kk = min(ks, deg);
                 for (uint32_t k = 0; k < kk; ++k) {
-                    const uint32_t v = decode_entry(ps, ld_stream_u32(words + off + 1 + k, pol));
+                    const uint32_t v = decode_entry(ps, ld_stream_u32(words + off + hdr + ew * k, pol));
                     if (v != start + u) uf_hook(parent, start + u, v);
                 }
             }
@@ -306,7 +307,7 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
         ps.rvt_start = c->dg.rvt_start;
         int sg = 0;
         GTS_TRY(sms_grid(c, (const void*)wcc_sample_kernel, kThreads, 0, &sg));
-        wcc_sample_kernel<<<sg, kThreads, 0, s>>>(ps, label[0], ctr[0], ks);
+        wcc_sample_kernel<<<sg, kThreads, 0, s>>>(ps, label[0], ctr[0], ks, g->weighted ? 1 : 0);
         wcc_finalize_kernel<<<eg, 256, 0, s>>>(label[0], n);
         GTS_TRY(c->buf(kBufWccGiant, (n + 31) / 32 * 4 + 16, (void**)&gbm));
         wcc_giant_kernel<<<eg, 256, 0, s>>>(label[0], n, gbm, gbm + (n + 31) / 32);

@@ -40,7 +40,7 @@ def _my_part(G, oracle, gr, g, pb, strategy, world, rank):
     d = gr.directory()
     pages = gr.pages().reshape(-1, pb)
     mine = np.nonzero(owner == rank)[0]
-    rp, col, w = oracle.decode_pages(pages[mine].reshape(-1), pb, g.n, g.m, weighted=g.weights is not None)
+    rp, col, w = oracle.decode_pages(pages[mine].reshape(-1), pb, g.n, g.m, weighted=bool(gr.stats()["weighted"]))
     verts = np.zeros(g.n, dtype=bool)          # vertices whose records live in my pages
     for p in mine:
         verts[d["start_vid"][p]:d["start_vid"][p] + d["nslots"][p]] = True

@@ -30,6 +30,14 @@ gr = G.gts_build_pages(g.row_ptr, g.col, order=True)
 grw = G.gts_build_pages(g.row_ptr, g.col, inputs.edge_weights(g), order=True) if "sssp" in algos else None
 ctx = G.gts_context_create(0)
 import torch  # noqa: E402
+try:   # the persisting-L2 limits the access-policy windows are clipped to
+    from cuda.bindings import runtime as rt
+    _, pmax = rt.cudaDeviceGetAttribute(rt.cudaDeviceAttr.cudaDevAttrMaxPersistingL2CacheSize, 0)
+    _, wmax = rt.cudaDeviceGetAttribute(rt.cudaDeviceAttr.cudaDevAttrMaxAccessPolicyWindowSize, 0)
+    print(json.dumps({"l2_bytes": torch.cuda.get_device_properties(0).L2_cache_size,
+                      "persisting_l2_max_bytes": pmax, "access_policy_window_max_bytes": wmax}), flush=True)
+except Exception as e:  # pragma: no cover
+    print(json.dumps({"l2_probe_error": repr(e)}), flush=True)
 n = g.n
 dev_u = torch.empty(n, dtype=torch.int32, device="cuda")
 dev_f = torch.empty(n, dtype=torch.float32, device="cuda")
