@@ -461,10 +461,22 @@ __global__ void pr_finish_kernel(float* x, float* acc, uint64_t n, uint64_t lo, 
     float4* x4 = reinterpret_cast<float4*>(x + lo + head);
     float4* acc4 = reinterpret_cast<float4*>(acc + lo + head);
     const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
-    for (uint64_t i = t0; i < nvec; i += stride) {
-        const float4 a = acc4[i];
-        x4[i] = make_float4(base + a.x, base + a.y, base + a.z, base + a.w);
-        acc4[i] = z;
+    // four float4 loads in flight per thread before their stores (one in flight measured
+    // 0.52 ms per RMAT-27 iteration, 48% of the copy peak)
+    constexpr int U = 4;
+    for (uint64_t i0 = t0; i0 < nvec; i0 += U * stride) {
+        float4 a[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if (i0 + u * stride < nvec) a[u] = acc4[i0 + u * stride];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint64_t i = i0 + u * stride;
+            if (i < nvec) {
+                x4[i] = make_float4(base + a[u].x, base + a[u].y, base + a[u].z, base + a[u].w);
+                acc4[i] = z;
+            }
+        }
     }
     const uint64_t tail0 = head + 4 * nvec;
     for (uint64_t k = t0; k < head + (len - tail0); k += stride) {     // head [0, head) and tail [tail0, len)
