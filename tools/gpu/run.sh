@@ -30,7 +30,7 @@ case "$what" in
     echo "ncu rc=$?"; tail -3 $O/ncu.log ;;
   sanitize)
     tool=${1:-memcheck}
-    timeout 2400 compute-sanitizer --tool $tool --print-limit 50 python tools/sanitize_run.py > $O/sanitize_$tool.log 2>&1
+    timeout ${SAN_TIMEOUT:-2400} compute-sanitizer --tool $tool --print-limit 50 python tools/sanitize_run.py > $O/sanitize_$tool.log 2>&1
     echo "sanitizer rc=$?"; tail -8 $O/sanitize_$tool.log ;;
   py)
     s=$1; shift

@@ -22,6 +22,8 @@ ap.add_argument("--scale", type=int, default=27)
 ap.add_argument("--reps", type=int, default=3)
 ap.add_argument("--algos", default="pr,bfs,sssp,wcc")
 ap.add_argument("--tag", default="")
+ap.add_argument("--variants", default="",
+                help='A/B of development switches read by libgts at call time: "name:ENV=V,ENV2=W;name2:..."')
 a = ap.parse_args()
 
 g = inputs.rmat(a.scale)
@@ -41,22 +43,31 @@ except Exception as e:  # pragma: no cover
 n = g.n
 dev_u = torch.empty(n, dtype=torch.int32, device="cuda")
 dev_f = torch.empty(n, dtype=torch.float32, device="cuda")
-for al in algos:
-    ks, cs, st = [], [], None
-    for _ in range(a.reps + 1):
-        if al == "pr":
-            _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=dev_f, timing=True)
-        elif al == "bfs":
-            _, st = G.gts_bfs(ctx, gr, 0, out=dev_u, timing=True)
-        elif al == "sssp":
-            _, st = G.gts_sssp(ctx, grw, 0, out=dev_u, timing=True)
-        else:
-            _, st = G.gts_wcc(ctx, gr, out=dev_u, timing=True)
-        ks.append(st["main_kernel_s"])
-        cs.append(st["wall_s"])
-    ks, cs = sorted(ks[1:]), sorted(cs[1:])
-    per = 10 if al == "pr" else 1
-    print(json.dumps({"tag": a.tag, "algo": al, "scale": a.scale, "main_kernel_ms": 1e3 * ks[len(ks) // 2] / per,
-                      "per": "iteration" if per == 10 else "call", "call_ms": 1e3 * cs[len(cs) // 2],
-                      "all_kernel_ms": [round(1e3 * k / per, 3) for k in ks], "edges": st["edges_traversed"],
-                      "levels": st["levels_or_iters"], "finish_ms": 1e3 * st["finish_s"] / per}), flush=True)
+variants = [v.partition(":") for v in a.variants.split(";")] if a.variants else [(a.tag, "", "")]
+for tag, _, envs in variants:
+    keys = []
+    for kv in filter(None, envs.split(",")):
+        k, v = kv.split("=")
+        os.environ[k] = v
+        keys.append(k)
+    for al in algos:
+        ks, cs, st = [], [], None
+        for _ in range(a.reps + 1):
+            if al == "pr":
+                _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=dev_f, timing=True)
+            elif al == "bfs":
+                _, st = G.gts_bfs(ctx, gr, 0, out=dev_u, timing=True)
+            elif al == "sssp":
+                _, st = G.gts_sssp(ctx, grw, 0, out=dev_u, timing=True)
+            else:
+                _, st = G.gts_wcc(ctx, gr, out=dev_u, timing=True)
+            ks.append(st["main_kernel_s"])
+            cs.append(st["wall_s"])
+        ks, cs = sorted(ks[1:]), sorted(cs[1:])
+        per = 10 if al == "pr" else 1
+        print(json.dumps({"tag": tag, "algo": al, "scale": a.scale, "main_kernel_ms": 1e3 * ks[len(ks) // 2] / per,
+                          "per": "iteration" if per == 10 else "call", "call_ms": 1e3 * cs[len(cs) // 2],
+                          "all_kernel_ms": [round(1e3 * k / per, 3) for k in ks], "edges": st["edges_traversed"],
+                          "levels": st["levels_or_iters"], "finish_ms": 1e3 * st["finish_s"] / per}), flush=True)
+    for k in keys:
+        del os.environ[k]
