@@ -67,10 +67,6 @@ struct TileSmem {
     uint32_t item;
     uint32_t pcount;                 // frontier vertices of the current page
     uint32_t list[kListWords * 32];  // sparse pages: compacted frontier vertices (slot indices)
-    // TMA staging of tile slot arrays (expand_pages<..., kTma = true>): the next active tile's
-    // slots (+ the one after it, for the last record's end) land here by cp.async.bulk
-    alignas(16) uint2 stage[2][kTile + 4];
-    alignas(8) uint64_t bar[2];
 };
 
 // Tile scan: frontier compaction by __ballot_sync/__popc (position of each
@@ -423,7 +419,7 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
     }
 }
 
-template <class Op, int kMicro = kMicroTile, bool kTma = false>
+template <class Op, int kMicro = kMicroTile>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
     const uint32_t npages = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
     // work items per page: ps.split, or 0 = automatic: slice LPs when the set has fewer
@@ -433,14 +429,6 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
     const uint32_t count = npages * S;
     const int tid = threadIdx.x;
     const uint64_t pol = policy_evict_first();
-    uint32_t ph[2] = {0u, 0u};               // kTma: phase of each staging barrier
-    if (kTma) {
-        if (tid == 0) {
-            mbar_init(&sm.bar[0], 1);
-            mbar_init(&sm.bar[1], 1);
-        }
-        __syncthreads();
-    }
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
         __syncthreads();
@@ -528,56 +516,18 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 while (t < ntiles && !active(t)) ++t;     // uniform: tiles without a frontier vertex cost nothing
                 return t;
             };
-            // kTma: slot bytes of tile t (slots t0 .. last, 16-byte aligned span; slots grow
-            // down from the page end, so the span starts at the last slot)
-            auto span = [&](uint32_t t, const uint8_t*& alo, uint32_t& bytes) {
-                const uint32_t t0 = t * kTile, nv = min((uint32_t)kTile, nslots - t0);
-                const uint32_t last = t0 + nv < nslots ? t0 + nv : t0 + nv - 1;
-                const uintptr_t lo = (uintptr_t)(end - kSpFooter - kSlotBytes * (uint64_t)(last + 1));
-                const uintptr_t hi = (uintptr_t)(end - kSpFooter - kSlotBytes * (uint64_t)t0);
-                alo = reinterpret_cast<const uint8_t*>(lo & ~(uintptr_t)15);
-                bytes = (uint32_t)(((hi + 15) & ~(uintptr_t)15) - (lo & ~(uintptr_t)15));
-            };
-            auto issue = [&](uint32_t t, int b) {         // one thread: prefetch tile t's slots into buffer b
-                const uint8_t* alo;
-                uint32_t bytes;
-                span(t, alo, bytes);
-                fence_proxy_async_smem();                 // earlier reads of the buffer before the async write
-                bulk_load(sm.stage[b], alo, bytes, &sm.bar[b]);
-            };
-            int b = 0;
-            const uint32_t tfirst = next_active(0);
-            if (kTma && tid == 0 && tfirst < ntiles) issue(tfirst, 0);
-            for (uint32_t ti = tfirst; ti < ntiles; ti = next_active(ti + 1), b ^= 1) {
-                if (kTma && tid == 0) {           // buffer b ^ 1 was last read before a barrier of the previous tile
-                    const uint32_t tn = next_active(ti + 1);
-                    if (tn < ntiles) issue(tn, b ^ 1);
-                }
+            // (Staging the next active tile's slot array into shared memory with a 1D TMA copy
+            // -- cp.async.bulk + mbarrier, double-buffered, one elected thread -- measured
+            // slower on RMAT-27: BFS 7.41 vs 7.36 ms, WCC 12.84 vs 12.64 ms; the slot loads are
+            // not what these kernels wait on.)
+            for (uint32_t ti = next_active(0); ti < ntiles; ti = next_active(ti + 1)) {
                 const uint32_t t0 = ti * kTile;
                 const uint32_t nv = min((uint32_t)kTile, nslots - t0);
                 const uint32_t v = start + t0 + tid;
                 const bool sel = (uint32_t)tid < nv && op.select(v);
                 // record offsets of the whole tile; the degree of a record is the distance to
                 // the next record (the last one reads its header)
-                if (kTma) {
-                    mbar_wait(&sm.bar[b], ph[b]);
-                    ph[b] ^= 1u;
-                    const uint8_t* alo;
-                    uint32_t bytes;
-                    span(ti, alo, bytes);
-                    const uint8_t* st = reinterpret_cast<const uint8_t*>(sm.stage[b]);
-                    auto staged_off = [&](uint32_t i) {   // OFF of slot i of the page
-                        return *reinterpret_cast<const uint32_t*>(st + (end - kSpFooter - kSlotBytes * (uint64_t)(i + 1) + 4 - alo));
-                    };
-                    if ((uint32_t)tid < nv) {
-                        const uint32_t o = staged_off(t0 + tid);
-                        sm.soff[tid] = o >> 2;
-                        if ((uint32_t)tid == nv - 1) {
-                            if (t0 + nv < nslots) sm.soff[nv] = staged_off(t0 + nv) >> 2;
-                            else sm.soff[nv] = (o >> 2) + rec_hdr_words(Op::kWeighted) + (ld32(data + o) << (Op::kWeighted ? 1 : 0));
-                        }
-                    }
-                } else if ((uint32_t)tid < nv) {         // coalesced slot reads
+                if ((uint32_t)tid < nv) {                // coalesced slot reads
                     const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + tid + 1);
                     const uint32_t o = ld_stream_u32(slot + 4, pol);
                     sm.soff[tid] = o >> 2;
@@ -603,7 +553,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 // records hold 2 words per edge, so there a tile is dense only when nearly
                 // every vertex is selected -- measured the better choice for SSSP (RMAT-27
                 // 35.7 ms vs 42.8 ms when the selected words are counted instead)
-                const bool dense = 2 * total >= W1 - W0;
+                const bool dense = (Op::kWeighted && ps.wdense) ? 4 * total >= W1 - W0 : 2 * total >= W1 - W0;
                 if (dense) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
                     // 128-word windows; owners from record-start masks (no binary search;

@@ -140,7 +140,7 @@ __device__ __forceinline__ uint32_t pr_decode(uint32_t e, const uint32_t* rvt) {
 // (records are packed in VID order from offset 0), streamed with 16-byte
 // evict_first loads, kPrUnroll in flight per thread; the owner of each 4-word
 // group is found by a binary search over the tile's record offsets.
-template <bool kWeighted, int kMode, int T, int kMinBlocks, uint32_t H, int VPT, bool kVid, bool kWW = false>
+template <bool kWeighted, int kMode, int T, int kMinBlocks, uint32_t H, int VPT, bool kVid>
 __global__ void __launch_bounds__(T, kMinBlocks)
 pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__ hot_keys,
                   float d, double* dang_out, uint32_t* work_ctr, uint32_t n_hot, const RouteParams rp) {
@@ -259,67 +259,12 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                 }
                 if (t0 + TV < nslots) prefetch(t0 + TV);
                 __syncthreads();
-                if constexpr (kWW) {
-                // Warp windows: the tile's record region is cut into 128-word windows (one
-                // 16-byte load per lane), each warp streams a contiguous run of them, and the
-                // owner of a word is j0 + #(record starts up to it) from a 128-bit record-start
-                // mask (win_mask: four redux.sync.or over 32 candidate offsets) -- one binary
-                // search per warp per tile instead of one per 16 bytes.
-                constexpr int kW = T / 32;
-                constexpr int kWU = 2;                       // windows in flight per warp
-                const int lane = tid & 31, warp = tid >> 5;
-                const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
-                const uint32_t wbase = W0 & ~3u;
-                const uint32_t nwin = (W1 - wbase + 127) >> 7;
-                const uint32_t per = (nwin + kW - 1) / kW;
-                const uint32_t wa = min(nwin, warp * per), wb = min(nwin, wa + per);
-                if (wa < wb) {
-                    const uint32_t base = wbase + (wa << 7);
-                    int lo = -1, hi = (int)nv;               // off[lo] < base <= off[hi]
-                    while (hi - lo > 1) {
-                        const int mid = (lo + hi) >> 1;
-                        if (sm.off[mid] < base) lo = mid; else hi = mid;
-                    }
-                    int j0 = lo;
-                    for (uint32_t wi = wa; wi < wb; wi += kWU) {
-                        uint4 v[kWU];
-#pragma unroll
-                        for (int u = 0; u < kWU; ++u) {
-                            const uint32_t q = ((wbase + ((wi + u) << 7)) >> 2) + lane;
-                            v[u] = make_uint4(0u, 0u, 0u, 0u);
-                            if (wi + u < wb && 4 * q < W1) v[u] = ld_stream_v4(q4 + q, pol);
-                        }
-#pragma unroll
-                        for (int u = 0; u < kWU; ++u) {
-                            if (wi + u >= wb) break;
-                            const uint32_t bw = wbase + ((wi + u) << 7);
-                            const uint32_t q = (bw >> 2) + lane;
-                            int ns;
-                            const WinMask wm = win_mask(sm.off, j0, nv, bw, ns);
-                            const uint32_t mw = lane >> 3;
-                            uint32_t before = 0;
-#pragma unroll
-                            for (int k = 0; k < 4; ++k) before += (uint32_t)k < mw ? __popc(wm.m[k]) : 0u;
-                            const uint32_t mword = mw == 0 ? wm.m[0] : mw == 1 ? wm.m[1] : mw == 2 ? wm.m[2] : wm.m[3];
-#pragma unroll
-                            for (int k = 0; k < 4; ++k) {
-                                const uint32_t w = 4 * q + k;
-                                const uint32_t bpos = (4 * lane + k) & 31;
-                                if (w < W0 || w >= W1 || ((mword >> bpos) & 1u)) continue;   // record starts
-                                const int j = j0 + (int)(before + __popc(mword & ((2u << bpos) - 1u)));
-                                if (kWeighted && (k & 1)) continue;   // the pad and weight words (odd)
-                                em.edge(pr_decode<kVid>(word_of(v[u], k), ps.rvt_start), sm.c[j]);
-                            }
-                            j0 += ns;
-                        }
-                    }
-                }
-                } else {
                 // the tile's record region, 16-byte evict_first loads, kPrUnroll in flight per
                 // thread (coalesced: lane-consecutive groups); the owner of each 16-byte group by
-                // a binary search over the tile's offsets, then record by record.  (Giving each
-                // thread 4 consecutive groups -- one search per 16 words -- measured slower on
-                // RMAT-27: 14.4 vs 11.5 ms, the uncoalesced loads cost more than the searches.)
+                // a binary search over the tile's offsets, then record by record.  (Measured on
+                // RMAT-27 and rejected: 4 consecutive groups per thread with one search per 16
+                // words, 14.4 vs 11.5 ms -- uncoalesced loads; warp windows with record-start
+                // masks instead of the searches, 10.82 vs 10.78 ms.)
                 const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
                 const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
                 for (uint32_t qb = qbeg + tid; qb < qend; qb += T * kPrUnroll) {
@@ -356,7 +301,6 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                             em.edge(pr_decode<kVid>(word_of(v[u], k), ps.rvt_start), sm.c[j]);
                         }
                     }
-                }
                 }
                 __syncthreads();
             }
@@ -587,11 +531,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
             if (m == kRoute)
                 kern = g->weighted ? GTS_PRK(true, kRoute, 1024, 1, kHotDenseBig, kPrVpt)
                                    : GTS_PRK(false, kRoute, 1024, 1, kHotDenseBig, kPrVpt);
-            else if (getenv("GTS_DEV_PRWW") && atoi(getenv("GTS_DEV_PRWW")) > 0)
-                kern = g->weighted ? (vid ? (const void*)pr_scatter_kernel<true, kDense, 1024, 1, kHotDenseBig, kPrVpt, true, true>
-                                          : (const void*)pr_scatter_kernel<true, kDense, 1024, 1, kHotDenseBig, kPrVpt, false, true>)
-                                   : (vid ? (const void*)pr_scatter_kernel<false, kDense, 1024, 1, kHotDenseBig, kPrVpt, true, true>
-                                          : (const void*)pr_scatter_kernel<false, kDense, 1024, 1, kHotDenseBig, kPrVpt, false, true>);
             else
                 kern = g->weighted ? GTS_PRK(true, kDense, 1024, 1, kHotDenseBig, kPrVpt)
                                    : GTS_PRK(false, kDense, 1024, 1, kHotDenseBig, kPrVpt);

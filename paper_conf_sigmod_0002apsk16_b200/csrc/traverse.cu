@@ -147,7 +147,7 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 
 // -------------------------------------------------------------- kernels ---
 
-template <bool W, int M = kMicroTile, int MB = 2, bool TMA = false>
+template <bool W, int M = kMicroTile, int MB = 2>
 __global__ void __launch_bounds__(kThreads, MB)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
                   uint32_t* work_ctr, unsigned long long* edges_out, const unsigned int* vprefix_words,
@@ -157,7 +157,7 @@ bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visite
     // so levels can be enqueued without a host round trip)
     const uint64_t vw = min((uint64_t)*vprefix_words, (n + 31) / 32);
     BfsOp<W> op{cur, visited, next, 0ull, (uint32_t)min(vw * 32, n)};
-    expand_pages<BfsOp<W>, M, TMA>(ps, op, sm, work_ctr);
+    expand_pages<BfsOp<W>, M>(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
 
@@ -548,8 +548,6 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     // covered by the other two (RMAT-27 BFS kernels 10.25 -> 9.26 ms against two)
     if (micro == kMicroTile)
         bfs_kern = g->weighted ? bfs_expand_kernel<true, kMicroTile, 3> : bfs_expand_kernel<false, kMicroTile, 3>;
-    if (micro == kMicroTile && getenv("GTS_DEV_TMA") && atoi(getenv("GTS_DEV_TMA")) > 0)   // (temporary A/B)
-        bfs_kern = g->weighted ? bfs_expand_kernel<true, kMicroTile, 3, true> : bfs_expand_kernel<false, kMicroTile, 3, true>;
     const uint32_t hybrid_deg = rc.hybrid_deg ? rc.hybrid_deg : 8u;
     // two 512-thread CTAs per SM for the SSSP expansion (three measured 35.7 vs 35.1 ms on
     // RMAT-27: the weighted walk spills at 40 registers)
@@ -620,6 +618,7 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
                                 // few pages in this level (e.g. the source hub's LPs): slice LPs so
                                 // every CTA gets work, decided on the device
                                 p2.split = 0u;
+                                p2.wdense = getenv("GTS_DEV_WDENSE") ? (uint32_t)atoi(getenv("GTS_DEV_WDENSE")) : 0u;
                                 const int gl = std::min(grid, cap);
                                 if (algo == kBFS) {
                                     bfs_kern<<<gl, kThreads, 0, s>>>(

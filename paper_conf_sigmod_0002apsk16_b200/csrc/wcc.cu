@@ -154,13 +154,13 @@ wcc_sample_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t ks,
     }
 }
 
-template <bool W, int MB = 2, bool TMA = false>
+template <bool W, int MB = 2>
 __global__ void __launch_bounds__(kThreads, MB)
 wcc_sweep_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t* changed, const uint32_t* gbm,
                  const uint32_t* rstar) {
     __shared__ TileSmem sm;
     WccOp<W> op{parent, false, gbm, gbm ? __ldg(rstar) : 0u};
-    expand_pages<WccOp<W>, kMicroTile, TMA>(ps, op, sm, work_ctr);
+    expand_pages(ps, op, sm, work_ctr);
     if (__syncthreads_or(op.changed) && threadIdx.x == 0) *changed = 1u;
 }
 
@@ -271,8 +271,6 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     // three 512-thread CTAs per SM for the sweep (40 registers; RMAT-27 sweep 17.4 -> 14.6 ms
     // against two: the third CTA covers the per-tile barriers)
     auto sweep_k = g->weighted ? wcc_sweep_kernel<true, 3> : wcc_sweep_kernel<false, 3>;
-    if (getenv("GTS_DEV_TMA") && atoi(getenv("GTS_DEV_TMA")) > 0)   // (temporary A/B)
-        sweep_k = g->weighted ? wcc_sweep_kernel<true, 3, true> : wcc_sweep_kernel<false, 3, true>;
     int grid = 0;
     GTS_TRY(sms_grid(c, (const void*)sweep_k, kThreads, 0, &grid));
     uint64_t launches = L, main_launches = 0;
