@@ -53,6 +53,10 @@ struct BfsOp {
         if (threadIdx.x == 0) nedges += len;
         return true;
     }
+    // Rows are sorted, so a frontier vertex whose largest neighbour lies below the
+    // all-visited prefix discovers nothing: its record is dropped after one load
+    // (Alg 2 l.17 would test and skip each of its neighbours).
+    __device__ __forceinline__ bool skip_record(uint32_t last) const { return last < vprefix; }
     // Alg 2 lines 17-20: if LV[ADJ_VID] = NULL then discover it.  Exactly one
     // thread wins the visited bit and records the vertex in the next frontier.
     // The visited words of the whole edge group are loaded first (independent
@@ -618,7 +622,6 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
                                 // few pages in this level (e.g. the source hub's LPs): slice LPs so
                                 // every CTA gets work, decided on the device
                                 p2.split = 0u;
-                                p2.wdense = getenv("GTS_DEV_WDENSE") ? (uint32_t)atoi(getenv("GTS_DEV_WDENSE")) : 0u;
                                 const int gl = std::min(grid, cap);
                                 if (algo == kBFS) {
                                     bfs_kern<<<gl, kThreads, 0, s>>>(
