@@ -14,7 +14,6 @@
 #pragma once
 
 #include <cstdint>
-#include <type_traits>
 
 #include "memops.cuh"
 #include "runtime.h"
@@ -150,27 +149,6 @@ __device__ __forceinline__ WinMask win_mask(const uint32_t* off, int j0, uint32_
 // loaded back to back, so each thread has that many independent loads in
 // flight, and the op can issue its own per-edge loads (visited bits, dist,
 // labels) as a batch before acting on them.
-// Optional op hook: bool skip_record(uint32_t last_entry) -- a selected vertex whose
-// LAST (largest, rows are sorted) neighbour makes the whole record a no-op is
-// dropped after one load instead of expanding all its edges (BFS: every neighbour
-// below the all-visited prefix).  The op still counts the vertex in payload().
-template <class Op, class = void>
-struct has_skip_record : std::false_type {};
-template <class Op>
-struct has_skip_record<Op, std::void_t<decltype(std::declval<Op&>().skip_record(0u))>> : std::true_type {};
-
-template <class Op>
-__device__ __forceinline__ bool skip_by_last(const PageSet& ps, Op& op, const uint32_t* words, uint32_t rec_word,
-                                             uint32_t deg, uint64_t pol) {
-    if constexpr (has_skip_record<Op>::value) {
-        const uint32_t e = ld_stream_l1_u32(words + rec_word + rec_hdr_words(Op::kWeighted) +
-                                                (deg - 1) * rec_edge_words(Op::kWeighted), pol);
-        return op.skip_record(decode_entry(ps, e));
-    } else {
-        return false;
-    }
-}
-
 // Edge-parallel expansion of nf compacted items (sm.off/deg/src/payload/pre):
 // 4 consecutive edges per thread, one binary search per 4 edges.
 template <class Op>
@@ -251,8 +229,7 @@ __device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, cons
             }
             const uint32_t v = start + j;
             const uint32_t pay = sel ? op.payload(v, deg) : 0u;
-            // items with edges only (and not skipped by the op's last-neighbour test)
-            const bool item = sel && deg > 0 && !skip_by_last(ps, op, words, off / 4, deg, pol);
+            const bool item = sel && deg > 0;            // items with edges only
             uint32_t p2, nf, ex2, total;
             tile_scan(item, item ? deg : 0u, p2, nf, ex2, total, sm);
             if (item) {
@@ -564,13 +541,12 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 if ((uint32_t)tid < nv)
                     deg = (sm.soff[tid + 1] - sm.soff[tid] - rec_hdr_words(Op::kWeighted)) >> (Op::kWeighted ? 1 : 0);
                 const uint32_t pay = sel ? op.payload(v, deg) : 0u;
-                const bool keep = sel && !(deg > 0 && skip_by_last(ps, op, words, sm.soff[tid], deg, pol));
                 if ((uint32_t)tid < nv) {               // published by tile_scan's barriers
-                    sm.sel[tid] = keep ? 1 : 0;
+                    sm.sel[tid] = sel ? 1 : 0;
                     sm.paytile[tid] = pay;
                 }
                 uint32_t pos, nf, excl, total;
-                const bool item = keep && deg > 0;       // sparse tiles compact items with edges only
+                const bool item = sel && deg > 0;        // sparse tiles compact items with edges only
                 tile_scan(item, item ? deg : 0u, pos, nf, excl, total, sm);
                 const uint32_t W0 = sm.soff[0], W1 = sm.soff[nv];
                 // dense: the selected edges are >= half of the tile's record words.  Weighted
