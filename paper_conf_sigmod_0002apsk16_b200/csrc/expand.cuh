@@ -554,7 +554,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 // every vertex is selected -- measured the better choice for SSSP (RMAT-27
                 // 35.7 ms vs 42.8 ms when the selected words are counted instead; with the
                 // interleaved (adj, w) records 33.5 vs 35.3 ms)
-                const bool dense = 2 * total >= W1 - W0;
+                const bool dense = 8 * total >= ps.dense8 * (W1 - W0);
                 if (dense) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
                     // 128-word windows; owners from record-start masks (no binary search;

@@ -112,13 +112,10 @@ struct PrEmitter {
 
 constexpr int kPrUnroll = 4;            // 16-byte loads in flight per thread
 
-constexpr uint32_t kPrCells = 64;       // coarse index cells per scatter tile
-
 template <int T>
 struct PrSmem {
     uint32_t off[T + 1];                // page-relative word index of each record of the tile; off[nv] = end
     float c[T];                         // d * x_u / outdeg(u)
-    uint32_t cell[kPrCells + 1];        // cell[k] = last record starting at or before W0 + (k << cell_shift)
     uint32_t item;
 };
 
@@ -260,21 +257,6 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                         sm.c[i] = c;
                     }
                 }
-                // coarse index of the tile's record region: cells of 2^cs words, at most
-                // kPrCells of them; one binary search per cell here narrows every 16-byte
-                // group's owner search below to the records of one cell
-                const uint32_t W0c = sm.off[0], span = sm.off[nv] - W0c;
-                uint32_t cs = 0;
-                while ((span >> cs) >= kPrCells) ++cs;
-                if ((uint32_t)tid <= kPrCells) {
-                    const uint32_t pos = W0c + ((uint32_t)tid << cs);
-                    uint32_t lo = 0, hi = nv;               // largest j < nv with off[j] <= pos
-                    while (hi - lo > 1) {
-                        const uint32_t mid = (lo + hi) >> 1;
-                        if (sm.off[mid] <= pos) lo = mid; else hi = mid;
-                    }
-                    sm.cell[tid] = lo;
-                }
                 if (t0 + TV < nslots) prefetch(t0 + TV);
                 __syncthreads();
                 // the tile's record region, 16-byte evict_first loads, kPrUnroll in flight per
@@ -282,7 +264,9 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                 // a binary search over the tile's offsets, then record by record.  (Measured on
                 // RMAT-27 and rejected: 4 consecutive groups per thread with one search per 16
                 // words, 14.4 vs 11.5 ms -- uncoalesced loads; warp windows with record-start
-                // masks instead of the searches, 10.82 vs 10.78 ms.)
+                // masks instead of the searches, 10.82 vs 10.78 ms; a 64-cell coarse index per
+                // tile narrowing each search to one cell's records, 10.90 ms -- the searches'
+                // stalls are not what bounds the kernel, its L2 reductions are.)
                 const uint32_t W0 = sm.off[0], W1 = sm.off[nv];
                 const uint32_t qbeg = W0 >> 2, qend = (W1 + 3) >> 2;
                 for (uint32_t qb = qbeg + tid; qb < qend; qb += T * kPrUnroll) {
@@ -297,9 +281,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                         const uint32_t q = qb + u * T;
                         if (q >= qend) break;
                         const uint32_t w0 = 4 * q;
-                        // off[lo] <= max(w0, W0) < off[hi] within the group's coarse cell
-                        const uint32_t ce = w0 > W0 ? min((w0 - W0) >> cs, kPrCells - 1) : 0u;
-                        uint32_t lo = sm.cell[ce], hi = sm.cell[ce + 1] + 1;
+                        uint32_t lo = 0, hi = nv;               // off[lo] <= max(w0, W0) < off[hi]
                         while (hi - lo > 1) {
                             const uint32_t mid = (lo + hi) >> 1;
                             if (sm.off[mid] <= w0) lo = mid; else hi = mid;

@@ -621,6 +621,7 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
                                 // few pages in this level (e.g. the source hub's LPs): slice LPs so
                                 // every CTA gets work, decided on the device
                                 p2.split = 0u;
+                                if (getenv("GTS_DEV_DENSE8")) p2.dense8 = (uint32_t)atoi(getenv("GTS_DEV_DENSE8"));
                                 const int gl = std::min(grid, cap);
                                 if (algo == kBFS) {
                                     bfs_kern<<<gl, kThreads, 0, s>>>(
