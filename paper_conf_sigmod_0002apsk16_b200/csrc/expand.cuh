@@ -14,6 +14,7 @@
 #pragma once
 
 #include <cstdint>
+#include <type_traits>
 
 #include "memops.cuh"
 #include "runtime.h"
@@ -149,6 +150,17 @@ __device__ __forceinline__ WinMask win_mask(const uint32_t* off, int j0, uint32_
 // loaded back to back, so each thread has that many independent loads in
 // flight, and the op can issue its own per-edge loads (visited bits, dist,
 // labels) as a batch before acting on them.
+// Dense-tile threshold: a tile streams its whole record region when its selected
+// edges are at least kDense8 / 8 of the region's words (an op may set kDense8;
+// default 4 = half).  BFS uses 6: RMAT-27 BFS kernels 7.15-7.19 ms against 7.32
+// (4), 7.62 (3), 7.69 (2), 7.21 (7), 7.42 (8), 7.44 (never dense).
+template <class Op, class = void>
+struct dense8_of : std::integral_constant<uint32_t, 4u> {};
+template <class Op>
+struct dense8_of<Op, std::void_t<decltype(Op::kDense8)>> : std::integral_constant<uint32_t, Op::kDense8> {};
+template <class Op>
+__device__ __forceinline__ constexpr uint32_t dense_eighths() { return dense8_of<Op>::value; }
+
 // Edge-parallel expansion of nf compacted items (sm.off/deg/src/payload/pre):
 // 4 consecutive edges per thread, one binary search per 4 edges.
 template <class Op>
@@ -554,7 +566,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 // every vertex is selected -- measured the better choice for SSSP (RMAT-27
                 // 35.7 ms vs 42.8 ms when the selected words are counted instead; with the
                 // interleaved (adj, w) records 33.5 vs 35.3 ms)
-                const bool dense = 8 * total >= ps.dense8 * (W1 - W0);
+                const bool dense = 8 * total >= dense_eighths<Op>() * (W1 - W0);
                 if (dense) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
                     // 128-word windows; owners from record-start masks (no binary search;

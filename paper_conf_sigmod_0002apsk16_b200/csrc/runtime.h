@@ -54,7 +54,6 @@ struct PageSet {
     uint32_t entry_encoding;
     const uint32_t* rvt_start; // START_VID per page (PID16 decode)
     uint32_t hybrid_deg = 8;   // GTS_MICRO_HYBRID: vertex-centric below this many edges per vertex (R24)
-    uint32_t dense8 = 4;       // (temporary A/B) a tile is dense when 8 * selected edges >= dense8 * words
     uint32_t split = 1;        // work items per page: an LP's chunk is cut into `split` slices
                                // (small page sets, e.g. a hub's LPs at BFS level 0); SPs use slice 0
 };

@@ -37,6 +37,7 @@ template <bool W>
 struct BfsOp {
     static constexpr bool kReadWeights = false;
     static constexpr bool kWeighted = W;
+    static constexpr uint32_t kDense8 = 6;    // dense tiles only at >= 3/4 selected (expand.cuh)
     const uint32_t* cur;
     uint32_t* visited;
     uint32_t* next;
@@ -621,7 +622,6 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
                                 // few pages in this level (e.g. the source hub's LPs): slice LPs so
                                 // every CTA gets work, decided on the device
                                 p2.split = 0u;
-                                if (getenv("GTS_DEV_DENSE8")) p2.dense8 = (uint32_t)atoi(getenv("GTS_DEV_DENSE8"));
                                 const int gl = std::min(grid, cap);
                                 if (algo == kBFS) {
                                     bfs_kern<<<gl, kThreads, 0, s>>>(
@@ -862,6 +862,7 @@ template <bool W>
 struct MBfsOp {
     static constexpr bool kReadWeights = false;
     static constexpr bool kWeighted = W;
+    static constexpr uint32_t kDense8 = 6;
     const uint32_t* cur;       // biased bitmaps (word w of the rank's range at ptr[w])
     uint32_t* visited;
     uint32_t* next;
