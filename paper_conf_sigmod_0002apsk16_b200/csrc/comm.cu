@@ -271,6 +271,48 @@ int Ranks::route_overflow(Route& rt, bool* any) {
     return GTS_OK;
 }
 
+int Ranks::barrier() {
+    if (world == 1 || virt) return GTS_OK;            // virtual ranks share one stream
+    uint64_t* d;
+    GTS_TRY(c->buf(98, 8, (void**)&d));
+    GTS_NCCL(ncclAllReduce(d, d, 1, ncclUint64, ncclSum, c->comm, c->stream));
+    return GTS_OK;
+}
+
+int Ranks::peer_map(void* const* base, std::vector<std::array<void*, kMaxRanks>>& out) {
+    out.assign(nloc, {});
+    if (virt || world == 1) {
+        for (int i = 0; i < nloc; ++i)
+            for (int q = 0; q < nloc; ++q) out[i][q] = base[q];
+        return GTS_OK;
+    }
+    // real ranks: all-gather the IPC handles of every rank's allocation, open the peers'
+    cudaIpcMemHandle_t mine;
+    GTS_CUDA(cudaIpcGetMemHandle(&mine, base[0]));
+    uint8_t* d;
+    GTS_TRY(c->buf(99, sizeof(cudaIpcMemHandle_t) * (world + 1), (void**)&d));
+    GTS_CUDA(cudaMemcpyAsync(d, &mine, sizeof(mine), cudaMemcpyHostToDevice, c->stream));
+    GTS_NCCL(ncclAllGather(d, d + sizeof(mine), sizeof(mine), ncclUint8, c->comm, c->stream));
+    std::vector<cudaIpcMemHandle_t> all(world);
+    GTS_CUDA(cudaMemcpyAsync(all.data(), d + sizeof(mine), sizeof(mine) * world, cudaMemcpyDeviceToHost, c->stream));
+    GTS_CUDA(cudaStreamSynchronize(c->stream));
+    for (int q = 0; q < world; ++q) {
+        if (q == r0) {
+            out[0][q] = base[0];
+            continue;
+        }
+        const std::string key(reinterpret_cast<const char*>(&all[q]), sizeof(cudaIpcMemHandle_t));
+        auto it = c->ipc_open.find(key);
+        if (it == c->ipc_open.end()) {
+            void* p = nullptr;
+            GTS_CUDA(cudaIpcOpenMemHandle(&p, all[q], cudaIpcMemLazyEnablePeerAccess));
+            it = c->ipc_open.emplace(key, p).first;
+        }
+        out[0][q] = it->second;
+    }
+    return GTS_OK;
+}
+
 // ---- capacities: remote edges per (sender, owner) --------------------------
 
 template <bool W>

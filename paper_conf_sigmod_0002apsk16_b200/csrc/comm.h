@@ -71,6 +71,13 @@ struct Ranks {
     int route_exchange(Route& rt);
     // Max over ranks of each slot's overflow flag (returned on the host).
     int route_overflow(Route& rt, bool* any);
+    // Peer memory: out[i][q] = rank q's allocation `base[q's slot]` as seen by slot i (virtual
+    // ranks: the same pointer; real ranks: a CUDA IPC mapping of the peer's allocation over
+    // NVLink, exchanged through an all-gather of the IPC handles and cached in the context).
+    // base[i] must be the start of a cudaMalloc allocation of slot i.
+    int peer_map(void* const* base, std::vector<std::array<void*, kMaxRanks>>& out);
+    // Every rank has reached this point in stream order (an 8-byte all-reduce).
+    int barrier();
 };
 
 // The ranks this call runs: virtual (V > 1 on a world-1 context), a real rank, or one.

@@ -485,6 +485,7 @@ extern "C" void gts_context_free(gts_context* c) {
     free_devgraph(c->dg);
     for (auto& d : c->parked) free_devgraph(d);
     free_cache(c->cache);
+    for (auto& kv : c->ipc_open) cudaIpcCloseMemHandle(kv.second);
     for (auto& b : c->scratch) cudaFree(b.first);
     for (Timer* t : {&c->t_main, &c->t_finish, &c->t_merge, &c->t_h2d})
         for (auto& p : t->pairs) {

@@ -23,6 +23,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <array>
 #include <cstdlib>
 #include <cstring>
 
@@ -55,7 +56,9 @@ struct RouteParams {
     float* hot_out;                    // [n_hot] hot partial sums of vertices outside [lo, hi)
     uint64_t lo, hi;
     int drop_remote;                   // paper-literal Strategy-S (every page on every rank): drop remote updates
-    RouteOut ro;                       // Strategy-S: (dst, value) messages to the owners
+    int direct;                        // GTS_ROUTE_PEER: remote updates are atomics into the owner's WA
+    RouteOut ro;                       // Strategy-S: (dst, value) messages to the owners (ro.vr: the ranges)
+    float* peer_acc[kMaxRanks];        // GTS_ROUTE_PEER: every owner's WA (biased, peer memory)
 };
 
 // Per-thread destination emitter: combines runs of equal destinations (rows
@@ -75,6 +78,7 @@ struct PrEmitter {
         if (kMode == kRoute) {
             if (dst < H) atomicAdd(hacc + dst, c);
             else if ((uint64_t)dst >= rp->lo && (uint64_t)dst < rp->hi) atomicAdd(rp->acc_loc + dst, c);
+            else if (rp->direct) atomicAdd(rp->peer_acc[route_owner(rp->ro, dst)] + dst, c);   // over NVLink
             else if (!rp->drop_remote) route_push<uint2>(rp->ro, dst, make_uint2(dst, __float_as_uint(c)));
             return;
         }
@@ -321,6 +325,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             const float v = hacc[i];
             if (v == 0.f) continue;
             if ((uint64_t)i >= rp.lo && (uint64_t)i < rp.hi) atomicAdd(rp.acc_loc + i, v);
+            else if (rp.direct) atomicAdd(rp.peer_acc[route_owner(rp.ro, i)] + i, v);
             else if (!rp.drop_remote) atomicAdd(rp.hot_out + i, v);
         }
     } else {
@@ -332,6 +337,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) dang += __shfl_down_sync(0xFFFFFFFFu, dang, o);
     if ((tid & 31) == 0 && dang != 0.0) atomicAdd(dang_out, dang);
+    if (kMode == kRoute && rp.direct) __threadfence_system();   // peer atomics before the kernel ends
 }
 
 // Plain push PageRank (Alg 4/5: c = d x[u] / deg(u), one red.add per edge, no
@@ -466,6 +472,8 @@ struct PrSlot {
     uint64_t lo = 0, hi = 0;              // WA range this rank finishes
     float *x = nullptr, *acc = nullptr;   // absolute-index (biased) pointers
     float* hot = nullptr;                 // Strategy-S: dense partials [0, n_hot) of remote hot vertices
+    float* acc2 = nullptr;                // GTS_ROUTE_PEER: the second WA buffer (odd iterations)
+    std::array<float*, kMaxRanks> peer[2] = {};   // GTS_ROUTE_PEER: every owner's acc / acc2 (biased)
     double* dang = nullptr;               // [2] dangling-mass accumulators (ping-pong)
     std::vector<uint32_t> pages;          // host page ids (ascending)
     const uint32_t* d_pages = nullptr;    // device page ids (nullptr: all local pages in order)
@@ -488,6 +496,10 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     const int N = R.world, L = R.nloc;
     const uint32_t strat = R.world > 1 ? rc.strategy : GTS_STRATEGY_P;
     const bool route = strat == GTS_STRATEGY_S, bcast = strat == GTS_STRATEGY_S_BCAST;
+    // GTS_ROUTE_PEER: the scatter adds remote updates straight into their owner's WA over
+    // peer memory (fused scatter + exchange); acc is double-buffered so that no rank adds
+    // into a buffer its owner is still finishing (iteration t adds into acc[t & 1])
+    const bool peer = route && (rc.flags & GTS_ROUTE_PEER);
     const bool sharded = route || bcast;     // WA range-partitioned (the kRoute scatter)
     const bool streamed = choose_streamed(c, g, rc, route ? 8 * n / N + 4 * kHotDenseBig : 8 * n);
     double upload_s = 0;
@@ -580,8 +592,14 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         GTS_TRY(c->buf(L == 1 ? kBufDang : kBufPrMulti + 8 * i + 3, 2 * sizeof(double), (void**)&m.dang));
         m.x = xb - xlo;
         m.acc = ab - alo;
-        if (route) GTS_TRY(c->buf(kBufPrMulti + 8 * i + 4, std::max<uint32_t>(n_hot, 1) * 4, (void**)&m.hot));
-        if (i == 0) wa_bytes = (xn + an) * 4 + (route ? (uint64_t)n_hot * 4 : 0);
+        if (route && !peer) GTS_TRY(c->buf(kBufPrMulti + 8 * i + 4, std::max<uint32_t>(n_hot, 1) * 4, (void**)&m.hot));
+        if (peer) {
+            float* ab2;
+            GTS_TRY(c->buf(kBufPrMulti + 8 * i + 5, std::max<uint64_t>(an, 1) * 4, (void**)&ab2));
+            GTS_CUDA(cudaMemsetAsync(ab2, 0, std::max<uint64_t>(an, 1) * 4, s));
+            m.acc2 = ab2 - alo;
+        }
+        if (i == 0) wa_bytes = (xn + an * (peer ? 2 : 1)) * 4 + (route && !peer ? (uint64_t)n_hot * 4 : 0);
         pr_init_kernel<<<eg, 256, 0, s>>>(xb, xn, ab, an, (float)(1.0 / (double)n));
         GTS_CUDA(cudaMemsetAsync(m.dang, 0, 2 * sizeof(double), s));
         if (m.hot) GTS_CUDA(cudaMemsetAsync(m.hot, 0, std::max<uint32_t>(n_hot, 1) * 4, s));
@@ -589,7 +607,17 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     uint32_t* ctr;
     GTS_TRY(c->buf(kBufPrCtr, 4, (void**)&ctr));
     Route rt;
-    if (route) {
+    if (peer) {                                  // map every owner's two WA buffers
+        for (int k = 0; k < 2; ++k) {
+            std::vector<void*> base(L);
+            for (int i = 0; i < L; ++i) base[i] = (k ? S[i].acc2 : S[i].acc) + S[i].lo;
+            std::vector<std::array<void*, kMaxRanks>> pm;
+            GTS_TRY(R.peer_map(base.data(), pm));
+            for (int i = 0; i < L; ++i)
+                for (int q = 0; q < N; ++q) S[i].peer[k][q] = static_cast<float*>(pm[i][q]) - vr[q];
+        }
+        GTS_TRY(R.barrier());                    // every owner's buffers are zero before anyone adds
+    } else if (route) {
         std::vector<std::vector<uint32_t>> pl(L);
         std::vector<const uint32_t*> dpl(L);
         for (int i = 0; i < L; ++i) {
@@ -633,17 +661,22 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     };
     for (uint32_t it = 0; it < iters; ++it) {
         const int cur_d = it & 1;
-        if (route) GTS_CUDA(cudaMemsetAsync(rt.d_scnt, 0, (size_t)L * kMaxRanks * 8, s));
+        if (route && !peer) GTS_CUDA(cudaMemsetAsync(rt.d_scnt, 0, (size_t)L * kMaxRanks * 8, s));
         for (int i = 0; i < L; ++i) {           // ---- a7 / a8: the scatter over this rank's pages ----
             PrSlot& m = S[i];
             RouteParams rp;
             std::memset(&rp, 0, sizeof(rp));
-            rp.acc_loc = m.acc;
+            rp.acc_loc = (peer && (it & 1)) ? m.acc2 : m.acc;
             rp.hot_out = m.hot;
             rp.lo = m.lo;
             rp.hi = m.hi;
             rp.drop_remote = bcast ? 1 : 0;
-            if (route) {
+            if (peer) {
+                rp.direct = 1;
+                for (int q = 0; q <= N; ++q) rp.ro.vr[q] = vr[q];
+                rp.ro.nranks = N;
+                for (int q = 0; q < N; ++q) rp.peer_acc[q] = m.peer[it & 1][q];
+            } else if (route) {
                 rp.ro.send = rt.send[i];
                 rp.ro.cnt = rt.d_scnt + (size_t)i * kMaxRanks;
                 rp.ro.ovf = rt.d_ovf + i;
@@ -671,7 +704,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                 std::vector<void*> ab(L);
                 for (int i = 0; i < L; ++i) ab[i] = S[i].acc;
                 GTS_TRY(R.allreduce(ab.data(), n, kCF32, kCSum));
-            } else if (route) {                 // hot partials to their owners, then the routed pairs
+            } else if (route && !peer) {        // hot partials to their owners, then the routed pairs
                 std::vector<float*> part(L), dst(L);
                 for (int i = 0; i < L; ++i) {
                     part[i] = S[i].hot;
@@ -694,7 +727,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         if (timing) { cudaEventRecord(ev.second, s); ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
         // ---- a9: fused damping / dangling / swap over each rank's range ----
         for (PrSlot& m : S) {
-            pr_finish_kernel<<<2 * eg, 256, 0, s>>>(m.x, m.acc, n, m.lo, m.hi, damping, m.dang + cur_d,
+            // (GTS_ROUTE_PEER: the D all-reduce above is also the barrier after every rank's peer adds)
+            pr_finish_kernel<<<2 * eg, 256, 0, s>>>(m.x, (peer && (it & 1)) ? m.acc2 : m.acc, n, m.lo, m.hi, damping,
+                                                     m.dang + cur_d,
                                                      m.dang + (cur_d ^ 1), dangling == GTS_DANGLING_UNIFORM ? 1 : 0);
             ++launches;
         }
@@ -706,7 +741,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         if (timing) cudaEventRecord(ev.second, s);
         GTS_CUDA(cudaGetLastError());
     }
-    if (route) {
+    if (route && !peer) {
         bool ovf = false;
         GTS_TRY(R.route_overflow(rt, &ovf));
         if (ovf) return fail(GTS_ECUDA, "Strategy-S route region overflow (capacity count mismatch)");

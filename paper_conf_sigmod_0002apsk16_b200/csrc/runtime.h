@@ -6,6 +6,7 @@
 
 #include <chrono>
 #include <map>
+#include <string>
 #include <cstdlib>
 #include <utility>
 #include <vector>
@@ -123,6 +124,7 @@ struct Context {
     cudaEvent_t ring_ready[64], ring_free[64];
     bool ring_events = false;
     uint64_t launches = 0, main_launches = 0;
+    std::map<std::string, void*> ipc_open;   // peer allocations opened by handle bytes (GTS_ROUTE_PEER)
     size_t persist_limit = 0;      // cudaLimitPersistingL2CacheSize set by this context
     size_t persist_max = 0;        // device attributes, queried once
     size_t window_max = 0;

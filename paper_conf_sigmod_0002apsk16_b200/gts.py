@@ -29,6 +29,7 @@ GTS_RESIDENCY_AUTO, GTS_RESIDENT, GTS_STREAMED = 0, 1, 2
 GTS_DANGLING_UNIFORM, GTS_DANGLING_DROP = 0, 1
 GTS_OUT_HOST, GTS_OUT_DEVICE = 0, 1
 GTS_RUN_TIMING = 1
+GTS_ROUTE_PEER = 2
 # micro-level technique inside each page (gts_run_config.flags bits 8-10; App E, Fig 14)
 GTS_MICRO_DEFAULT, GTS_MICRO_EDGE, GTS_MICRO_VERTEX, GTS_MICRO_HYBRID, GTS_MICRO_TILE = 0, 1 << 8, 2 << 8, 3 << 8, 4 << 8
 MICRO = {"default": GTS_MICRO_DEFAULT, "edge": GTS_MICRO_EDGE, "vertex": GTS_MICRO_VERTEX,
@@ -322,9 +323,12 @@ def gts_bfs(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RE
 
 def gts_pagerank(ctx, graph, iters=10, damping=0.85, dangling=GTS_DANGLING_UNIFORM, out=None,
                  strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0, batch_pages=0, timing=False,
-                 micro=GTS_MICRO_DEFAULT, virtual_ranks=0, tune=None):
+                 micro=GTS_MICRO_DEFAULT, virtual_ranks=0, tune=None, route_peer=False):
+    """route_peer: Strategy-S adds remote updates straight into their owner's WA over peer memory."""
     out, ptr, loc = _out(out, graph.n, np.float32, ctx)
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, 0, micro, virtual_ranks, tune)
+    if route_peer:
+        cfg.flags |= GTS_ROUTE_PEER
     st = RunStats()
     _check(_lib.gts_pagerank(ctx.handle, graph.handle, int(iters), float(damping), int(dangling),
                              ctypes.byref(cfg), ptr, ctypes.byref(st)))

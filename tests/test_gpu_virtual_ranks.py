@@ -177,3 +177,24 @@ def test_virtual_ranks_rejected_on_bad_values(G, ctx):
     with pytest.raises(G.GtsError) as e:
         G.gts_bfs(ctx, gr, 0, virtual_ranks=2, micro="edge")
     assert e.value.code == G.GTS_EUNSUPPORTED
+
+
+@pytest.mark.parametrize("name", GRAPHS + ["instar"])
+@pytest.mark.parametrize("order", [False, True])
+@pytest.mark.parametrize("V", VS)
+def test_pagerank_strategy_s_peer(G, ctx, name, order, V):
+    """GTS_ROUTE_PEER: the Strategy-S scatter adds every remote update (and every remote
+    hot partial) straight into the owner's WA -- the fused scatter + exchange over peer
+    memory -- with WA double-buffered across iterations; same result as the oracle."""
+    g, pb = case(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=order)
+    for dangling in (0, 1):
+        want = oracle.pagerank(g.row_ptr, g.col, 10, 0.85, dangling=dangling)
+        got, st = G.gts_pagerank(ctx, gr, 10, 0.85, dangling=dangling, strategy=STRATS["S"], virtual_ranks=V,
+                                 route_peer=True)
+        ok, rel = pr_ok(got, want)
+        assert ok, (name, order, V, dangling, rel)
+        assert st["routed_msgs"] == 0
+    got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, strategy=STRATS["S"], virtual_ranks=V, route_peer=True,
+                            residency=G.GTS_STREAMED, batch_pages=4, ring_slots=2)
+    assert pr_ok(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85))[0]
