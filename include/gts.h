@@ -96,12 +96,15 @@ enum { GTS_RESIDENCY_AUTO = 0, GTS_RESIDENT = 1, GTS_STREAMED = 2 };
 enum { GTS_DANGLING_UNIFORM = 0, GTS_DANGLING_DROP = 1 };
 enum { GTS_OUT_HOST = 0, GTS_OUT_DEVICE = 1 };
 enum { GTS_RUN_TIMING = 1u };   /* gts_run_config.flags: time the main kernels with CUDA events */
-/* gts_run_config.flags: Strategy-S PageRank routes its remote updates by atomics
- * straight into the owner's WA over peer memory (NVLink / NVSwitch; CUDA IPC
- * mappings between the ranks' processes), fusing the scatter with the exchange:
- * no message buffers, counts or send/recv -- one kernel does the compute and the
- * "collective".  Default off (routed messages over NCCL).  Virtual ranks map the
- * other ranks' buffers on the same GPU. */
+/* gts_run_config.flags: Strategy-S routes its remote updates by atomics straight
+ * into the owner's WA over peer memory (NVLink / NVSwitch; CUDA IPC mappings
+ * between the ranks' processes), fusing the sweep with the exchange: no message
+ * buffers, counts or send/recv -- one kernel does the compute and the
+ * "collective" (PageRank atomicAdd into the owner's acc, BFS atomicOr into its
+ * visited / next bitmaps, SSSP / WCC atomicMin into its dist / labels).  The
+ * owners' WA buffers that receive updates while they are read are
+ * double-buffered by iteration / level.  Default off (routed messages over
+ * NCCL).  Virtual ranks map the other ranks' buffers on the same GPU. */
 enum { GTS_ROUTE_PEER = 2u };
 /* gts_run_config.flags bits 8-10: the micro-level technique applied inside each
  * slotted page (App E, Fig 14), for gts_bfs and

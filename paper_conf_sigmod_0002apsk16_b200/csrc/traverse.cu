@@ -21,6 +21,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <array>
 #include <cstring>
 
 #include "comm.h"
@@ -858,6 +859,14 @@ enum { kDstAll = 0, kDstRoute = 1, kDstDrop = 2 };   // remote destinations: (no
 
 __device__ __forceinline__ bool in_range(uint32_t v, uint64_t lo, uint64_t hi) { return (uint64_t)v - lo < hi - lo; }
 
+// GTS_ROUTE_PEER: every owner's WA as seen by this rank (biased pointers: absolute
+// VIDs / bitmap words), so a remote update is one atomic over peer memory
+struct PeerWA {
+    uint32_t* val[kMaxRanks];   // LV / dist / label
+    uint32_t* vis[kMaxRanks];   // BFS visited bitmap
+    uint32_t* nxt[kMaxRanks];   // next-frontier bitmap of this level
+};
+
 template <bool W>
 struct MBfsOp {
     static constexpr bool kReadWeights = false;
@@ -871,6 +880,8 @@ struct MBfsOp {
     uint64_t lo, hi;
     int mode;
     RouteOut ro;
+    int direct;                // GTS_ROUTE_PEER
+    PeerWA pw;
     __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
@@ -893,7 +904,12 @@ struct MBfsOp {
             if (in_range(v, lo, hi)) {
                 if (!(__ldcg(visited + wi) & b) && !(atomicOr(visited + wi, b) & b)) atomicOr(next + wi, b);
             } else if (mode == kDstRoute) {
-                if (!(__ldcg(sent + wi) & b) && !(atomicOr(sent + wi, b) & b)) route_push<uint32_t>(ro, v, v);
+                if (direct) {          // discovery in the owner's bitmaps over peer memory
+                    const int q = route_owner(ro, v);
+                    if (!(atomicOr(pw.vis[q] + wi, b) & b)) atomicOr(pw.nxt[q] + wi, b);
+                } else if (!(__ldcg(sent + wi) & b) && !(atomicOr(sent + wi, b) & b)) {
+                    route_push<uint32_t>(ro, v, v);
+                }
             }
         }
     }
@@ -916,6 +932,8 @@ struct MMinOp {
     uint64_t lo, hi;
     int mode;
     RouteOut ro;
+    int direct;                // GTS_ROUTE_PEER
+    PeerWA pw;
     __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v) && (!kSssp || __ldcg(val + v) <= T); }
     __device__ uint32_t payload(uint32_t v, uint32_t deg) {
@@ -947,7 +965,12 @@ struct MMinOp {
             if (in_range(v, lo, hi)) {
                 if (cand < __ldcg(val + v) && cand < atomicMin(val + v, cand)) atomicOr(next + (v >> 5), 1u << (v & 31));
             } else if (mode == kDstRoute) {
-                route_push<uint2>(ro, v, make_uint2(v, cand));
+                if (direct) {          // atomicMin in the owner's WA over peer memory
+                    const int q = route_owner(ro, v);
+                    if (cand < atomicMin(pw.val[q] + v, cand)) atomicOr(pw.nxt[q] + (v >> 5), 1u << (v & 31));
+                } else {
+                    route_push<uint2>(ro, v, make_uint2(v, cand));
+                }
             }
         }
     }
@@ -960,6 +983,7 @@ mbfs_expand_kernel(PageSet ps, MBfsOp<W> op, uint32_t* work_ctr, unsigned long l
     __shared__ TileSmem sm;
     expand_pages(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
+    if (op.direct) __threadfence_system();     // peer atomics before the kernel ends
 }
 
 template <bool W, bool kSssp>
@@ -970,6 +994,7 @@ mmin_expand_kernel(PageSet ps, MMinOp<W, kSssp> op, uint32_t* work_ctr, unsigned
     expand_pages(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
     if (__syncthreads_or(op.ovf) && threadIdx.x == 0) *ovf_flag = 1u;
+    if (op.direct) __threadfence_system();
 }
 
 struct RecvView {
@@ -1024,6 +1049,8 @@ struct MSlot {
     uint32_t *value = nullptr, *visited = nullptr, *cur = nullptr, *next = nullptr, *sent = nullptr;  // biased
     uint32_t *gathered = nullptr, *list = nullptr, *d_pages = nullptr;
     Counters* ctr = nullptr;
+    uint32_t *cur0 = nullptr, *next0 = nullptr;   // the two frontier buffers as allocated (biased)
+    std::array<uint32_t*, kMaxRanks> pval{}, pvis{}, pcur0{}, pnext0{};   // GTS_ROUTE_PEER: owners' WA
     std::vector<uint32_t> pages, h_list;
     Counters h = {};
 };
@@ -1038,6 +1065,9 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
     const int N = R.world, L = R.nloc;
     const uint32_t strat = rc.strategy;
     const bool route = strat == GTS_STRATEGY_S;
+    // GTS_ROUTE_PEER: remote updates are atomics into the owner's WA over peer memory (the
+    // expansion fused with the exchange); the owners' next bitmaps are double-buffered by level
+    const bool peer = route && (rc.flags & GTS_ROUTE_PEER);
     const int mode = strat == GTS_STRATEGY_P ? kDstAll : route ? kDstRoute : kDstDrop;
     if (algo == kWCCLP && !route) return fail(GTS_EINVAL, "label propagation is the Strategy-S WCC");
     if (algo == kWCCLP && !g->symmetric)
@@ -1086,7 +1116,9 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
         m.next = nx - m.w0;
         if (i == 0) wa_bytes = nv * 4 + nw * 4 * (algo == kBFS ? 3 : 2);
         if (!route) GTS_TRY(c->buf(kBufMulti + 16 * i + 5, (size_t)N * words * 4, (void**)&m.gathered));
-        if (route && algo == kBFS) {
+        m.cur0 = m.cur;
+        m.next0 = m.next;
+        if (route && algo == kBFS && !peer) {
             GTS_TRY(c->buf(kBufMulti + 16 * i + 6, words * 4, (void**)&m.sent));
             GTS_CUDA(cudaMemsetAsync(m.sent, 0, words * 4, s));
             if (i == 0) wa_bytes += words * 4;
@@ -1127,7 +1159,28 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
     }
     GTS_CUDA(cudaStreamSynchronize(s));        // host vectors above are read by the copies
     Route rt;
-    if (route) {
+    if (peer) {                        // map every owner's WA allocations into this rank
+        auto map = [&](auto get, auto put, bool words_bias) -> int {
+            std::vector<void*> base(L);
+            for (int i = 0; i < L; ++i) base[i] = get(S[i]);
+            std::vector<std::array<void*, kMaxRanks>> pm;
+            GTS_TRY(R.peer_map(base.data(), pm));
+            for (int i = 0; i < L; ++i)
+                for (int q = 0; q < N; ++q)
+                    put(S[i], q, static_cast<uint32_t*>(pm[i][q]) - (words_bias ? (vr[q] >> 5) : vr[q]));
+            return GTS_OK;
+        };
+        GTS_TRY(map([](MSlot& m) { return (void*)(m.value + m.lo); },
+                    [](MSlot& m, int q, uint32_t* p) { m.pval[q] = p; }, false));
+        if (algo == kBFS)
+            GTS_TRY(map([](MSlot& m) { return (void*)(m.visited + m.w0); },
+                        [](MSlot& m, int q, uint32_t* p) { m.pvis[q] = p; }, true));
+        GTS_TRY(map([](MSlot& m) { return (void*)(m.cur0 + m.w0); },
+                    [](MSlot& m, int q, uint32_t* p) { m.pcur0[q] = p; }, true));
+        GTS_TRY(map([](MSlot& m) { return (void*)(m.next0 + m.w0); },
+                    [](MSlot& m, int q, uint32_t* p) { m.pnext0[q] = p; }, true));
+        GTS_TRY(R.barrier());          // every owner's WA is initialised before anyone writes into it
+    } else if (route) {
         std::vector<std::vector<uint32_t>> pl(L);
         std::vector<const uint32_t*> dpl(L);
         for (int i = 0; i < L; ++i) {
@@ -1151,22 +1204,31 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
     uint32_t levels = 0;
     SweepStats ss;
     for (uint32_t lev = 0;; ++lev) {
-        if (route) GTS_CUDA(cudaMemsetAsync(rt.d_scnt, 0, (size_t)L * kMaxRanks * 8, s));
+        if (route && !peer) GTS_CUDA(cudaMemsetAsync(rt.d_scnt, 0, (size_t)L * kMaxRanks * 8, s));
         for (int i = 0; i < L; ++i) {
             MSlot& m = S[i];
             pages_processed += m.h.list_count;
             RouteOut ro{};
             if (route) {
+                for (int q = 0; q <= N; ++q) ro.vr[q] = vr[q];
+                ro.nranks = N;
+            }
+            if (route && !peer) {
                 ro.send = rt.send[i];
                 ro.cnt = rt.d_scnt + (size_t)i * kMaxRanks;
                 ro.ovf = rt.d_ovf + i;
-                for (int q = 0; q <= N; ++q) ro.vr[q] = vr[q];
                 for (int q = 0; q < N; ++q) {
                     ro.off[q] = rt.soff[i][q];
                     ro.cap[q] = rt.scap[i][q];
                 }
-                ro.nranks = N;
             }
+            PeerWA pwl{};
+            if (peer)                  // this level's next bitmap of every owner: the buffers alternate
+                for (int q = 0; q < N; ++q) {
+                    pwl.val[q] = m.pval[q];
+                    pwl.vis[q] = m.pvis[q];
+                    pwl.nxt[q] = (lev & 1) ? m.pcur0[q] : m.pnext0[q];
+                }
             auto launch = [&](const PageSet& ps, int gcap) -> int {
                 GTS_CUDA(cudaMemsetAsync(&m.ctr->work, 0, 4, s));
                 std::pair<cudaEvent_t, cudaEvent_t> ev;
@@ -1176,22 +1238,22 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
                 const int gl = std::min(grid, gcap);
                 if (algo == kBFS) {
                     if (W) {
-                        MBfsOp<true> op{m.cur, m.visited, m.next, m.sent, 0ull, m.lo, m.hi, mode, ro};
+                        MBfsOp<true> op{m.cur, m.visited, m.next, m.sent, 0ull, m.lo, m.hi, mode, ro, peer ? 1 : 0, pwl};
                         mbfs_expand_kernel<true><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges);
                     } else {
-                        MBfsOp<false> op{m.cur, m.visited, m.next, m.sent, 0ull, m.lo, m.hi, mode, ro};
+                        MBfsOp<false> op{m.cur, m.visited, m.next, m.sent, 0ull, m.lo, m.hi, mode, ro, peer ? 1 : 0, pwl};
                         mbfs_expand_kernel<false><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges);
                     }
                 } else if (algo == kSSSP) {
-                    MMinOp<true, true> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro};
+                    MMinOp<true, true> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro, peer ? 1 : 0, pwl};
                     mmin_expand_kernel<true, true><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges,
                                                                          &m.ctr->flag);
                 } else if (W) {
-                    MMinOp<true, false> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro};
+                    MMinOp<true, false> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro, peer ? 1 : 0, pwl};
                     mmin_expand_kernel<true, false><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges,
                                                                           &m.ctr->flag);
                 } else {
-                    MMinOp<false, false> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro};
+                    MMinOp<false, false> op{m.cur, m.value, m.next, 0ull, false, T, m.lo, m.hi, mode, ro, peer ? 1 : 0, pwl};
                     mmin_expand_kernel<false, false><<<gl, kThreads, 0, s>>>(p2, op, &m.ctr->work, &m.ctr->edges,
                                                                            &m.ctr->flag);
                 }
@@ -1205,7 +1267,9 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
         // ---- merge (a12) ----
         std::pair<cudaEvent_t, cudaEvent_t> ev;
         if (timing) { ev = c->t_merge.next(); cudaEventRecord(ev.first, s); }
-        if (route) {
+        if (peer) {
+            GTS_TRY(R.barrier());      // every rank's peer atomics of this level are done
+        } else if (route) {
             GTS_TRY(R.route_exchange(rt));
             for (int i = 0; i < L; ++i) {
                 RecvView rv{};
@@ -1250,6 +1314,9 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
             frontier_pages_kernel<<<eg, 256, 0, s>>>(m.next, c->dg.rvt_start, c->dg.nslots, m.d_pages,
                                                      (uint32_t)m.pages.size(), m.list, &m.ctr->list_count);
             launches += 2;
+            // GTS_ROUTE_PEER: this level's cur becomes the next level's next, which other ranks
+            // write into once they pass the count all-reduce below -- clear it before it
+            if (peer) GTS_CUDA(cudaMemsetAsync(m.cur + m.w0, 0, (m.w1 - m.w0) * 4, s));
         }
         if (route) {                       // frontier counts are per range: sum (SSSP: and min) over ranks
             std::vector<void*> b(L);
@@ -1284,10 +1351,10 @@ int traverse_multi(gts_context* c, const gts_graph* g, uint64_t src, const gts_r
                 }
             }
             std::swap(m.cur, m.next);
-            GTS_CUDA(cudaMemsetAsync(m.next + m.w0, 0, (m.w1 - m.w0) * 4, s));
+            if (!peer) GTS_CUDA(cudaMemsetAsync(m.next + m.w0, 0, (m.w1 - m.w0) * 4, s));
         }
     }
-    if (route) {
+    if (route && !peer) {
         bool ovf = false;
         GTS_TRY(R.route_overflow(rt, &ovf));
         if (ovf) return fail(GTS_ECUDA, "Strategy-S route region overflow (capacity count mismatch)");

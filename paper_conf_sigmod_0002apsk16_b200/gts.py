@@ -311,11 +311,13 @@ def _out(out, n, dtype, ctx=None):
 
 
 def gts_bfs(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-            batch_pages=0, timing=False, cache_mib=0, micro=GTS_MICRO_DEFAULT, virtual_ranks=0, tune=None):
+            batch_pages=0, timing=False, cache_mib=0, micro=GTS_MICRO_DEFAULT, virtual_ranks=0, tune=None,
+            route_peer=False):
     """Returns (levels, stats dict).  micro: GTS_MICRO_* or "default"/"edge"/"vertex"/"hybrid".
     virtual_ranks=V: run the V-rank job of `strategy` on this GPU.  tune: {gts_run_config 1.1 field: value}."""
     out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib, micro, virtual_ranks, tune)
+    cfg.flags |= GTS_ROUTE_PEER if route_peer else 0
     st = RunStats()
     _check(_lib.gts_bfs(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()
@@ -336,18 +338,20 @@ def gts_pagerank(ctx, graph, iters=10, damping=0.85, dangling=GTS_DANGLING_UNIFO
 
 
 def gts_sssp(ctx, graph, src, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-             batch_pages=0, timing=False, cache_mib=0, virtual_ranks=0, tune=None):
+             batch_pages=0, timing=False, cache_mib=0, virtual_ranks=0, tune=None, route_peer=False):
     out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, cache_mib, 0, virtual_ranks, tune)
+    cfg.flags |= GTS_ROUTE_PEER if route_peer else 0
     st = RunStats()
     _check(_lib.gts_sssp(ctx.handle, graph.handle, int(src), ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()
 
 
 def gts_wcc(ctx, graph, out=None, strategy=GTS_STRATEGY_P, residency=GTS_RESIDENCY_AUTO, ring_slots=0,
-            batch_pages=0, timing=False, virtual_ranks=0, tune=None):
+            batch_pages=0, timing=False, virtual_ranks=0, tune=None, route_peer=False):
     out, ptr, loc = _out(out, graph.n, np.uint32, ctx)
     cfg = _run_config(strategy, residency, ring_slots, batch_pages, loc, timing, 0, 0, virtual_ranks, tune)
+    cfg.flags |= GTS_ROUTE_PEER if route_peer else 0
     st = RunStats()
     _check(_lib.gts_wcc(ctx.handle, graph.handle, ctypes.byref(cfg), ptr, ctypes.byref(st)))
     return out, st.as_dict()

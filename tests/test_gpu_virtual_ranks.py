@@ -198,3 +198,28 @@ def test_pagerank_strategy_s_peer(G, ctx, name, order, V):
     got, _ = G.gts_pagerank(ctx, gr, 10, 0.85, strategy=STRATS["S"], virtual_ranks=V, route_peer=True,
                             residency=G.GTS_STREAMED, batch_pages=4, ring_slots=2)
     assert pr_ok(got, oracle.pagerank(g.row_ptr, g.col, 10, 0.85))[0]
+
+
+@pytest.mark.parametrize("name", GRAPHS)
+@pytest.mark.parametrize("V", VS)
+def test_bfs_sssp_wcc_strategy_s_peer(G, ctx, name, V):
+    """GTS_ROUTE_PEER for the BFS-like algorithms: remote discoveries / relaxations / label
+    updates are atomics in the owner's visited / next bitmaps, dist and labels (the next
+    bitmaps alternate by level); bit-exact vs the oracle, resident and streamed."""
+    g, pb = case(name)
+    w = inputs.edge_weights(g)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+    grw = G.gts_build_pages(g.row_ptr, g.col, w, page_bytes=pb)
+    grs = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, symmetric=True, order=(V == 3))
+    for kw in ({}, dict(residency=G.GTS_STREAMED, batch_pages=4, ring_slots=2)):
+        kw = dict(kw, strategy=STRATS["S"], virtual_ranks=V, route_peer=True)
+        for src in (0, int(np.argmax(np.diff(g.row_ptr)))):
+            got, st = G.gts_bfs(ctx, gr, src, **kw)
+            assert np.array_equal(got, oracle.bfs(g.row_ptr, g.col, src)), (name, V, src, kw)
+            assert st["routed_msgs"] == 0
+            got, _ = G.gts_sssp(ctx, grw, src, **kw)
+            assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, src)), (name, V, src, kw)
+        got, _ = G.gts_wcc(ctx, grs, **kw)
+        assert np.array_equal(got, oracle.wcc(g.row_ptr, g.col)), (name, V, kw)
+    got, _ = G.gts_sssp(ctx, grw, 0, strategy=STRATS["S"], virtual_ranks=V, route_peer=True, tune={"sssp_delta": 32})
+    assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, 0))
