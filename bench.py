@@ -558,7 +558,7 @@ def main():
         hl = torch.empty(n, dtype=torch.int32, pin_memory=True)      # pinned host result buffers
         hp = torch.empty(n, dtype=torch.float32, pin_memory=True)
         tb, tp_ = [], []
-        for _ in range(max(1, min(K, 3))):
+        for _ in range(max(1, min(K, 5))):
             ctx.evict(gr)
             barrier()
             t0 = time.perf_counter()
