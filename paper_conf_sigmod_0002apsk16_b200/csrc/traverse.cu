@@ -556,7 +556,8 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     const uint32_t hybrid_deg = rc.hybrid_deg ? rc.hybrid_deg : 8u;
     // two 512-thread CTAs per SM for the SSSP expansion (three measured 35.7 vs 35.1 ms on
     // RMAT-27: the weighted walk spills at 40 registers)
-    auto sssp_kern = sssp_expand_kernel<2>;
+    auto sssp_kern = (getenv("GTS_DEV_SSSP3") && atoi(getenv("GTS_DEV_SSSP3")) > 0) ? sssp_expand_kernel<3>
+                                                                                      : sssp_expand_kernel<2>;   // (temporary A/B)
     const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_kern;
     int grid = 0;
     GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
