@@ -54,15 +54,6 @@ namespace gts {
 //              per-CTA aggregation a hub's fp32 sum takes millions of sequential adds)
 enum PrMode : int { kHash = 0, kDense = 1, kRoute = 2, kRouteHash = 3 };
 
-// Where the scatter reads x (XSrc.accp == nullptr: the materialised x)
-struct XSrc {
-    const float* accp;                 // previous iteration's acc: x_u = base(D_prev) + accp[u]
-    const double* dprev;               // previous iteration's dangling mass
-    double d;
-    uint64_t n;
-    int uniform;
-};
-
 struct RouteParams {
     float* acc_loc;                    // local WA, biased: acc_loc[v] for v in [lo, hi)
     float* hot_out;                    // [n_hot] hot partial sums of vertices outside [lo, hi)
@@ -165,12 +156,7 @@ __device__ __forceinline__ uint32_t pr_decode(uint32_t e, const uint32_t* rvt) {
 template <bool kWeighted, int kMode, int T, int kMinBlocks, uint32_t H, int VPT, bool kVid>
 __global__ void __launch_bounds__(T, kMinBlocks)
 pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__ hot_keys,
-                  float d, double* dang_out, uint32_t* work_ctr, uint32_t n_hot, const RouteParams rp, const XSrc xs) {
-    // x_u of this iteration: x[u], or (the previous finish fused into this read) the previous
-    // iteration's base + acc_prev[u], base computed exactly as pr_finish_kernel does
-    const float xbase = xs.accp ? (float)((1.0 - xs.d) / (double)xs.n + (xs.uniform ? xs.d * *xs.dprev / (double)xs.n : 0.0))
-                                : 0.f;
-    const float* xr = xs.accp ? xs.accp : x;
+                  float d, double* dang_out, uint32_t* work_ctr, uint32_t n_hot, const RouteParams rp) {
     __shared__ PrSmem<T * VPT> sm;
     extern __shared__ uint4 dyn_smem[];
     uint32_t* hkeys = reinterpret_cast<uint32_t*>(dyn_smem);
@@ -208,7 +194,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
             const uint32_t vid = ld32(end - kLpFooter - kSlotBytes);
             const uint32_t total = ld32(end - 16);
             const uint32_t len = ld32(data);
-            const float c = d * (xbase + __ldg(xr + vid)) / (float)total;
+            const float c = d * __ldg(x + vid) / (float)total;
             // entries: words [hdr, hdr + len) (unweighted) or the even words of [2, 2 + 2 len)
             constexpr uint32_t hdr = rec_hdr_words(kWeighted);
             const uint32_t wend = hdr + (len << wshift), qend = (wend + 3) >> 2;
@@ -250,7 +236,7 @@ pr_scatter_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uin
                     if (i < nv) {
                         const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(t0 + i + 1);
                         r_off[k] = ld_stream_u32(slot + 4, pol);
-                        r_x[k] = xbase + ld_stream_f32(xr + start + t0 + i, pol);
+                        r_x[k] = ld_stream_f32(x + start + t0 + i, pol);
                         if (i == nv - 1)              // end of the tile's last record: the next slot's offset
                             r_nxt = t0 + nv < nslots ? ld_stream_u32(slot - kSlotBytes + 4, pol) : 0xFFFFFFFFu;
                     }
@@ -408,7 +394,7 @@ struct PrMicroOp {
 template <bool W, int M>
 __global__ void __launch_bounds__(kThreads, 2)
 pr_micro_kernel(PageSet ps, const float* __restrict__ x, float* acc, const uint32_t* __restrict__, float d,
-                double* dang_out, uint32_t* work_ctr, uint32_t, const RouteParams, const XSrc) {
+                double* dang_out, uint32_t* work_ctr, uint32_t, const RouteParams) {
     __shared__ TileSmem sm;
     PrMicroOp<W> op{x, acc, d, 0.0};
     expand_pages<PrMicroOp<W>, M>(ps, op, sm, work_ctr);
@@ -488,7 +474,7 @@ __global__ void pr_route_apply_kernel(PrRecv rv, float* acc) {
     }
 }
 
-enum { kBufX = 20, kBufAcc, kBufDang, kBufPrCtr, kBufPrHot = 24, kBufAcc2 = 25, kBufPrList = 28 };
+enum { kBufX = 20, kBufAcc, kBufDang, kBufPrCtr, kBufPrHot = 24, kBufPrList = 28 };
 constexpr int kBufPrMulti = 300;   // multi-rank slot i: kBufPrMulti + 8 i + k
 constexpr int kBufPrRoute = 120;   // route buffers
 
@@ -531,11 +517,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     // peer memory (fused scatter + exchange); acc is double-buffered so that no rank adds
     // into a buffer its owner is still finishing (iteration t adds into acc[t & 1])
     const bool peer = route && (rc.flags & GTS_ROUTE_PEER);
-    // one rank: the finish of iteration t is fused into iteration t+1's read of x
-    // (x_u = base(D_t) + acc_t[u]); acc alternates between two buffers, the one just read is
-    // cleared by a memset, and x is materialised once after the last iteration
-    const char* dfx = getenv("GTS_DEV_FUSEX");   // (temporary A/B)
-    const bool fusedx = N == 1 && !((rc.flags & GTS_MICRO_MASK) >> 8) && dfx && atoi(dfx) > 0;
+    // (Fusing iteration t's finish into iteration t+1's read of x -- x_u = base(D_t) + acc_t[u],
+    // acc double-buffered, the buffer just read cleared by a memset -- measured on RMAT-27: call
+    // 113.9 vs 115.0 ms but the scatter 11.03 vs 10.88 ms; not adopted.)
     const bool sharded = route || bcast;     // WA range-partitioned (the kRoute scatter)
     const bool streamed = choose_streamed(c, g, rc, route ? 8 * n / N + 4 * kHotDenseBig : 8 * n);
     double upload_s = 0;
@@ -635,12 +619,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         m.x = xb - xlo;
         m.acc = ab - alo;
         if (route && !peer) GTS_TRY(c->buf(kBufPrMulti + 8 * i + 4, std::max<uint32_t>(n_hot, 1) * 4, (void**)&m.hot));
-        if (fusedx) {
-            float* ab2;
-            GTS_TRY(c->buf(kBufAcc2, std::max<uint64_t>(an, 1) * 4, (void**)&ab2));
-            GTS_CUDA(cudaMemsetAsync(ab2, 0, std::max<uint64_t>(an, 1) * 4, s));
-            m.acc2 = ab2;
-        }
         if (peer) {
             float* ab2;
             GTS_TRY(c->buf(kBufPrMulti + 8 * i + 5, std::max<uint64_t>(an, 1) * 4, (void**)&ab2));
@@ -685,8 +663,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     SweepStats ss;
     const float dmp = (float)damping;
     const uint32_t* hk = c->dg.hot_keys;
-    XSrc xs{nullptr, nullptr, damping, n, dangling == GTS_DANGLING_UNIFORM ? 1 : 0};
-    float* target = nullptr;                     // fusedx: this iteration's acc
     auto scatter = [&](PrSlot& m, const PageSet& ps, int gcap, double* D, const RouteParams& rp) -> int {
         GTS_CUDA(cudaMemsetAsync(ctr, 0, 4, s));
         std::pair<cudaEvent_t, cudaEvent_t> e2;
@@ -694,9 +670,9 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         PageSet p2 = ps;
         p2.hybrid_deg = hybrid_deg;
         const float* xr = m.x;
-        float* ar = fusedx ? target : m.acc;
+        float* ar = m.acc;
         void* args[] = {(void*)&p2, (void*)&xr, (void*)&ar, (void*)&hk, (void*)&dmp, (void*)&D, (void*)&ctr,
-                        (void*)&n_hot, (void*)&rp, (void*)&xs};
+                        (void*)&n_hot, (void*)&rp};
         cudaLaunchConfig_t lc;
         std::memset(&lc, 0, sizeof(lc));
         lc.gridDim = dim3(std::min(grid, gcap));
@@ -711,13 +687,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
     };
     for (uint32_t it = 0; it < iters; ++it) {
         const int cur_d = it & 1;
-        if (fusedx) {
-            PrSlot& m = S[0];
-            target = (it & 1) ? m.acc2 : m.acc;
-            xs.accp = it == 0 ? nullptr : ((it & 1) ? m.acc : m.acc2);
-            xs.dprev = m.dang + (cur_d ^ 1);
-            GTS_CUDA(cudaMemsetAsync(m.dang + cur_d, 0, sizeof(double), s));
-        }
         if (route && !peer) GTS_CUDA(cudaMemsetAsync(rt.d_scnt, 0, (size_t)L * kMaxRanks * 8, s));
         for (int i = 0; i < L; ++i) {           // ---- a7 / a8: the scatter over this rank's pages ----
             PrSlot& m = S[i];
@@ -744,8 +713,7 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
                 }
                 rp.ro.nranks = N;
             }
-            if (persist)
-                GTS_TRY(persist_window(c, s, fusedx ? target : m.acc, std::min<size_t>(l2_persist_mib(rc) << 20, n * 4)));
+            if (persist) GTS_TRY(persist_window(c, s, m.acc, std::min<size_t>(l2_persist_mib(rc) << 20, n * 4)));
             std::vector<uint32_t> hl(m.pages);
             GTS_TRY(sweep_pages(c, g, rc, streamed, &hl, m.d_pages, (uint32_t)hl.size(), nullptr,
                                 [&](const PageSet& ps, int gcap) -> int {
@@ -784,20 +752,6 @@ extern "C" int gts_pagerank(gts_context* c, const gts_graph* g, uint32_t iters, 
         }
         if (timing) { cudaEventRecord(ev.second, s); ev = c->t_finish.next(); cudaEventRecord(ev.first, s); }
         // ---- a9: fused damping / dangling / swap over each rank's range ----
-        if (fusedx) {                             // clear the acc just read; x only after the last iteration
-            PrSlot& m = S[0];
-            if (xs.accp) GTS_CUDA(cudaMemsetAsync(const_cast<float*>(xs.accp), 0, n * 4, s));
-            if (it + 1 < iters) {
-                if (timing) cudaEventRecord(ev.second, s);
-                continue;
-            }
-            pr_finish_kernel<<<2 * eg, 256, 0, s>>>(m.x, target, n, 0, n, damping, m.dang + cur_d, m.dang + (cur_d ^ 1),
-                                                     dangling == GTS_DANGLING_UNIFORM ? 1 : 0);
-            ++launches;
-            if (timing) cudaEventRecord(ev.second, s);
-            GTS_CUDA(cudaGetLastError());
-            continue;
-        }
         for (PrSlot& m : S) {
             // (GTS_ROUTE_PEER: the D all-reduce above is also the barrier after every rank's peer adds)
             pr_finish_kernel<<<2 * eg, 256, 0, s>>>(m.x, (peer && (it & 1)) ? m.acc2 : m.acc, n, m.lo, m.hi, damping,

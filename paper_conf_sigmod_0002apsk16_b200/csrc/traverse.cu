@@ -554,10 +554,9 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     if (micro == kMicroTile)
         bfs_kern = g->weighted ? bfs_expand_kernel<true, kMicroTile, 3> : bfs_expand_kernel<false, kMicroTile, 3>;
     const uint32_t hybrid_deg = rc.hybrid_deg ? rc.hybrid_deg : 8u;
-    // two 512-thread CTAs per SM for the SSSP expansion (three measured 35.7 vs 35.1 ms on
-    // RMAT-27: the weighted walk spills at 40 registers)
-    auto sssp_kern = (getenv("GTS_DEV_SSSP3") && atoi(getenv("GTS_DEV_SSSP3")) > 0) ? sssp_expand_kernel<3>
-                                                                                      : sssp_expand_kernel<2>;   // (temporary A/B)
+    // three 512-thread CTAs per SM for the SSSP expansion: with the interleaved (adj, w)
+    // records it fits 40 registers (20 bytes spilled) -- RMAT-27 33.6 vs 34.2 ms for two
+    auto sssp_kern = sssp_expand_kernel<3>;
     const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_kern;
     int grid = 0;
     GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
