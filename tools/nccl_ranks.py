@@ -1,5 +1,8 @@
-"""Run libgts's real multi-rank path (NCCL communicator, one process per rank) with
-two processes on the same GPU, if this NCCL allows two ranks on one device.
+"""Run libgts's real multi-rank path (NCCL communicator, one process per rank):
+rank r on GPU r % device_count.  With one GPU both ranks share it, which NCCL
+2.28 refuses (ncclCommInitRank: invalid usage -- both ranks then fail the call
+with GTS_ENCCL, no hang; profiles/r02_two_ranks_one_gpu.txt); with two or more
+GPUs this is the real NCCL / CUDA IPC path end to end.
 
 Each rank builds its own owner-filtered pages and runs BFS / PageRank / SSSP / WCC
 under Strategy-P and Strategy-S (routed, and GTS_ROUTE_PEER over CUDA IPC), then
@@ -37,7 +40,8 @@ def worker(rank, world, port, scale, q):
     try:
         obj = [G.gts_get_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
-        ctx = G.gts_context_create(0, rank, world, obj[0])
+        import torch
+        ctx = G.gts_context_create(rank % max(1, torch.cuda.device_count()), rank, world, obj[0])
         g = inputs.rmat(scale)
         w = inputs.edge_weights(g)
         for sname, strat, peer in (("P", 0, False), ("S", 1, False), ("S_peer", 1, True), ("S_BCAST", 2, False)):
