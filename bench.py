@@ -19,6 +19,7 @@ the host cores as the reference arm (rank 0 only).
 from __future__ import annotations
 
 import argparse
+import gc
 import json
 import os
 import subprocess
@@ -98,6 +99,7 @@ class ClockSampler:
             log("NVML unavailable:", e)
             return
         self.nv = pynvml
+        self.sample_s = []
         self.h = pynvml.nvmlDeviceGetHandleByIndex(self.device)
         self.stop_ev = threading.Event()
         self.kick_ev = threading.Event() if kicked else None
@@ -115,8 +117,10 @@ class ClockSampler:
                         continue
                     self.kick_ev.clear()
                     time.sleep(0.01)          # inside the PageRank call
+                t0 = time.perf_counter()
                 sm = pynvml.nvmlDeviceGetClockInfo(self.h, pynvml.NVML_CLOCK_SM)
                 r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                self.sample_s.append(time.perf_counter() - t0)
                 act = ["Active" if r & b else "Not Active" for b in bits.values()]
                 self.lines.append(", ".join([str(sm), str(mx), "0", hex(r)] + act))
                 if self.kick_ev is None:
@@ -151,8 +155,11 @@ class ClockSampler:
             for nm, v in zip(names, f[4:8]):
                 if v.lower() == "active":
                     reasons.add(nm)
-        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+        out = {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+               "reasons": sorted(reasons), "samples": len(sm)}
+        if getattr(self, "sample_s", None):
+            out["nvml_query_ms_max"] = round(1e3 * max(self.sample_s), 3)
+        return out
 
 
 # --------------------------------------------------------------------- reference arm ---
@@ -469,6 +476,10 @@ def main():
             sampler.kick()
             _step(record)
     rec = {}
+    # no cyclic-GC pause inside the timed region (a collection between two calls would idle
+    # the GPU while the host is stopped)
+    gc.collect()
+    gc.disable()
     barrier()
     t_start = torch.cuda.Event(enable_timing=True)
     t_end = torch.cuda.Event(enable_timing=True)
@@ -477,6 +488,7 @@ def main():
         step(rec)
     t_end.record(stream)
     barrier()
+    gc.enable()
     clocks = sampler.stop()
     total_s = t_start.elapsed_time(t_end) * 1e-3
 

@@ -161,6 +161,13 @@ struct dense8_of<Op, std::void_t<decltype(Op::kDense8)>> : std::integral_constan
 template <class Op>
 __device__ __forceinline__ constexpr uint32_t dense_eighths() { return dense8_of<Op>::value; }
 
+// An op with kSparseSelect = true also filters the frontier vertices of sparse pages
+// through select() (default: the frontier bit alone selects them there).
+template <class Op, class = void>
+struct sparse_select_of : std::false_type {};
+template <class Op>
+struct sparse_select_of<Op, std::void_t<decltype(Op::kSparseSelect)>> : std::integral_constant<bool, Op::kSparseSelect> {};
+
 // Edge-parallel expansion of nf compacted items (sm.off/deg/src/payload/pre):
 // 4 consecutive edges per thread, one binary search per 4 edges.
 template <class Op>
@@ -231,10 +238,10 @@ __device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, cons
         __syncthreads();
         for (uint32_t b0 = 0; b0 < tot; b0 += kTile) {
             const uint32_t kk = b0 + tid;
-            const bool sel = kk < tot;
-            uint32_t j = 0, off = 0, deg = 0;
+            bool sel = kk < tot;
+            uint32_t j = sel ? sm.list[kk] : 0u, off = 0, deg = 0;
+            if constexpr (sparse_select_of<Op>::value) sel = sel && op.select(start + j);
             if (sel) {
-                j = sm.list[kk];
                 const uint8_t* slot = end - kSpFooter - kSlotBytes * (uint64_t)(j + 1);
                 off = ld_stream_u32(slot + 4, pol);
                 deg = ld_stream_u32(data + off, pol) ;

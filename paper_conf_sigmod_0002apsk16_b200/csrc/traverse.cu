@@ -44,6 +44,8 @@ struct BfsOp {
     uint32_t* next;
     unsigned long long nedges;
     uint32_t vprefix;          // every vertex below this ID is already visited (no test needed)
+    const uint32_t* vhead;     // shared-memory copy of visited words [0, hv_words) taken at launch
+    uint32_t hv_bits;          // 32 * hv_words (0 = no copy)
     __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
@@ -66,8 +68,13 @@ struct BfsOp {
                                           const bool* valid) {
         uint32_t vis[kEdgesPerThread];
 #pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q)
-            vis[q] = (valid[q] && dst[q] >= vprefix) ? __ldca(visited + (dst[q] >> 5)) : ~0u;
+        for (int q = 0; q < kEdgesPerThread; ++q) {
+            // bits only go 0 -> 1 during a level, so a bit set in the launch-time copy is
+            // set in visited; a clear one is re-tested in global memory
+            const bool probe = valid[q] && dst[q] >= vprefix &&
+                               !(dst[q] < hv_bits && ((vhead[dst[q] >> 5] >> (dst[q] & 31)) & 1u));
+            vis[q] = probe ? __ldca(visited + (dst[q] >> 5)) : ~0u;
+        }
 #pragma unroll
         for (int q = 0; q < kEdgesPerThread; ++q) {
             const uint32_t wi = dst[q] >> 5, b = 1u << (dst[q] & 31);
@@ -83,17 +90,30 @@ template <bool W>
 struct SsspOp {
     static constexpr bool kReadWeights = true;
     static constexpr bool kWeighted = W;
+    static constexpr bool kSparseSelect = true;   // sparse pages also call select() (expand.cuh)
     const uint32_t* cur;
     uint32_t* dist;
     uint32_t* next;
     unsigned long long nedges;
     bool ovf;
     uint32_t T;                // near-far threshold: only pending vertices with dist <= T are expanded
+    // dexp[v] = the distance v's out-edges were last relaxed with (UNREACHED = never).  A
+    // pending vertex whose distance has not dropped below it was improved earlier in the
+    // round it was expanded in, after which its expansion already used the improved value:
+    // expanding it again relaxes nothing.  nullptr = off.  SP vertices only: the slices of
+    // an LP vertex run in several CTAs and each must see the same selection.
+    uint32_t* dexp;
     __device__ const uint32_t* frontier() const { return cur; }
-    __device__ bool select(uint32_t v) { return test_bit(cur, v) && __ldcg(dist + v) <= T; }
+    __device__ bool select(uint32_t v) {
+        if (!test_bit(cur, v)) return false;
+        const uint32_t d = __ldcg(dist + v);
+        return d <= T && (!dexp || d < __ldcg(dexp + v));
+    }
     __device__ uint32_t payload(uint32_t v, uint32_t deg) {
         nedges += deg;
-        return *((volatile uint32_t*)dist + v);
+        const uint32_t d = *((volatile uint32_t*)dist + v);
+        if (dexp) __stcg(dexp + v, d);
+        return d;
     }
     __device__ bool select_lp(uint32_t vid, uint32_t, uint32_t len, uint32_t& pl) {
         if (!test_bit(cur, vid)) return false;
@@ -152,16 +172,23 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 
 // -------------------------------------------------------------- kernels ---
 
+constexpr uint32_t kVisitedHeadWords = 8192;   // 32 KB: vertices [0, 262144)
+
 template <bool W, int M = kMicroTile, int MB = 2>
 __global__ void __launch_bounds__(kThreads, MB)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
                   uint32_t* work_ctr, unsigned long long* edges_out, const unsigned int* vprefix_words,
-                  uint64_t n) {
+                  uint64_t n, uint32_t hv_words) {
     __shared__ TileSmem sm;
+    // head of the visited bitmap (degree-ordered pages: the most probed words), copied once
+    // per CTA at launch; hv_words = 0: no copy
+    extern __shared__ __align__(16) uint32_t vhead[];           // hv_words (dynamic)
     // all-visited prefix from the previous level's visited_prefix_kernel (device-side,
     // so levels can be enqueued without a host round trip)
     const uint64_t vw = min((uint64_t)*vprefix_words, (n + 31) / 32);
-    BfsOp<W> op{cur, visited, next, 0ull, (uint32_t)min(vw * 32, n)};
+    for (uint32_t k = threadIdx.x; k < hv_words; k += kThreads) vhead[k] = __ldcg(visited + k);
+    __syncthreads();
+    BfsOp<W> op{cur, visited, next, 0ull, (uint32_t)min(vw * 32, n), vhead, 32u * hv_words};
     expand_pages<BfsOp<W>, M>(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
@@ -169,9 +196,9 @@ bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visite
 template <int MB = 2>
 __global__ void __launch_bounds__(kThreads, MB)
 sssp_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* dist, uint32_t* next,
-                   uint32_t* work_ctr, unsigned long long* edges_out, uint32_t* ovf_flag, uint32_t T) {
+                   uint32_t* work_ctr, unsigned long long* edges_out, uint32_t* ovf_flag, uint32_t T, uint32_t* dexp) {
     __shared__ TileSmem sm;
-    SsspOp<true> op{cur, dist, next, 0ull, false, T};
+    SsspOp<true> op{cur, dist, next, 0ull, false, T, dexp};
     expand_pages(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
     if (__syncthreads_or(op.ovf) && threadIdx.x == 0) *ovf_flag = 1u;
@@ -440,7 +467,8 @@ struct Counters {               // device scratch, slot kCtr
     unsigned int vprefix_words;    // BFS: all-visited prefix of the bitmap (words)
 };
 
-enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather, kBufLvSlots, kBufLv8, kBufLvCnt };
+enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather, kBufLvSlots, kBufLv8, kBufLvCnt,
+       kBufDexp };
 
 // deliver() for byte levels of a degree-ordered graph: out[v] = lv8[new_of_old[v]]
 static int deliver_levels8(Context* c, const Graph* g, const uint8_t* lv8, bool nibbles, void* out,
@@ -504,6 +532,11 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     GTS_TRY(c->buf(kBufList, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&list));
     GTS_TRY(c->buf(kBufCtr, sizeof(Counters), (void**)&ctr));
     cudaStream_t s = c->stream;
+    uint32_t* dexp = nullptr;            // SSSP: distance of each vertex's last expansion (SsspOp)
+    if (algo == kSSSP) {     // RMAT-27: 4.51 G -> 3.12 G relaxed edges, kernels 33.1 -> 26.1 ms
+        GTS_TRY(c->buf(kBufDexp, n * 4, (void**)&dexp));
+        GTS_CUDA(cudaMemsetAsync(dexp, 0xFF, n * 4, s));
+    }
     // BFS level slots: the frontier of level L lives in slot L of a K-slot bitmap
     // store, and LV is written once at the end by level_fill_kernel.  A traversal
     // deeper than K levels fills LV from the slots and continues with the
@@ -554,12 +587,16 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     if (micro == kMicroTile)
         bfs_kern = g->weighted ? bfs_expand_kernel<true, kMicroTile, 3> : bfs_expand_kernel<false, kMicroTile, 3>;
     const uint32_t hybrid_deg = rc.hybrid_deg ? rc.hybrid_deg : 8u;
+    const uint32_t hv_want = getenv("GTS_DEV_VHEAD") ? (uint32_t)atoi(getenv("GTS_DEV_VHEAD")) : kVisitedHeadWords;
+    const uint32_t hv_words = (algo == kBFS && g->ordered && micro == kMicroTile)
+                                  ? (uint32_t)std::min<uint64_t>(hv_want, words) : 0u;
     // three 512-thread CTAs per SM for the SSSP expansion: with the interleaved (adj, w)
     // records it fits 40 registers (20 bytes spilled) -- RMAT-27 33.6 vs 34.2 ms for two
     auto sssp_kern = sssp_expand_kernel<3>;
     const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_kern;
+    if (hv_words) GTS_CUDA(cudaFuncSetAttribute(kexp, cudaFuncAttributeMaxDynamicSharedMemorySize, hv_words * 4));
     int grid = 0;
-    GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
+    GTS_TRY(sms_grid(c, kexp, kThreads, hv_words * 4, &grid));
     const int fin_grid = c->num_sms * 4;
     uint64_t pages_processed = l0.size();
     uint32_t levels = 0;
@@ -625,11 +662,12 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
                                 p2.split = 0u;
                                 const int gl = std::min(grid, cap);
                                 if (algo == kBFS) {
-                                    bfs_kern<<<gl, kThreads, 0, s>>>(
-                                        p2, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n);
+                                    bfs_kern<<<gl, kThreads, hv_words * 4, s>>>(
+                                        p2, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n,
+                                        hv_words);
                                 } else
                                     sssp_kern<<<gl, kThreads, 0, s>>>(
-                                        p2, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T);
+                                        p2, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T, dexp);
                                 if (timing) cudaEventRecord(ev.second, s);
                                 GTS_CUDA(cudaGetLastError());
                                 ++main_launches;
@@ -1651,8 +1689,8 @@ static int betweenness(gts_context* c, const gts_graph* g, const uint64_t* sourc
                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n);
-                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n);
+                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, 0u);
+                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, 0u);
                 if (timing) cudaEventRecord(ev.second, s);
                 GTS_CUDA(cudaGetLastError());
                 ++main_launches;

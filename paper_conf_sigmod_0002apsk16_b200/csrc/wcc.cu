@@ -267,7 +267,7 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
         GTS_TRY(c->buf(L == 1 ? kBufWccCtr : kBufWccMulti + 4 * i + 2, 8, (void**)&ctr[i]));
         wcc_init_kernel<<<eg, 256, 0, s>>>(label[i], n);
     }
-    GTS_CUDA(cudaStreamSynchronize(s));
+    GTS_CUDA(cudaGetLastError());
     // three 512-thread CTAs per SM for the sweep (40 registers; RMAT-27 sweep 17.4 -> 14.6 ms
     // against two: the third CTA covers the per-tile barriers)
     auto sweep_k = g->weighted ? wcc_sweep_kernel<true, 3> : wcc_sweep_kernel<false, 3>;
