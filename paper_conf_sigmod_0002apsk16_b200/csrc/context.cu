@@ -207,6 +207,12 @@ bool choose_streamed(Context* c, const Graph* g, const gts_run_config& rc, uint6
     if (rc.residency == GTS_STREAMED) return true;
     if (rc.residency == GTS_RESIDENT) return false;
     if (c->dg.uid == g->uid && c->dg.resident) return false;
+    // a parked resident copy comes back without an upload (ensure_graph).  (cudaMemGetInfo
+    // below measured 1-27 ms per call on B200: asked on every switch between two graphs, it
+    // was the per-call outliers of SSSP and WCC in the bench step, tools/call_jitter.py)
+    uint32_t strat_key = c->world > 1 ? rc.strategy : 0;
+    for (const DevGraph& p : c->parked)
+        if (p.uid == g->uid && p.resident && p.strategy == strat_key && p.world == c->world) return false;
     size_t free_b = 0, total_b = 0;
     if (cudaMemGetInfo(&free_b, &total_b) != cudaSuccess) {
         cudaGetLastError();

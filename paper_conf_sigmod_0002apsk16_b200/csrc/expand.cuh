@@ -168,6 +168,54 @@ struct sparse_select_of : std::false_type {};
 template <class Op>
 struct sparse_select_of<Op, std::void_t<decltype(Op::kSparseSelect)>> : std::integral_constant<bool, Op::kSparseSelect> {};
 
+// An op with kFastDense = true may take the plain dense walk below: a dense tile whose
+// vertices with edges all satisfy op.done(v) (expanding any of their edges changes
+// nothing the level computes) is streamed without owners or selection, and only words
+// >= op.fast_floor() reach op.edges.  Record headers are never below the floor when
+// fast_floor() >= page_bytes / 4 (an SP record has fewer entries than that), so they
+// need no record-start mask either.
+template <class Op, class = void>
+struct fast_dense_of : std::false_type {};
+template <class Op>
+struct fast_dense_of<Op, std::void_t<decltype(Op::kFastDense)>> : std::integral_constant<bool, Op::kFastDense> {};
+
+constexpr int kFastUnroll = 4;       // 16-byte loads in flight per lane in the plain dense walk
+
+// Plain dense walk (kFastDense ops, unweighted VID32 pages): window i of the tile's record
+// region goes to warp i mod kWarps, one 16-byte load per lane.
+template <class Op>
+__device__ __forceinline__ void dense_tile_plain(Op& op, const uint4* q4, uint32_t W0, uint32_t W1, uint32_t floor,
+                                                 uint64_t pol) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t wbase = W0 & ~3u;
+    const uint32_t nwin = (W1 - wbase + 127) >> 7;
+    for (uint32_t wi = warp; wi < nwin; wi += kWarps * kFastUnroll) {
+        uint4 vv[kFastUnroll];
+#pragma unroll
+        for (int u = 0; u < kFastUnroll; ++u) {
+            const uint32_t q = ((wbase + ((wi + u * kWarps) << 7)) >> 2) + lane;
+            vv[u] = make_uint4(0u, 0u, 0u, 0u);
+            if (wi + u * kWarps < nwin && 4 * q < W1) vv[u] = ld_stream_v4(q4 + q, pol);
+        }
+#pragma unroll
+        for (int u = 0; u < kFastUnroll; ++u) {
+            const uint32_t q = ((wbase + ((wi + u * kWarps) << 7)) >> 2) + lane;
+            uint32_t dst[kEdgesPerThread], wt[kEdgesPerThread] = {0u, 0u, 0u, 0u}, pl[kEdgesPerThread] = {0u, 0u, 0u, 0u},
+                     src[kEdgesPerThread] = {0u, 0u, 0u, 0u};
+            bool valid[kEdgesPerThread];
+            bool any = false;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const uint32_t w = 4 * q + k;
+                dst[k] = word_of(vv[u], k);
+                valid[k] = dst[k] >= floor && w >= W0 && w < W1;
+                any |= valid[k];
+            }
+            if (any) op.edges(dst, wt, pl, src, valid);
+        }
+    }
+}
+
 // Edge-parallel expansion of nf compacted items (sm.off/deg/src/payload/pre):
 // 4 consecutive edges per thread, one binary search per 4 edges.
 template <class Op>
@@ -448,6 +496,11 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
     const uint32_t count = npages * S;
     const int tid = threadIdx.x;
     const uint64_t pol = policy_evict_first();
+    uint32_t ffloor = 0;                 // plain dense walk: probe floor (0 = not this launch)
+    if constexpr (fast_dense_of<Op>::value) {
+        ffloor = op.fast_floor();
+        if (ffloor < ps.page_bytes / 4 || ps.entry_encoding != GTS_ENTRY_VID32) ffloor = 0;
+    }
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
         __syncthreads();
@@ -574,6 +627,14 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 // 35.7 ms vs 42.8 ms when the selected words are counted instead; with the
                 // interleaved (adj, w) records 33.5 vs 35.3 ms)
                 const bool dense = 8 * total >= dense_eighths<Op>() * (W1 - W0);
+                if constexpr (fast_dense_of<Op>::value) {
+                    if (ffloor && 8 * total >= op.plain8 * (W1 - W0) &&
+                        __syncthreads_and((uint32_t)tid >= nv || deg == 0 || op.done(v))) {
+                        dense_tile_plain(op, q4, W0, W1, ffloor, pol);
+                        __syncthreads();
+                        continue;
+                    }
+                }
                 if (dense) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
                     // 128-word windows; owners from record-start masks (no binary search;

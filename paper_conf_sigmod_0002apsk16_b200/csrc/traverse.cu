@@ -38,14 +38,21 @@ template <bool W>
 struct BfsOp {
     static constexpr bool kReadWeights = false;
     static constexpr bool kWeighted = W;
+    static constexpr bool kFastDense = !W;    // plain dense walk (expand.cuh dense_tile_plain)
     static constexpr uint32_t kDense8 = 6;    // dense tiles only at >= 3/4 selected (expand.cuh)
     const uint32_t* cur;
     uint32_t* visited;
     uint32_t* next;
     unsigned long long nedges;
     uint32_t vprefix;          // every vertex below this ID is already visited (no test needed)
-    const uint32_t* vhead;     // shared-memory copy of visited words [0, hv_words) taken at launch
-    uint32_t hv_bits;          // 32 * hv_words (0 = no copy)
+    // visited at the start of this level (levels <= the frontier's), nullptr = none: every
+    // out-neighbour of such a vertex is already visited (BFS levels differ by at most one
+    // along an edge), so expanding its edges discovers nothing -- a dense tile of such
+    // vertices can be streamed without selecting the frontier's records
+    const uint32_t* vstart;
+    uint32_t plain8;           // plain walk when the tile's selected edges are >= plain8/8 of its words
+    __device__ uint32_t fast_floor() const { return vstart ? vprefix : 0u; }
+    __device__ bool done(uint32_t v) const { return test_bit(vstart, v); }
     __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
@@ -68,13 +75,8 @@ struct BfsOp {
                                           const bool* valid) {
         uint32_t vis[kEdgesPerThread];
 #pragma unroll
-        for (int q = 0; q < kEdgesPerThread; ++q) {
-            // bits only go 0 -> 1 during a level, so a bit set in the launch-time copy is
-            // set in visited; a clear one is re-tested in global memory
-            const bool probe = valid[q] && dst[q] >= vprefix &&
-                               !(dst[q] < hv_bits && ((vhead[dst[q] >> 5] >> (dst[q] & 31)) & 1u));
-            vis[q] = probe ? __ldca(visited + (dst[q] >> 5)) : ~0u;
-        }
+        for (int q = 0; q < kEdgesPerThread; ++q)
+            vis[q] = (valid[q] && dst[q] >= vprefix) ? __ldca(visited + (dst[q] >> 5)) : ~0u;
 #pragma unroll
         for (int q = 0; q < kEdgesPerThread; ++q) {
             const uint32_t wi = dst[q] >> 5, b = 1u << (dst[q] & 31);
@@ -172,23 +174,16 @@ __device__ __forceinline__ void block_add_u64(unsigned long long v, unsigned lon
 
 // -------------------------------------------------------------- kernels ---
 
-constexpr uint32_t kVisitedHeadWords = 8192;   // 32 KB: vertices [0, 262144)
-
 template <bool W, int M = kMicroTile, int MB = 2>
 __global__ void __launch_bounds__(kThreads, MB)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
                   uint32_t* work_ctr, unsigned long long* edges_out, const unsigned int* vprefix_words,
-                  uint64_t n, uint32_t hv_words) {
+                  uint64_t n, const uint32_t* vstart, uint32_t plain8) {
     __shared__ TileSmem sm;
-    // head of the visited bitmap (degree-ordered pages: the most probed words), copied once
-    // per CTA at launch; hv_words = 0: no copy
-    extern __shared__ __align__(16) uint32_t vhead[];           // hv_words (dynamic)
     // all-visited prefix from the previous level's visited_prefix_kernel (device-side,
     // so levels can be enqueued without a host round trip)
     const uint64_t vw = min((uint64_t)*vprefix_words, (n + 31) / 32);
-    for (uint32_t k = threadIdx.x; k < hv_words; k += kThreads) vhead[k] = __ldcg(visited + k);
-    __syncthreads();
-    BfsOp<W> op{cur, visited, next, 0ull, (uint32_t)min(vw * 32, n), vhead, 32u * hv_words};
+    BfsOp<W> op{cur, visited, next, 0ull, (uint32_t)min(vw * 32, n), vstart, plain8};
     expand_pages<BfsOp<W>, M>(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
@@ -468,7 +463,7 @@ struct Counters {               // device scratch, slot kCtr
 };
 
 enum { kBufValue = 0, kBufVisited, kBufCur, kBufNext, kBufList, kBufCtr, kBufGather, kBufLvSlots, kBufLv8, kBufLvCnt,
-       kBufDexp };
+       kBufDexp, kBufVstart };
 
 // deliver() for byte levels of a degree-ordered graph: out[v] = lv8[new_of_old[v]]
 static int deliver_levels8(Context* c, const Graph* g, const uint8_t* lv8, bool nibbles, void* out,
@@ -532,6 +527,13 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     GTS_TRY(c->buf(kBufList, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&list));
     GTS_TRY(c->buf(kBufCtr, sizeof(Counters), (void**)&ctr));
     cudaStream_t s = c->stream;
+    // BFS, unweighted degree-ordered pages: visited as of the start of each level, for the
+    // plain dense walk (BfsOp::vstart; written after each level's visited_prefix_kernel, so
+    // it is valid whenever that level's all-visited prefix is large enough to enable the walk)
+    uint32_t* vstart = nullptr;
+    if (algo == kBFS && g->ordered && !g->weighted && !getenv("GTS_DEV_NO_PLAIN"))
+        GTS_TRY(c->buf(kBufVstart, words * 4, (void**)&vstart));
+    const uint32_t plain8 = getenv("GTS_DEV_PLAIN8") ? (uint32_t)atoi(getenv("GTS_DEV_PLAIN8")) : 6u;
     uint32_t* dexp = nullptr;            // SSSP: distance of each vertex's last expansion (SsspOp)
     if (algo == kSSSP) {     // RMAT-27: 4.51 G -> 3.12 G relaxed edges, kernels 33.1 -> 26.1 ms
         GTS_TRY(c->buf(kBufDexp, n * 4, (void**)&dexp));
@@ -587,16 +589,12 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     if (micro == kMicroTile)
         bfs_kern = g->weighted ? bfs_expand_kernel<true, kMicroTile, 3> : bfs_expand_kernel<false, kMicroTile, 3>;
     const uint32_t hybrid_deg = rc.hybrid_deg ? rc.hybrid_deg : 8u;
-    const uint32_t hv_want = getenv("GTS_DEV_VHEAD") ? (uint32_t)atoi(getenv("GTS_DEV_VHEAD")) : kVisitedHeadWords;
-    const uint32_t hv_words = (algo == kBFS && g->ordered && micro == kMicroTile)
-                                  ? (uint32_t)std::min<uint64_t>(hv_want, words) : 0u;
     // three 512-thread CTAs per SM for the SSSP expansion: with the interleaved (adj, w)
     // records it fits 40 registers (20 bytes spilled) -- RMAT-27 33.6 vs 34.2 ms for two
     auto sssp_kern = sssp_expand_kernel<3>;
     const void* kexp = algo == kBFS ? (const void*)bfs_kern : (const void*)sssp_kern;
-    if (hv_words) GTS_CUDA(cudaFuncSetAttribute(kexp, cudaFuncAttributeMaxDynamicSharedMemorySize, hv_words * 4));
     int grid = 0;
-    GTS_TRY(sms_grid(c, kexp, kThreads, hv_words * 4, &grid));
+    GTS_TRY(sms_grid(c, kexp, kThreads, 0, &grid));
     const int fin_grid = c->num_sms * 4;
     uint64_t pages_processed = l0.size();
     uint32_t levels = 0;
@@ -662,9 +660,9 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
                                 p2.split = 0u;
                                 const int gl = std::min(grid, cap);
                                 if (algo == kBFS) {
-                                    bfs_kern<<<gl, kThreads, hv_words * 4, s>>>(
+                                    bfs_kern<<<gl, kThreads, 0, s>>>(
                                         p2, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n,
-                                        hv_words);
+                                        vstart, plain8);
                                 } else
                                     sssp_kern<<<gl, kThreads, 0, s>>>(
                                         p2, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T, dexp);
@@ -687,6 +685,7 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
             GTS_CUDA(cudaMemsetAsync(&ctr->vprefix_words, 0xFF, 4, s));
             visited_prefix_kernel<<<fin_grid, 256, 0, s>>>(visited, words, &ctr->vprefix_words);
             ++launches;
+            if (vstart) GTS_CUDA(cudaMemcpyAsync(vstart, visited, words * 4, cudaMemcpyDeviceToDevice, s));
         } else {
             GTS_CUDA(cudaMemsetAsync(&ctr->near, 0, 8, s));
             GTS_CUDA(cudaMemsetAsync(&ctr->minpend, 0xFF, 4, s));
@@ -1689,8 +1688,8 @@ static int betweenness(gts_context* c, const gts_graph* g, const uint64_t* sourc
                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, 0u);
-                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, 0u);
+                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, nullptr, 8u);
+                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, nullptr, 8u);
                 if (timing) cudaEventRecord(ev.second, s);
                 GTS_CUDA(cudaGetLastError());
                 ++main_launches;

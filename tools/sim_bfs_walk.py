@@ -77,8 +77,14 @@ def main():
         dw = 0
         noflag = 0
         maxlane_sum = 0
+        allsel_e = 0
+        dense_e = 0
         for t in np.nonzero(dense)[0]:
             v0, v1 = t * T, min(n, (t + 1) * T)
+            has = ideg[v0:v1] > 0
+            dense_e += int(sel_e[v0:v1].sum())
+            if np.all(visited[v0:v1][has]):        # every vertex with edges visited: no selection needed
+                allsel_e += int(sel_e[v0:v1].sum())
             W0, W1 = woff[v0], woff[v1]
             words = np.zeros(W1 - W0, bool)
             e0, e1 = irow[v0], irow[v1]
@@ -104,7 +110,9 @@ def main():
         spf = int((sp_e & (icol >= vp)).sum())
         print(f"{L:3d} {len(fv):9d} {vp:9d} {int(sel_e.sum()):10d} {100 * nflag / max(1, sel_e.sum()):8.1f} "
               f"{int(dense.sum()):8d} {int(sparse.sum()):8d} {dw:10d} {100 * noflag / max(1, dw):12.1f} "
-              f"{maxlane_sum / max(1, dw):11.2f} {spn:13d} {100 * spf / max(1, spn):12.1f}")
+              f"{maxlane_sum / max(1, dw):11.2f} {spn:13d} {100 * spf / max(1, spn):12.1f}  "
+              f"dense_e {dense_e} all_visited_e {allsel_e} ({100 * allsel_e / max(1, dense_e):.1f}%) "
+              f"maxdeg {int(ideg.max())}")
         # next level
         nb = icol[np.repeat(front, ideg)]
         nxt = np.zeros(n, bool)
