@@ -168,12 +168,13 @@ struct sparse_select_of : std::false_type {};
 template <class Op>
 struct sparse_select_of<Op, std::void_t<decltype(Op::kSparseSelect)>> : std::integral_constant<bool, Op::kSparseSelect> {};
 
-// An op with kFastDense = true may take the plain dense walk below: a dense tile whose
+// An op with kFastDense = true may take the plain dense walk below: a tile whose
 // vertices with edges all satisfy op.done(v) (expanding any of their edges changes
 // nothing the level computes) is streamed without owners or selection, and only words
-// >= op.fast_floor() reach op.edges.  Record headers are never below the floor when
-// fast_floor() >= page_bytes / 4 (an SP record has fewer entries than that), so they
-// need no record-start mask either.
+// >= op.fast_floor() reach op.edges, as edges of the vertex op.plain_src() (payload
+// and source alike).  An unweighted record's header is its entry count,
+// so when every record of the tile has fewer entries than the floor the headers are
+// filtered out with the rest and no record-start mask is needed either.
 template <class Op, class = void>
 struct fast_dense_of : std::false_type {};
 template <class Op>
@@ -200,8 +201,9 @@ __device__ __forceinline__ void dense_tile_plain(Op& op, const uint4* q4, uint32
 #pragma unroll
         for (int u = 0; u < kFastUnroll; ++u) {
             const uint32_t q = ((wbase + ((wi + u * kWarps) << 7)) >> 2) + lane;
-            uint32_t dst[kEdgesPerThread], wt[kEdgesPerThread] = {0u, 0u, 0u, 0u}, pl[kEdgesPerThread] = {0u, 0u, 0u, 0u},
-                     src[kEdgesPerThread] = {0u, 0u, 0u, 0u};
+            const uint32_t ps0 = op.plain_src();
+            uint32_t dst[kEdgesPerThread], wt[kEdgesPerThread] = {0u, 0u, 0u, 0u}, pl[kEdgesPerThread] = {ps0, ps0, ps0, ps0},
+                     src[kEdgesPerThread] = {ps0, ps0, ps0, ps0};
             bool valid[kEdgesPerThread];
             bool any = false;
 #pragma unroll
@@ -499,7 +501,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
     uint32_t ffloor = 0;                 // plain dense walk: probe floor (0 = not this launch)
     if constexpr (fast_dense_of<Op>::value) {
         ffloor = op.fast_floor();
-        if (ffloor < ps.page_bytes / 4 || ps.entry_encoding != GTS_ENTRY_VID32) ffloor = 0;
+        if (ps.entry_encoding != GTS_ENTRY_VID32) ffloor = 0;
     }
     for (;;) {
         if (tid == 0) sm.item = atomicAdd(work_ctr, 1u);
@@ -629,7 +631,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 const bool dense = 8 * total >= dense_eighths<Op>() * (W1 - W0);
                 if constexpr (fast_dense_of<Op>::value) {
                     if (ffloor && 8 * total >= op.plain8 * (W1 - W0) &&
-                        __syncthreads_and((uint32_t)tid >= nv || deg == 0 || op.done(v))) {
+                        __syncthreads_and((uint32_t)tid >= nv || deg == 0 || (deg < ffloor && op.done(v)))) {
                         dense_tile_plain(op, q4, W0, W1, ffloor, pol);
                         __syncthreads();
                         continue;

@@ -78,7 +78,23 @@ __device__ __forceinline__ void gather_x4(uint32_t* out, const uint32_t* __restr
     const uint64_t n4 = n >> 2;
     const uint4* idx4 = reinterpret_cast<const uint4*>(idx);
     uint4* out4 = reinterpret_cast<uint4*>(out);
-    for (uint64_t q = t; q < n4; q += stride) {
+    // two 16-byte index loads, then eight random reads, in flight per thread
+    uint64_t q = t;
+    for (; q + stride < n4; q += 2 * stride) {
+        const uint4 i = __ldcs(idx4 + q), j = __ldcs(idx4 + q + stride);
+        uint4 o, p;
+        o.x = f(i.x);
+        o.y = f(i.y);
+        o.z = f(i.z);
+        o.w = f(i.w);
+        p.x = f(j.x);
+        p.y = f(j.y);
+        p.z = f(j.z);
+        p.w = f(j.w);
+        __stcs(out4 + q, o);
+        __stcs(out4 + q + stride, p);
+    }
+    if (q < n4) {
         const uint4 i = __ldcs(idx4 + q);
         uint4 o;
         o.x = f(i.x);

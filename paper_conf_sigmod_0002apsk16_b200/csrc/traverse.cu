@@ -53,6 +53,7 @@ struct BfsOp {
     uint32_t plain8;           // plain walk when the tile's selected edges are >= plain8/8 of its words
     __device__ uint32_t fast_floor() const { return vstart ? vprefix : 0u; }
     __device__ bool done(uint32_t v) const { return test_bit(vstart, v); }
+    __device__ uint32_t plain_src() const { return 0u; }
     __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
@@ -216,7 +217,7 @@ sssp_check_kernel(PageSet ps, const uint32_t* __restrict__ dist, uint32_t* work_
 // reached vertex when level != nullptr.
 __global__ void frontier_finish_kernel(const uint32_t* __restrict__ gathered, int world, uint64_t gwords, uint64_t w0,
                                        uint64_t w1, uint32_t* next, uint32_t* visited, uint32_t* level,
-                                       uint32_t new_level, unsigned long long* count) {
+                                       uint32_t new_level, unsigned long long* count, uint32_t* vstart = nullptr) {
     unsigned long long c = 0;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t w = w0 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < w1; w += stride) {
@@ -230,6 +231,7 @@ __global__ void frontier_finish_kernel(const uint32_t* __restrict__ gathered, in
             bits = next[w];
         }
         c += __popc(bits);
+        if (vstart && bits) vstart[w] |= bits;    // visited as of the next level's start
         if (level) {
             while (bits) {
                 const int b = __ffs(bits) - 1;
@@ -527,13 +529,20 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     GTS_TRY(c->buf(kBufList, std::max<uint64_t>(g->num_pages, 1) * 4, (void**)&list));
     GTS_TRY(c->buf(kBufCtr, sizeof(Counters), (void**)&ctr));
     cudaStream_t s = c->stream;
+    // micro-level technique inside each page (GTS_MICRO_*, App E): BFS only
+    uint32_t micro = (rc.flags & GTS_MICRO_MASK) >> 8;
+    if (micro == (GTS_MICRO_TILE >> 8)) micro = kMicroTile;
+    if (micro > kMicroHybrid) return fail(GTS_EINVAL, "unknown GTS_MICRO value");
+    if (algo == kSSSP && micro) return fail(GTS_EUNSUPPORTED, "GTS_MICRO_* techniques apply to gts_bfs and gts_pagerank");
     // BFS, unweighted degree-ordered pages: visited as of the start of each level, for the
-    // plain dense walk (BfsOp::vstart; written after each level's visited_prefix_kernel, so
-    // it is valid whenever that level's all-visited prefix is large enough to enable the walk)
+    // plain dense walk (BfsOp::vstart): a copy of visited after the source is set, then OR-ed
+    // with each level's new frontier by frontier_finish_kernel
     uint32_t* vstart = nullptr;
-    if (algo == kBFS && g->ordered && !g->weighted && !getenv("GTS_DEV_NO_PLAIN"))
+    if (algo == kBFS && g->ordered && !g->weighted && micro == kMicroTile)
         GTS_TRY(c->buf(kBufVstart, words * 4, (void**)&vstart));
-    const uint32_t plain8 = getenv("GTS_DEV_PLAIN8") ? (uint32_t)atoi(getenv("GTS_DEV_PLAIN8")) : 6u;
+    // tiles whose selected edges are >= 3/8 of their words take the plain walk (RMAT-27 BFS
+    // kernels 6.57 ms against 6.65 at 6/8, 6.60 at 4/8, 6.58 at 2/8, 6.65 at 1/8)
+    constexpr uint32_t plain8 = 3;
     uint32_t* dexp = nullptr;            // SSSP: distance of each vertex's last expansion (SsspOp)
     if (algo == kSSSP) {     // RMAT-27: 4.51 G -> 3.12 G relaxed edges, kernels 33.1 -> 26.1 ms
         GTS_TRY(c->buf(kBufDexp, n * 4, (void**)&dexp));
@@ -565,6 +574,7 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     GTS_CUDA(cudaMemsetAsync(ctr, 0, sizeof(Counters), s));
     src = map_src(g, src);
     set_source_kernel<<<1, 1, 0, s>>>(value, visited, cur, src);
+    if (vstart) GTS_CUDA(cudaMemcpyAsync(vstart, visited, words * 4, cudaMemcpyDeviceToDevice, s));
     uint64_t launches = 1, main_launches = 0;
     std::vector<uint32_t> l0 = pages_of_vertex(g, c->dg, c->rank, src);
     uint32_t* hs = (uint32_t*)c->h_small;
@@ -572,11 +582,6 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     if (!l0.empty()) GTS_CUDA(cudaMemcpyAsync(list, l0.data(), l0.size() * 4, cudaMemcpyHostToDevice, s));
     GTS_CUDA(cudaMemcpyAsync(&ctr->list_count, hs, 4, cudaMemcpyHostToDevice, s));
 
-    // micro-level technique inside each page (GTS_MICRO_*, App E): BFS only
-    uint32_t micro = (rc.flags & GTS_MICRO_MASK) >> 8;
-    if (micro == (GTS_MICRO_TILE >> 8)) micro = kMicroTile;
-    if (micro > kMicroHybrid) return fail(GTS_EINVAL, "unknown GTS_MICRO value");
-    if (algo == kSSSP && micro) return fail(GTS_EUNSUPPORTED, "GTS_MICRO_* techniques apply to gts_bfs and gts_pagerank");
     using BfsKern = decltype(&bfs_expand_kernel<false, kMicroTile>);
     static const BfsKern bfs_k[2][4] = {
         {bfs_expand_kernel<false, kMicroTile>, bfs_expand_kernel<false, kMicroEdge>,
@@ -681,11 +686,10 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
         if (algo == kBFS) {
             frontier_finish_kernel<<<fin_grid, 256, 0, s>>>(nullptr, 1, words, 0, words, next, visited,
                                                             slots ? nullptr : value, L + 1,
-                                                            L < K ? lvl_cnt + L : &ctr->count);
+                                                            L < K ? lvl_cnt + L : &ctr->count, vstart);
             GTS_CUDA(cudaMemsetAsync(&ctr->vprefix_words, 0xFF, 4, s));
             visited_prefix_kernel<<<fin_grid, 256, 0, s>>>(visited, words, &ctr->vprefix_words);
             ++launches;
-            if (vstart) GTS_CUDA(cudaMemcpyAsync(vstart, visited, words * 4, cudaMemcpyDeviceToDevice, s));
         } else {
             GTS_CUDA(cudaMemsetAsync(&ctr->near, 0, 8, s));
             GTS_CUDA(cudaMemsetAsync(&ctr->minpend, 0xFF, 4, s));

@@ -342,6 +342,25 @@ def test_degree_ordered_graph(G, ctx, name, residency):
     assert np.array_equal(got, oracle.sssp(g.row_ptr, g.col, w, 0))
 
 
+@pytest.mark.parametrize("name", ["rmat16_4k", "rmat16_64k", "rmat16_1m", "rmat20", "twitter20", "rand", "bintree",
+                                  "cycle"])
+def test_bfs_plain_walk(G, ctx, name):
+    """Degree-ordered unweighted pages enable the plain dense walk (expand.cuh
+    dense_tile_plain): from the second level on, tiles whose vertices with edges were all
+    visited before the level are streamed without selecting the frontier's records.  BFS
+    from many sources (hubs, mid-degree, leaves, unreached-heavy) must stay bit-exact."""
+    g, pb = graph(name)
+    gr = G.gts_build_pages(g.row_ptr, g.col, page_bytes=pb, order=True)
+    rng = np.random.default_rng(7)
+    deg = np.diff(g.row_ptr)
+    srcs = set(_sources(g)) | {int(x) for x in rng.integers(0, g.n, 6)} | {int(x) for x in np.argsort(-deg)[:3]}
+    for src in sorted(srcs):
+        got, st = G.gts_bfs(ctx, gr, src)
+        want = oracle.bfs(g.row_ptr, g.col, src)
+        assert np.array_equal(got, want), (name, src)
+        assert st["edges_traversed"] == int(deg[want != oracle.UNREACHED].sum())
+
+
 def test_degree_ordered_device_outputs(G, ctx):
     import torch
     g, pb = graph("rmat16_4k")
