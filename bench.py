@@ -592,25 +592,31 @@ def main():
     if not args.no_streamed and world == 1 and "pr" in algos and "bfs" in algos:
         peak_h2d = h2d_peak_gbs()
         ctx.evict(gr)
+        # one untimed streamed iteration first: the ring and its events are allocated on
+        # the first streamed call (a cold 2-iteration measurement read 0.68 of the link)
+        G.gts_pagerank(ctx, gr, 1, 0.85, out=pr, residency=G.GTS_STREAMED)
+        torch.cuda.synchronize()
+        SPI = 3
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        _, sp = G.gts_pagerank(ctx, gr, 2, 0.85, out=pr, residency=G.GTS_STREAMED, timing=True)
+        _, sp = G.gts_pagerank(ctx, gr, SPI, 0.85, out=pr, residency=G.GTS_STREAMED, timing=True)
         e1.record(stream)
         torch.cuda.synchronize()
-        t_pr = e0.elapsed_time(e1) * 1e-3 / 2
+        t_pr = e0.elapsed_time(e1) * 1e-3 / SPI
         e0.record(stream)
         _, sb = G.gts_bfs(ctx, gr, src, out=lv, residency=G.GTS_STREAMED, timing=True)
         e1.record(stream)
         torch.cuda.synchronize()
         t_bfs = e0.elapsed_time(e1) * 1e-3
-        link_pr = sp["h2d_bytes"] / 2 / t_pr / 1e9
+        link_pr = sp["h2d_bytes"] / SPI / t_pr / 1e9
         link_bfs = sb["h2d_bytes"] / t_bfs / 1e9
         streamed = {"pagerank_s_per_iter": t_pr, "bfs_gteps": sb["edges_traversed"] / t_bfs / 1e9, "bfs_s": t_bfs,
-                    "h2d_bytes_per_pr_iter": sp["h2d_bytes"] / 2, "h2d_bytes_bfs": sb["h2d_bytes"],
+                    "h2d_bytes_per_pr_iter": sp["h2d_bytes"] / SPI, "h2d_bytes_bfs": sb["h2d_bytes"],
                     "link_gbs_pr": link_pr, "link_gbs_bfs": link_bfs, "h2d_peak_gbs": peak_h2d,
                     "link_frac": link_pr / peak_h2d, "link_frac_bfs": link_bfs / peak_h2d,
                     "what": "GTS_STREAMED (forced): topology pages copied from pinned host memory into a 4 x 64 MiB "
-                            "device ring per iteration / level, kernels overlapped; RA/WA resident; CUDA events "
+                            "device ring per iteration / level, kernels overlapped; RA/WA resident; PageRank: 3 "
+                            "iterations after an untimed one; CUDA events "
                             "on the call stream; peak = pinned H2D of 256 MiB in this process, best of 10"}
 
     cpu = None
