@@ -58,6 +58,7 @@ struct TileSmem {
                                // dense_tile_ww reads 8-byte windows up to sel[nv + 3])
     uint32_t paytile[kTile];   // dense mode: payload of vertex t of the tile
     uint32_t tmask[kMaxTileWords];   // tiles of the current page holding a frontier vertex
+    uint32_t tplain[kMaxTileWords];  // tiles of the current page taken by the plain walk
     uint32_t off[kTile];       // word index of the first ADJLIST entry of item j
     uint32_t deg[kTile];
     uint32_t src[kTile];       // VID of item j
@@ -488,6 +489,60 @@ __device__ __forceinline__ void dense_tile_ww(const PageSet& ps, Op& op, TileSme
     }
 }
 
+// Plain-walk plan of one SP (kFastDense ops, levels with a probe floor): one pass over the
+// page's slots marks the tiles that qualify -- every vertex with edges satisfies op.done(v)
+// and has fewer entries than the floor, and the selected edges are >= op.plain8 / 8 of the
+// tile's record words -- in sm.tplain, and leaves each tile's first record word in
+// tstart[t] (tstart[ntiles] = end of the page's records) and its selected edges in tsum[t]
+// (both in sm.list, which only sparse pages use).  Runs of consecutive plain tiles are then
+// streamed as one range: no per-tile setup and one barrier per run.
+template <class Op>
+__device__ __forceinline__ void plan_plain_tiles(Op& op, TileSmem& sm, const uint8_t* data, const uint8_t* end,
+                                                 uint32_t start, uint32_t nslots, uint32_t ntiles,
+                                                 const uint32_t* fbm, uint32_t floor, uint64_t pol) {
+    const int tid = threadIdx.x, lane = tid & 31;
+    uint32_t* tsum = sm.list;
+    uint32_t* tstart = sm.list + 32 * kMaxTileWords;
+    uint32_t* tbad = sm.list + 64 * kMaxTileWords + 1;
+    for (uint32_t k = tid; k < ntiles; k += kThreads) tsum[k] = 0u;
+    for (uint32_t k = tid; k < kMaxTileWords; k += kThreads) tbad[k] = 0u;
+    __syncthreads();
+    for (uint32_t j0 = 0; j0 < nslots; j0 += kThreads) {     // uniform trip count
+        const uint32_t j = j0 + tid;
+        const bool in = j < nslots;
+        uint32_t o = 0;
+        if (in) o = ld_stream_u32(end - kSpFooter - kSlotBytes * (uint64_t)(j + 1) + 4, pol) >> 2;
+        uint32_t on = __shfl_down_sync(0xFFFFFFFFu, o, 1);
+        if (in && (lane == 31 || j + 1 == nslots)) {
+            if (j + 1 < nslots) on = ld_stream_u32(end - kSpFooter - kSlotBytes * (uint64_t)(j + 2) + 4, pol) >> 2;
+            else on = o + 1 + ld32(data + 4ull * o);             // unweighted record: header = entry count
+        }
+        const uint32_t deg = in ? on - o - 1 : 0u;
+        const uint32_t v = start + j, t = j0 / kTile;            // a warp's vertices share one tile
+        if (in && (j & (kTile - 1)) == 0) tstart[t] = o;
+        if (in && j + 1 == nslots) tstart[ntiles] = on;
+        const bool sel = in && deg > 0 && (!fbm || test_bit(fbm, v));
+        uint32_t se = sel ? deg : 0u;
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) se += __shfl_down_sync(0xFFFFFFFFu, se, d);
+        if (lane == 0 && se) atomicAdd(&tsum[t], se);
+        const bool bad = in && deg > 0 && !(deg < floor && op.done(v));
+        if (__any_sync(0xFFFFFFFFu, bad) && lane == 0) atomicOr(&tbad[t >> 5], 1u << (t & 31));
+    }
+    __syncthreads();
+    for (uint32_t k = tid; k < kMaxTileWords; k += kThreads) {
+        uint32_t m = 0;
+        for (uint32_t b = 0; b < 32; ++b) {
+            const uint32_t t = 32 * k + b;
+            if (t < ntiles && !((tbad[k] >> b) & 1u) && 8ull * tsum[t] >= (uint64_t)op.plain8 * (tstart[t + 1] - tstart[t]) &&
+                tsum[t] > 0)
+                m |= 1u << b;
+        }
+        sm.tplain[k] = m;
+    }
+    __syncthreads();
+}
+
 template <class Op, int kMicro = kMicroTile>
 __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* work_ctr) {
     const uint32_t npages = ps.d_count ? *(volatile const uint32_t*)ps.d_count : ps.count;
@@ -585,6 +640,14 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     continue;
                 }
             }
+            bool plain = false;                   // this page has a plain-walk plan (sm.tplain)
+            if constexpr (fast_dense_of<Op>::value) {
+                if (ffloor >= op.plan_floor && ntiles <= 32 * kMaxTileWords) {
+                    plan_plain_tiles(op, sm, data, end, start, nslots, ntiles, fbm, ffloor, pol);
+                    plain = true;
+                }
+            }
+            auto is_plain = [&](uint32_t t) { return plain && ((sm.tplain[t >> 5] >> (t & 31)) & 1u); };
             auto active = [&](uint32_t t) { return !fbm || ((sm.tmask[t >> 5] >> (t & 31)) & 1u); };
             auto next_active = [&](uint32_t t) {
                 while (t < ntiles && !active(t)) ++t;     // uniform: tiles without a frontier vertex cost nothing
@@ -595,6 +658,18 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             // slower on RMAT-27: BFS 7.41 vs 7.36 ms, WCC 12.84 vs 12.64 ms; the slot loads are
             // not what these kernels wait on.)
             for (uint32_t ti = next_active(0); ti < ntiles; ti = next_active(ti + 1)) {
+                if constexpr (fast_dense_of<Op>::value) {
+                    if (is_plain(ti)) {                   // uniform: a run of plain tiles, one range
+                        uint32_t tj = ti + 1, se = sm.list[ti];
+                        while (tj < ntiles && is_plain(tj)) se += sm.list[tj++];
+                        const uint32_t* tstart = sm.list + 32 * kMaxTileWords;
+                        dense_tile_plain(op, q4, tstart[ti], tstart[tj], ffloor, pol);
+                        if (tid == 0) op.plain_edges(se);
+                        __syncthreads();
+                        ti = tj - 1;
+                        continue;
+                    }
+                }
                 const uint32_t t0 = ti * kTile;
                 const uint32_t nv = min((uint32_t)kTile, nslots - t0);
                 const uint32_t v = start + t0 + tid;
@@ -630,7 +705,8 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 // interleaved (adj, w) records 33.5 vs 35.3 ms)
                 const bool dense = 8 * total >= dense_eighths<Op>() * (W1 - W0);
                 if constexpr (fast_dense_of<Op>::value) {
-                    if (ffloor && 8 * total >= op.plain8 * (W1 - W0) &&
+                    // no page plan (small floor): the same test per tile, after its setup
+                    if (!plain && ffloor && 8 * total >= op.plain8 * (W1 - W0) &&
                         __syncthreads_and((uint32_t)tid >= nv || deg == 0 || (deg < ffloor && op.done(v)))) {
                         dense_tile_plain(op, q4, W0, W1, ffloor, pol);
                         __syncthreads();

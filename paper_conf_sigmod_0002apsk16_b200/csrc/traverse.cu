@@ -51,9 +51,11 @@ struct BfsOp {
     // vertices can be streamed without selecting the frontier's records
     const uint32_t* vstart;
     uint32_t plain8;           // plain walk when the tile's selected edges are >= plain8/8 of its words
+    uint32_t plan_floor;       // whole-page plain plans from this probe floor up (per-tile tests below it)
     __device__ uint32_t fast_floor() const { return vstart ? vprefix : 0u; }
     __device__ bool done(uint32_t v) const { return test_bit(vstart, v); }
     __device__ uint32_t plain_src() const { return 0u; }
+    __device__ void plain_edges(uint32_t e) { nedges += e; }   // the frontier's edges in a plain run
     __device__ const uint32_t* frontier() const { return cur; }
     __device__ bool select(uint32_t v) { return test_bit(cur, v); }
     __device__ uint32_t payload(uint32_t, uint32_t deg) {
@@ -179,12 +181,12 @@ template <bool W, int M = kMicroTile, int MB = 2>
 __global__ void __launch_bounds__(kThreads, MB)
 bfs_expand_kernel(PageSet ps, const uint32_t* __restrict__ cur, uint32_t* visited, uint32_t* next,
                   uint32_t* work_ctr, unsigned long long* edges_out, const unsigned int* vprefix_words,
-                  uint64_t n, const uint32_t* vstart, uint32_t plain8) {
+                  uint64_t n, const uint32_t* vstart, uint32_t plain8, uint32_t plan_floor) {
     __shared__ TileSmem sm;
     // all-visited prefix from the previous level's visited_prefix_kernel (device-side,
     // so levels can be enqueued without a host round trip)
     const uint64_t vw = min((uint64_t)*vprefix_words, (n + 31) / 32);
-    BfsOp<W> op{cur, visited, next, 0ull, (uint32_t)min(vw * 32, n), vstart, plain8};
+    BfsOp<W> op{cur, visited, next, 0ull, (uint32_t)min(vw * 32, n), vstart, plain8, plan_floor};
     expand_pages<BfsOp<W>, M>(ps, op, sm, work_ctr);
     block_add_u64(op.nedges, edges_out);
 }
@@ -543,6 +545,10 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
     // tiles whose selected edges are >= 3/8 of their words take the plain walk (RMAT-27 BFS
     // kernels 6.57 ms against 6.65 at 6/8, 6.60 at 4/8, 6.58 at 2/8, 6.65 at 1/8)
     constexpr uint32_t plain8 = 3;
+    // BFS decides per tile, after the tile's own setup: whole-page plans (expand.cuh
+    // plan_plain_tiles) measured slower at every floor (RMAT-27 BFS kernels 6.53 ms per tile,
+    // 6.73-6.92 ms with plans from floors of 8 M down to 0)
+    constexpr uint32_t plan_floor = 0xFFFFFFFFu;
     uint32_t* dexp = nullptr;            // SSSP: distance of each vertex's last expansion (SsspOp)
     if (algo == kSSSP) {     // RMAT-27: 4.51 G -> 3.12 G relaxed edges, kernels 33.1 -> 26.1 ms
         GTS_TRY(c->buf(kBufDexp, n * 4, (void**)&dexp));
@@ -667,7 +673,7 @@ static int traverse_single(gts_context* c, const gts_graph* g, uint64_t src, con
                                 if (algo == kBFS) {
                                     bfs_kern<<<gl, kThreads, 0, s>>>(
                                         p2, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n,
-                                        vstart, plain8);
+                                        vstart, plain8, plan_floor);
                                 } else
                                     sssp_kern<<<gl, kThreads, 0, s>>>(
                                         p2, cur, value, next, &ctr->work, &ctr->edges, &ctr->flag, T, dexp);
@@ -1692,8 +1698,8 @@ static int betweenness(gts_context* c, const gts_graph* g, const uint64_t* sourc
                 GTS_CUDA(cudaMemsetAsync(&ctr->work, 0, 4, s));
                 std::pair<cudaEvent_t, cudaEvent_t> ev;
                 if (timing) { ev = c->t_main.next(); cudaEventRecord(ev.first, s); }
-                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, nullptr, 8u);
-                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, nullptr, 8u);
+                if (wgt) bfs_expand_kernel<true><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, nullptr, 8u, 0xFFFFFFFFu);
+                else bfs_expand_kernel<false><<<std::min(grid, cap), kThreads, 0, s>>>(ps, cur, visited, next, &ctr->work, &ctr->edges, &ctr->vprefix_words, n, nullptr, 8u, 0xFFFFFFFFu);
                 if (timing) cudaEventRecord(ev.second, s);
                 GTS_CUDA(cudaGetLastError());
                 ++main_launches;

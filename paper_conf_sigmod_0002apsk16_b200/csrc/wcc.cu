@@ -88,9 +88,11 @@ struct WccOp {
     uint32_t rstar;
     uint32_t gfloor;          // all-giant prefix (vertices); 0 = no plain walk
     uint32_t plain8;
+    uint32_t plan_floor;
     __device__ uint32_t fast_floor() const { return gbm ? gfloor : 0u; }
     __device__ bool done(uint32_t v) const { return test_bit(gbm, v); }
     __device__ uint32_t plain_src() const { return rstar; }
+    __device__ void plain_edges(uint32_t) {}
     __device__ const uint32_t* frontier() const { return nullptr; }
     __device__ bool select(uint32_t) { return true; }
     __device__ uint32_t payload(uint32_t v, uint32_t) { return __ldcg(parent + v); }
@@ -168,11 +170,11 @@ wcc_sample_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t ks,
 template <bool W, int MB = 2>
 __global__ void __launch_bounds__(kThreads, MB)
 wcc_sweep_kernel(PageSet ps, uint32_t* parent, uint32_t* work_ctr, uint32_t* changed, const uint32_t* gbm,
-                 const uint32_t* rstar, uint32_t plain8) {
+                 const uint32_t* rstar, uint32_t plain8, uint32_t wcc_plan_floor) {
     __shared__ TileSmem sm;
     // rstar[1] = first gbm word that is not all ones (wcc_giant_kernel)
     const uint32_t gfloor = gbm && plain8 <= 8 ? (uint32_t)min((uint64_t)__ldg(rstar + 1) * 32, (uint64_t)0xFFFFFFFFu) : 0u;
-    WccOp<W> op{parent, false, gbm, gbm ? __ldg(rstar) : 0u, gfloor, plain8};
+    WccOp<W> op{parent, false, gbm, gbm ? __ldg(rstar) : 0u, gfloor, plain8, wcc_plan_floor};
     expand_pages(ps, op, sm, work_ctr);
     if (__syncthreads_or(op.changed) && threadIdx.x == 0) *changed = 1u;
 }
@@ -291,6 +293,9 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     // plain walk of all-giant tiles (WccOp): every tile qualifies by its selected edges
     // (WCC selects every vertex); RMAT-27 WCC kernels 12.60 -> 10.83 ms
     constexpr uint32_t wcc_plain8 = 0u;
+    // whole-page plans (expand.cuh plan_plain_tiles): runs of all-giant tiles streamed as one
+    // range; RMAT-27 WCC kernels 9.90 ms against 10.84 deciding per tile
+    constexpr uint32_t wcc_plan_floor = 0u;
     int grid = 0;
     GTS_TRY(sms_grid(c, (const void*)sweep_k, kThreads, 0, &grid));
     uint64_t launches = L, main_launches = 0;
@@ -347,7 +352,7 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
                                     if (timing) { e2 = c->t_main.next(); cudaEventRecord(e2.first, s); }
                                     sweep_k<<<std::min(grid, cap), kThreads, 0, s>>>(
                                         ps, label[i], ctr[i], ctr[i] + 1, gbm, gbm ? gbm + (n + 31) / 32 : nullptr,
-                                        wcc_plain8);
+                                        wcc_plain8, wcc_plan_floor);
                                     if (timing) cudaEventRecord(e2.second, s);
                                     GTS_CUDA(cudaGetLastError());
                                     ++main_launches;
