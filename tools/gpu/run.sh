@@ -8,6 +8,10 @@
 #   ncu <kernel-regex> [n] [bench args]   ncu --set full of the n-th launch matching the regex
 #   sanitize <tool>           compute-sanitizer <tool> over tools/sanitize_run.py (RMAT-16, every kernel)
 #   py <script> [args]        any python script, stdout -> gpurun_out/<script basename>.out
+#   ab <pytest -k expr> <algos> <variants>   GPU tests matching the expression, then tools/kernel_ab.py
+#                             over development-switch variants ("name:ENV=V;name2:..."; "" = the build as is)
+#   ncuk <kernel-regex> <n> <algos>   ncu --set full of the n-th launch of a kernel in a bench run of <algos>
+#   microbench                tools/microbench.cu (primitive rates) -> gpurun_out/microbench.txt
 set -u
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
 O=gpurun_out
@@ -35,5 +39,19 @@ case "$what" in
   py)
     s=$1; shift
     timeout 3000 python "$s" "$@" > $O/$(basename "$s" .py).out 2>&1; echo "py rc=$?"; tail -40 $O/$(basename "$s" .py).out ;;
+  ab)
+    k=$1; algos=$2; variants=${3:-}
+    timeout 1200 python -m pytest -m gpu -x -q -k "$k" tests > $O/ab_tests.log 2>&1; echo "tests rc=$?"; tail -2 $O/ab_tests.log
+    timeout 1500 python tools/kernel_ab.py --scale ${AB_SCALE:-27} --algos $algos --reps ${AB_REPS:-5} --variants "$variants" \
+      > $O/ab.jsonl 2> $O/ab.log; echo "ab rc=$?"; cut -c1-300 $O/ab.jsonl ;;
+  ncuk)
+    k=$1; c=$2; algos=$3
+    timeout 1200 ncu --set full --clock-control none --import-source on -k "regex:$k" -s $((c - 1)) -c 1 \
+      -o $O/ncu_${k}_$c -f python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --no-streamed \
+      --algos $algos > $O/ncu_${k}_$c.log 2>&1
+    echo "ncu $k $c rc=$?" ;;
+  microbench)
+    nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/microbench tools/microbench.cu && \
+      timeout 300 /tmp/microbench > $O/microbench.txt 2>&1; echo "microbench rc=$?"; cat $O/microbench.txt ;;
   *) echo "unknown job $what"; exit 2 ;;
 esac
