@@ -59,7 +59,6 @@ struct TileSmem {
     uint32_t paytile[kTile];   // dense mode: payload of vertex t of the tile
     uint32_t tmask[kMaxTileWords];   // tiles of the current page holding a frontier vertex
     uint32_t tplain[kMaxTileWords];  // tiles of the current page taken by the plain walk
-    uint32_t fsum[3];                // per-tile plain test: selected edges (three slots, see expand_pages)
     uint32_t off[kTile];       // word index of the first ADJLIST entry of item j
     uint32_t deg[kTile];
     uint32_t src[kTile];       // VID of item j
@@ -616,10 +615,6 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             // Frontier-driven ops: one pass over the page's frontier-bitmap words marks
             // the tiles that hold a selected vertex, so inactive tiles cost nothing.
             const uint32_t* fbm = ntiles <= 32 * kMaxTileWords ? op.frontier() : nullptr;
-            if constexpr (fast_dense_of<Op>::value) {
-                if (tid < 3) sm.fsum[tid] = 0u;    // per-tile plain test slots
-                if (!fbm) __syncthreads();         // (else published by the barrier below)
-            }
             if (fbm) {
                 for (uint32_t k = tid; k < kMaxTileWords; k += kThreads) sm.tmask[k] = 0u;
                 if (tid == 0) sm.pcount = 0;
@@ -662,7 +657,6 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
             // -- cp.async.bulk + mbarrier, double-buffered, one elected thread -- measured
             // slower on RMAT-27: BFS 7.41 vs 7.36 ms, WCC 12.84 vs 12.64 ms; the slot loads are
             // not what these kernels wait on.)
-            uint32_t kt = 0;                       // tiles set up so far on this page (fsum slot)
             for (uint32_t ti = next_active(0); ti < ntiles; ti = next_active(ti + 1)) {
                 if constexpr (fast_dense_of<Op>::value) {
                     if (is_plain(ti)) {                   // uniform: a run of plain tiles, one range
@@ -691,44 +685,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                         else sm.soff[nv] = (o >> 2) + rec_hdr_words(Op::kWeighted) + (ld32(data + o) << (Op::kWeighted ? 1 : 0));
                     }
                 }
-                if constexpr (fast_dense_of<Op>::value) {
-                    // per-tile plain test fused into the barrier that publishes soff: degrees from
-                    // the neighbouring slot (shuffle; lane 31 and the tile's last vertex load it),
-                    // the selected edges summed into fsum[kt % 3] (slot kt+1 is cleared here: its
-                    // last readers passed this barrier's predecessor), qualification by count
-                    if (!plain && ffloor) {
-                        const int lane = tid & 31;
-                        uint32_t o = (uint32_t)tid < nv ? sm.soff[tid] : 0u;
-                        uint32_t on = __shfl_down_sync(0xFFFFFFFFu, o, 1);
-                        if ((uint32_t)tid < nv && (lane == 31 || (uint32_t)tid == nv - 1)) {
-                            const uint32_t j = t0 + tid;
-                            if (j + 1 < nslots) on = ld_stream_u32(end - kSpFooter - kSlotBytes * (uint64_t)(j + 2) + 4, pol) >> 2;
-                            else on = o + 1 + ld32(data + 4ull * o);
-                        }
-                        const uint32_t dg = (uint32_t)tid < nv ? on - o - 1 : 0u;
-                        const bool harmless = dg == 0 || (dg < ffloor && op.done(v));
-                        uint32_t se = sel ? dg : 0u;
-#pragma unroll
-                        for (int d = 16; d > 0; d >>= 1) se += __shfl_down_sync(0xFFFFFFFFu, se, d);
-                        if (lane == 0 && se) atomicAdd(&sm.fsum[kt % 3], se);
-                        if (tid == 0) sm.fsum[(kt + 1) % 3] = 0u;
-                        const int hc = __syncthreads_count(harmless);     // (also publishes soff)
-                        const uint32_t tot = sm.fsum[kt % 3];
-                        ++kt;
-                        if (tot == 0 && !__syncthreads_or(sel)) continue;  // nothing selected with edges
-                        const uint32_t W0 = sm.soff[0], W1 = sm.soff[nv];
-                        if (hc == kThreads && tot > 0 && 8ull * tot >= (uint64_t)op.plain8 * (W1 - W0)) {
-                            dense_tile_plain(op, q4, W0, W1, ffloor, pol);
-                            if (tid == 0) op.plain_edges(tot);
-                            __syncthreads();
-                            continue;
-                        }
-                    } else if (!__syncthreads_or(sel)) {
-                        continue;                         // (also publishes soff)
-                    }
-                } else {
-                    if (!__syncthreads_or(sel)) continue;   // (also publishes soff)
-                }
+                if (!__syncthreads_or(sel)) continue;   // (also publishes soff)
                 uint32_t deg = 0;
                 if ((uint32_t)tid < nv)
                     deg = (sm.soff[tid + 1] - sm.soff[tid] - rec_hdr_words(Op::kWeighted)) >> (Op::kWeighted ? 1 : 0);
@@ -747,6 +704,15 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 // 35.7 ms vs 42.8 ms when the selected words are counted instead; with the
                 // interleaved (adj, w) records 33.5 vs 35.3 ms)
                 const bool dense = 8 * total >= dense_eighths<Op>() * (W1 - W0);
+                if constexpr (fast_dense_of<Op>::value) {
+                    // no page plan (small floor): the same test per tile, after its setup
+                    if (!plain && ffloor && 8 * total >= op.plain8 * (W1 - W0) &&
+                        __syncthreads_and((uint32_t)tid >= nv || deg == 0 || (deg < ffloor && op.done(v)))) {
+                        dense_tile_plain(op, q4, W0, W1, ffloor, pol);
+                        __syncthreads();
+                        continue;
+                    }
+                }
                 if (dense) {
                     // dense tile, warp-window walk: each warp streams a contiguous run of
                     // 128-word windows; owners from record-start masks (no binary search;
