@@ -12,6 +12,8 @@
 #                             over development-switch variants ("name:ENV=V;name2:..."; "" = the build as is)
 #   ncuk <kernel-regex> <n> <algos>   ncu --set full of the n-th launch of a kernel in a bench run of <algos>
 #   microbench                tools/microbench.cu (primitive rates) -> gpurun_out/microbench.txt
+#   abso <algos> <alt.so>...  compile-time A/B: tools/kernel_ab.py with the in-tree libgts.so, then with
+#                             each alternative build swapped in (the in-tree library is restored after)
 set -u
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
 O=gpurun_out
@@ -53,5 +55,16 @@ case "$what" in
   microbench)
     nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/microbench tools/microbench.cu && \
       timeout 300 /tmp/microbench > $O/microbench.txt 2>&1; echo "microbench rc=$?"; cat $O/microbench.txt ;;
+  abso)
+    algos=$1; shift
+    L=paper_conf_sigmod_0002apsk16_b200/lib/libgts.so
+    cp $L /tmp/libgts_base.so
+    for so in base "$@"; do
+      [ "$so" != base ] && cp "$so" $L
+      timeout 1500 python tools/kernel_ab.py --scale ${AB_SCALE:-27} --algos $algos --reps ${AB_REPS:-5} \
+        --tag "$(basename $so)" >> $O/abso.jsonl 2>> $O/abso.log; echo "ab $so rc=$?"
+      cp /tmp/libgts_base.so $L
+    done
+    cut -c1-260 $O/abso.jsonl ;;
   *) echo "unknown job $what"; exit 2 ;;
 esac
