@@ -312,7 +312,9 @@ __device__ void expand_sparse_page(const PageSet& ps, Op& op, TileSmem& sm, cons
             if (tid == 0) sm.pre[nf] = total;
             __syncthreads();
             gather_items(ps, op, sm, words, nf, total, pol);
-            __syncthreads();
+            // no barrier here: the gather reads only the item arrays, and the next batch
+            // rewrites them only after its tile_scan barriers, which every thread reaches
+            // after finishing this gather
         }
     }
 }
@@ -709,8 +711,7 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                     if (!plain && ffloor && 8 * total >= op.plain8 * (W1 - W0) &&
                         __syncthreads_and((uint32_t)tid >= nv || deg == 0 || (deg < ffloor && op.done(v)))) {
                         dense_tile_plain(op, q4, W0, W1, ffloor, pol);
-                        __syncthreads();
-                        continue;
+                        continue;           // (the plain walk reads no shared memory: no barrier)
                     }
                 }
                 if (dense) {
@@ -736,7 +737,8 @@ __device__ void expand_pages(const PageSet& ps, Op& op, TileSmem& sm, uint32_t* 
                 if (tid == 0) sm.pre[nf] = total;
                 __syncthreads();
                 gather_items(ps, op, sm, words, nf, total, pol);
-                __syncthreads();
+                // (no trailing barrier: the next tile rewrites the item arrays only after its
+                // own tile_scan barriers; its soff / sel / paytile writes are not read here)
             }
         }
         op.end_page();
