@@ -292,7 +292,9 @@ extern "C" int gts_wcc(gts_context* c, const gts_graph* g, const gts_run_config*
     auto sweep_k = g->weighted ? wcc_sweep_kernel<true, 3> : wcc_sweep_kernel<false, 3>;
     // plain walk of all-giant tiles (WccOp): every tile qualifies by its selected edges
     // (WCC selects every vertex); RMAT-27 WCC kernels 12.60 -> 10.83 ms
-    constexpr uint32_t wcc_plain8 = 0u;
+    // (degree-ordered pages only: in natural VID order the all-giant prefix is a few
+    // vertices, no tile qualifies, and the plan would be pure overhead; 9 = off)
+    const uint32_t wcc_plain8 = g->ordered ? 0u : 9u;
     // whole-page plans (expand.cuh plan_plain_tiles): runs of all-giant tiles streamed as one
     // range; RMAT-27 WCC kernels 9.90 ms against 10.84 deciding per tile
     constexpr uint32_t wcc_plan_floor = 0u;
