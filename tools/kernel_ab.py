@@ -22,6 +22,8 @@ ap.add_argument("--scale", type=int, default=27)
 ap.add_argument("--reps", type=int, default=3)
 ap.add_argument("--algos", default="pr,bfs,sssp,wcc")
 ap.add_argument("--tag", default="")
+ap.add_argument("--tunes", default="",
+                help='gts_run_config tuning variants (gts.TUNABLE fields): "name:field=v,field2=w;name2:..."')
 ap.add_argument("--variants", default="",
                 help='A/B of development switches read by libgts at call time: "name:ENV=V,ENV2=W;name2:..."')
 a = ap.parse_args()
@@ -44,7 +46,12 @@ n = g.n
 dev_u = torch.empty(n, dtype=torch.int32, device="cuda")
 dev_f = torch.empty(n, dtype=torch.float32, device="cuda")
 variants = [v.partition(":") for v in a.variants.split(";")] if a.variants else [(a.tag, "", "")]
-for tag, _, envs in variants:
+tunes = [t.partition(":") for t in a.tunes.split(";")] if a.tunes else []
+# every tuning variant runs with the build as is (no environment switches)
+variants = [(tag, "", "", {}) for tag, _, envs in variants if not envs] + \
+           [(tag, "", envs, {}) for tag, _, envs in variants if envs] + \
+           [(tag, "", "", dict(kv.split("=") for kv in filter(None, tv.split(",")))) for tag, _, tv in tunes]
+for tag, _, envs, tune in variants:
     keys = []
     for kv in filter(None, envs.split(",")):
         k, v = kv.split("=")
@@ -54,13 +61,13 @@ for tag, _, envs in variants:
         ks, cs, st = [], [], None
         for _ in range(a.reps + 1):
             if al == "pr":
-                _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=dev_f, timing=True)
+                _, st = G.gts_pagerank(ctx, gr, 10, 0.85, out=dev_f, timing=True, tune=tune)
             elif al == "bfs":
-                _, st = G.gts_bfs(ctx, gr, 0, out=dev_u, timing=True)
+                _, st = G.gts_bfs(ctx, gr, 0, out=dev_u, timing=True, tune=tune)
             elif al == "sssp":
-                _, st = G.gts_sssp(ctx, grw, 0, out=dev_u, timing=True)
+                _, st = G.gts_sssp(ctx, grw, 0, out=dev_u, timing=True, tune=tune)
             else:
-                _, st = G.gts_wcc(ctx, gr, out=dev_u, timing=True)
+                _, st = G.gts_wcc(ctx, gr, out=dev_u, timing=True, tune=tune)
             ks.append(st["main_kernel_s"])
             cs.append(st["wall_s"])
         ks, cs = sorted(ks[1:]), sorted(cs[1:])
