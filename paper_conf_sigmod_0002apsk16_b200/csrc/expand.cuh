@@ -176,6 +176,10 @@ struct sparse_select_of<Op, std::void_t<decltype(Op::kSparseSelect)>> : std::int
 // and source alike).  An unweighted record's header is its entry count,
 // so when every record of the tile has fewer entries than the floor the headers are
 // filtered out with the rest and no record-start mask is needed either.
+// Members such an op provides: uint32_t fast_floor() (0 = no plain walk this launch),
+// bool done(v), uint32_t plain_src(), void plain_edges(selected edges of a planned run),
+// uint32_t plain8 (qualifying share of selected edges, in eighths of the tile's words)
+// and uint32_t plan_floor (whole-page plans from this floor up, see plan_plain_tiles).
 template <class Op, class = void>
 struct fast_dense_of : std::false_type {};
 template <class Op>
