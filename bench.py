@@ -22,8 +22,10 @@ import argparse
 import gc
 import json
 import os
+import shutil
 import subprocess
 import sys
+import tempfile
 import threading
 import time
 
@@ -312,14 +314,25 @@ def make_graph(args, rank, world, dist):
     gen = (lambda: inputs.rmat(args.scale)) if args.workload == "rmat" else inputs.twitter_like
     if world == 1:
         return gen()
-    tag = f"/dev/shm/gts_bench_{args.workload}_{args.scale}_{os.environ.get('MASTER_PORT', '0')}"
+    obj = [None]
     if rank == 0:
         g = gen()
+        # /dev/shm when it has room for the CSR (a container's default is 64 MB), else the temp dir
+        need = g.row_ptr.nbytes + g.col.nbytes + (1 << 30)
+        base = "/dev/shm"
+        try:
+            if shutil.disk_usage(base).free < need:
+                base = tempfile.gettempdir()
+        except OSError:
+            base = tempfile.gettempdir()
+        tag = os.path.join(base, f"gts_bench_{args.workload}_{args.scale}_{os.environ.get('MASTER_PORT', '0')}")
         np.save(tag + "_rp.npy", g.row_ptr)
         np.save(tag + "_col.npy", g.col)
-    dist.barrier()
+        obj = [tag]
+    dist.broadcast_object_list(obj, src=0)
+    args._shared_tag = obj[0]
     if rank != 0:
-        g = inputs.CSR(np.load(tag + "_rp.npy", mmap_mode="r"), np.load(tag + "_col.npy", mmap_mode="r"))
+        g = inputs.CSR(np.load(obj[0] + "_rp.npy", mmap_mode="r"), np.load(obj[0] + "_col.npy", mmap_mode="r"))
     return g
 
 
@@ -327,10 +340,9 @@ def drop_shared_graph(args, rank, world, dist):
     if world > 1:
         dist.barrier()
         if rank == 0:
-            tag = f"/dev/shm/gts_bench_{args.workload}_{args.scale}_{os.environ.get('MASTER_PORT', '0')}"
             for suf in ("_rp.npy", "_col.npy"):
                 try:
-                    os.remove(tag + suf)
+                    os.remove(args._shared_tag + suf)
                 except OSError:
                     pass
 
