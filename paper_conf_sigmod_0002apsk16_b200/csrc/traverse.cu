@@ -264,6 +264,12 @@ __global__ void sssp_finish_kernel(const uint32_t* __restrict__ gathered, int wo
         } else {
             bits = next[w];
         }
+        if (T == 0xFFFFFFFEu) {          // unbounded bucket: every pending distance is within T
+            if (gathered) next[w] = bits;
+            c += __popc(bits);
+            nr += __popc(bits);
+            continue;
+        }
         uint32_t keep = cur[w] & ~bits;
         while (keep) {
             const int b = __ffs(keep) - 1;
