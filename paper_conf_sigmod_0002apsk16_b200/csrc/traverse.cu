@@ -383,17 +383,20 @@ __global__ void level_fill4_kernel(uint8_t* lv4, const uint32_t* __restrict__ sl
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; w < words; w += stride) {
         const LevelPlanes lp = level_planes(slots, nlev, words, w);
+        // bit b of plane k becomes bit k of nibble b: spread each byte of a plane to every
+        // fourth bit (bit i -> bit 4i) and shift it into place; unreached nibbles are 0xF
+        auto spread = [](uint32_t x) {         // 8 bits -> bits 0, 4, ..., 28
+            x = (x | (x << 12)) & 0x000F000Fu;
+            x = (x | (x << 6)) & 0x03030303u;
+            return (x | (x << 3)) & 0x11111111u;
+        };
         uint32_t e[4];
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
-            uint32_t x = 0;
-#pragma unroll
-            for (int k = 0; k < 8; ++k) {
-                const int b = 8 * q + k;
-                const uint32_t l = ((lp.reached >> b) & 1u) ? level_of_bit(lp, b) : 0xFu;
-                x |= l << (4 * k);
-            }
-            e[q] = x;
+            const int sh = 8 * q;
+            e[q] = spread((lp.p[0] >> sh) & 0xFFu) | spread((lp.p[1] >> sh) & 0xFFu) << 1 |
+                   spread((lp.p[2] >> sh) & 0xFFu) << 2 | spread((lp.p[3] >> sh) & 0xFFu) << 3 |
+                   spread(~(lp.reached >> sh) & 0xFFu) * 0xFu;
         }
         reinterpret_cast<uint4*>(lv4)[w] = make_uint4(e[0], e[1], e[2], e[3]);
     }
